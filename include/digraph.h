@@ -1,0 +1,220 @@
+/*
+ * digraph.h -- C ABI of the B200-native DiGraph hot path.
+ *
+ * DiGraph (Zhang et al., ASPLOS'19; /root/reference/PAPER.md) processes an
+ * iterative directed-graph algorithm by splitting the graph into disjoint
+ * directed paths and propagating vertex states along each path inside one
+ * round ("path-based asynchronous execution", sec. 3.1, lines
+ * 88-102).  This header is the boundary between the (thin) Python binding and
+ * the native library libdigraph.so: plain C types, plain pointers and sizes.
+ *
+ * Conventions (all functions):
+ *   - return 0 on success, a negative DG_E* code on failure; the message of
+ *     the last failure on the calling thread is dg_last_error();
+ *   - no function falls back to the CPU for a computation step: when the
+ *     CUDA device or the kernels are unavailable the call fails with
+ *     DG_ENOCUDA;
+ *   - pointers documented as HOST are ordinary host memory (pageable or
+ *     pinned) and are only read/written during the call; DEVICE pointers
+ *     are CUDA device pointers on the graph's device;
+ *   - the library never takes ownership of caller memory.
+ *
+ * Lifecycle: dg_create -> dg_load_csr -> dg_build_paths -> (dg_run ->
+ * dg_get_states)* -> dg_destroy.
+ */
+#ifndef DIGRAPH_H
+#define DIGRAPH_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define DG_OK 0
+#define DG_EINVAL (-1)   /* bad argument / wrong lifecycle order            */
+#define DG_ENOMEM (-2)   /* host or device allocation failed                */
+#define DG_ENOCUDA (-3)  /* no CUDA device / kernel launch failed           */
+#define DG_ENOCONV (-4)  /* max_rounds reached before convergence           */
+
+/* Unreachable vertex distance for SSSP/BFS (reading R-INF). */
+#define DG_INF 0x7FFFFFFFu
+
+/* Algorithms (sec. 4 benchmarks + BASELINE.json north_star). */
+typedef enum {
+    DG_SSSP = 0,       /* min-plus relaxation, integer weights >= 0           */
+    DG_BFS = 1,        /* SSSP with unit weights                              */
+    DG_PAGERANK = 2,   /* delta-accumulative PageRank, d = `param`           */
+    DG_WCC = 3,        /* min-label propagation over both edge directions     */
+    DG_SCC = 4,        /* forward colouring + backward reachability rounds    */
+    DG_ADSORPTION = 5  /* accumulative Adsorption (dg_set_vertex_params)      */
+} dg_algo;
+
+/* Execution model. */
+typedef enum {
+    DG_MODE_PATH = 0,    /* DiGraph path-based asynchronous model (the product) */
+    DG_MODE_VERTEX = 1   /* vertex-centric frontier kernel (ablation baseline)  */
+} dg_mode;
+
+typedef struct dg_graph dg_graph;
+
+/* Parameters of the preprocessing rows (sec. 3.2.1, 3.2.3). */
+typedef struct {
+    int32_t d_max;         /* DFS depth bound D_MAX of Algorithm 1 (line 3); paper default 16 */
+    int32_t l_merge;       /* max edges of a merged path (reading R-MERGE); 0 = no merge */
+    int32_t n_sub;         /* number of subgraphs Algorithm 1 runs on in parallel (line 114) */
+    int32_t order;         /* successor/root order: 0 = degree desc (line 5), 1 = vertex id */
+    float hot_factor;      /* hot path iff avg degree >= hot_factor * mean degree (R-HOT) */
+    int32_t part_entries;  /* target path entries per partition (scheduling unit) */
+    int32_t rank;          /* this process's rank for multi-GPU path partitioning */
+    int32_t world;         /* number of ranks (1 = single GPU) */
+} dg_path_params;
+
+/* Fill *p with the defaults (d_max 16, l_merge 64, n_sub 64, order 0,
+ * hot_factor 2, part_entries 2048, rank 0, world 1). */
+void dg_default_params(dg_path_params *p);
+
+/* Statistics of one dg_run (device-side counters). */
+typedef struct {
+    double time_ms;               /* device time of the run (CUDA events)          */
+    int64_t rounds;               /* rounds until the active counter reached zero  */
+    int64_t vertex_updates;       /* master-state changes (successful relax/fold)  */
+    int64_t edges_processed;      /* path edges (or CSR edges) walked              */
+    int64_t units_processed;      /* partitions (path) / vertices (vertex) dispatched */
+    int64_t kernel_launches;      /* kernels launched by this run                  */
+    int64_t outer_iterations;     /* SCC colouring iterations (0 otherwise)        */
+} dg_run_stats;
+
+/* Static description of the built layout (sizes; for tests and benchmarks). */
+typedef struct {
+    int64_t n, m;                 /* vertices, edges                                */
+    int64_t n_paths;              /* paths after merging (this rank)                */
+    int64_t n_entries;            /* path entries = sum(len+1) (this rank)          */
+    int64_t n_partitions;         /* partitions (this rank)                         */
+    int64_t n_hot_paths;          /* hot paths (this rank)                          */
+    int64_t n_layers;             /* layers of the DAG sketch                       */
+    int64_t n_dep_sccs;           /* SCCs of the path dependency graph containing paths */
+    int64_t giant_scc_paths;      /* paths in the largest dependency SCC            */
+    int64_t n_boundary;           /* vertices replicated on >1 rank                 */
+    int64_t paths_before_merge;   /* paths produced by Algorithm 1                  */
+    double preprocess_ms;         /* host time of dg_build_paths                    */
+    int64_t device_bytes;         /* device memory held by the layout               */
+} dg_layout_info;
+
+/* Create an empty graph bound to CUDA device `device` (cudaSetDevice is
+ * called on entry of every function).  *out receives the handle. */
+int dg_create(dg_graph **out, int device);
+
+/* Destroy a graph and free all host and device memory it holds. */
+void dg_destroy(dg_graph *g);
+
+/* Thread-local message of the last failure ("" if none). */
+const char *dg_last_error(void);
+
+/* Load a directed graph in CSR form (sec. 3.1: G = (V, E)).
+ *   n        number of vertices (ids 0..n-1, n < 2^30)
+ *   m        number of directed edges
+ *   row_ptr  HOST int64[n+1], non-decreasing, row_ptr[0] = 0, row_ptr[n] = m
+ *   col      HOST int32[m], destination of edge k (source = the row)
+ *   weight   HOST int32[m] edge weights (>= 0) or NULL (all weights 1)
+ * The arrays are copied (host copy for preprocessing, device copy for the
+ * vertex-centric ablation).  Invalidates a previous layout. */
+int dg_load_csr(dg_graph *g, int64_t n, int64_t m, const int64_t *row_ptr,
+                const int32_t *col, const int32_t *weight);
+
+/* Build the path layout on the host (C++, OpenMP; no device needed):
+ * Algorithm 1 path decomposition, short-path
+ * merging (line 157), hot/cold classification (line 112), path dependency
+ * graph + Tarjan SCC condensation + layering (lines 98-102, 159, 169),
+ * priority order Pri(p) (line 192), partitions (line 161/163) and, when
+ * p->world > 1, the partitions owned by p->rank plus the boundary-vertex set
+ * ("state synchronization of vertex replicas").
+ * p may be NULL (defaults). */
+int dg_build_paths(dg_graph *g, const dg_path_params *p);
+
+/* Copy the host CSR and the built layout to the device (the H2D part of an
+ * end-to-end run).  dg_run / dg_run_begin / dg_set_vertex_params call it
+ * implicitly when the layout is not on the device yet.  Fails with
+ * DG_ENOCUDA when no CUDA device is present. */
+int dg_upload(dg_graph *g);
+
+/* Per-vertex inputs of Adsorption (reading R-ADS):
+ *   p_inj, p_cont, inj  HOST double[n]; x_v = p_inj*inj + sum p_cont(u) w(u,v)/W(u) x_u.
+ * Must be called before dg_run(DG_ADSORPTION). */
+int dg_set_vertex_params(dg_graph *g, const double *p_inj, const double *p_cont,
+                         const double *inj);
+
+/* Run `algo` to convergence on the device.
+ *   source   SSSP/BFS source vertex (ignored otherwise)
+ *   epsilon  PageRank/Adsorption per-vertex stop threshold on the delta
+ *            (north_star: 1e-7 with unnormalised ranks (1-d) + d*sum);
+ *            ignored by the exact algorithms
+ *   param    PageRank damping d (0 < d < 1); ignored otherwise
+ *   mode     DG_MODE_PATH or DG_MODE_VERTEX (ablation)
+ *   max_rounds  safety cap (<= 0: 1,000,000)
+ *   stats    may be NULL
+ * States stay on the device until dg_get_states.  Single-rank only: with
+ * world > 1 use dg_rounds / dg_boundary_* (multi-GPU protocol). */
+int dg_run(dg_graph *g, int algo, int64_t source, double epsilon, double param,
+           int mode, int64_t max_rounds, dg_run_stats *stats);
+
+/* Copy the final states of the last dg_run into `out` (n elements):
+ *   SSSP/BFS      uint32 distances (DG_INF unreachable)
+ *   PAGERANK      float32 ranks normalised to sum 1 (reading R-PR)
+ *   ADSORPTION    float32 scores x_v
+ *   WCC / SCC     int32 label = smallest vertex id of the component
+ *   out_is_device 0: `out` is HOST memory; 1: DEVICE memory. */
+int dg_get_states(dg_graph *g, void *out, int64_t n, int out_is_device);
+
+/* Layout sizes / preprocessing time. */
+int dg_get_layout_info(const dg_graph *g, dg_layout_info *info);
+
+/* Export the built paths (this rank, priority order) for validation:
+ *   path_off  HOST int64[n_paths+1] (may be NULL to query only)
+ *   vertices  HOST int32[n_entries]: vertices of each path in path order
+ *   layer     HOST int32[n_paths] layer number L(p) (may be NULL)
+ *   scc       HOST int64[n_paths] canonical SCC label: smallest merged-order
+ *             index of a path in the same dependency SCC (may be NULL)
+ *   merged_index HOST int64[n_paths] index of the path in merge order (may be NULL)
+ *   hot       HOST uint8[n_paths] hot flag (may be NULL)
+ *   part_off  HOST int64[n_partitions+1] partition -> entry offsets (may be NULL) */
+int dg_export_paths(const dg_graph *g, int64_t *path_off, int32_t *vertices, int32_t *layer,
+                    int64_t *scc, int64_t *merged_index, uint8_t *hot, int64_t *part_off);
+
+/* ---- multi-GPU protocol (one process per GPU; PyTorch/NCCL moves bytes) ----
+ * A run is: dg_round_begin, then repeat { dg_rounds (local rounds until the
+ * local active counter is zero or max_rounds); dg_boundary_pack;
+ * all-reduce the buffer across ranks (MIN for SSSP/BFS/WCC, SUM for
+ * PageRank/Adsorption); dg_boundary_unpack } until the all-reduced active
+ * count is zero; dg_run_end. */
+
+/* Number of boundary vertices and the buffer element type of this rank:
+ * *elem_bytes = 4 (uint32 for MIN algorithms, float32 for SUM algorithms). */
+int dg_boundary_size(const dg_graph *g, int64_t *n_boundary);
+
+/* Export the boundary vertex ids (HOST int32[n_boundary], ascending). */
+int dg_boundary_vertices(const dg_graph *g, int32_t *out);
+
+/* Start a multi-round run (resets states as dg_run does). */
+int dg_run_begin(dg_graph *g, int algo, int64_t source, double epsilon, double param);
+
+/* Run up to max_rounds local rounds; *active = partitions still active. */
+int dg_rounds(dg_graph *g, int64_t max_rounds, int64_t *active);
+
+/* Pack boundary states into DEVICE buffer `buf` (n_boundary x 4 bytes):
+ * MIN algorithms: the current states; SUM algorithms: the increments since
+ * the last unpack ("each mirror always sends its new state
+ * to its master"). */
+int dg_boundary_pack(dg_graph *g, void *buf);
+
+/* Apply the all-reduced DEVICE buffer; vertices whose state changed
+ * re-activate their partitions.  *active = partitions activated. */
+int dg_boundary_unpack(dg_graph *g, const void *buf, int64_t *active);
+
+/* Finish the run: normalisation (PageRank) and statistics. */
+int dg_run_end(dg_graph *g, dg_run_stats *stats);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DIGRAPH_H */

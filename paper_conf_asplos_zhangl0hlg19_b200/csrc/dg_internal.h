@@ -1,0 +1,94 @@
+// Internal declarations shared by the host preprocessing (dg_host.cpp) and
+// the CUDA kernels (dg_kernels.cu).  Not part of the public ABI.
+#pragma once
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/digraph.h"
+
+namespace dg {
+
+// Path entry encoding in e_idx (uint32): vertex id in bits 0..29,
+// bit 31 = first vertex of a path (head), bit 30 = last vertex (tail).
+constexpr uint32_t kHead = 0x80000000u;
+constexpr uint32_t kTail = 0x40000000u;
+constexpr uint32_t kVMask = 0x3FFFFFFFu;
+
+struct HostCSR {
+    int64_t n = 0, m = 0;
+    std::vector<int64_t> row_ptr;
+    std::vector<int32_t> col, w;
+    bool has_w = false;
+    std::vector<int32_t> indeg, outdeg;
+};
+
+// Host copy of the built layout (one rank's share).
+struct HostLayout {
+    bool built = false;
+    dg_path_params params{};
+    // paths of this rank in priority order
+    std::vector<int64_t> path_off;      // n_paths+1, into entries
+    std::vector<int32_t> layer;         // per path
+    std::vector<int64_t> scc;           // canonical dependency-SCC label per path
+    std::vector<int64_t> merged_index;  // merge-order index per path
+    std::vector<uint8_t> hot;           // per path
+    // entries
+    std::vector<uint32_t> e_idx;        // vertex | head | tail
+    std::vector<int32_t> e_w;           // weight of the path edge INTO this entry (0 at heads)
+    std::vector<int64_t> part_off;      // n_part+1
+    // vertex -> partitions maps
+    std::vector<int64_t> vsrc_ptr;  std::vector<int32_t> vsrc;   // non-tail occurrences
+    std::vector<int64_t> vdst_ptr;  std::vector<int32_t> vdst;   // non-head occurrences
+    // multi-rank
+    std::vector<int32_t> boundary;      // vertices present on >1 rank (ascending)
+    // stats
+    int64_t n_layers = 0, n_dep_sccs = 0, giant = 0, paths_before_merge = 0, n_hot = 0;
+    double preprocess_ms = 0;
+};
+
+void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L);
+
+// ---------------- device side ----------------
+struct DevLayout {
+    int64_t n = 0, m = 0, M = 0, n_part = 0, n_bnd = 0;
+    uint32_t* e_idx = nullptr;
+    int32_t* e_w = nullptr;
+    int64_t* part_off = nullptr;
+    int64_t* vsrc_ptr = nullptr; int32_t* vsrc = nullptr;
+    int64_t* vdst_ptr = nullptr; int32_t* vdst = nullptr;
+    int32_t* bnd = nullptr;
+    // CSR (for the vertex-centric ablation and per-vertex coefficients)
+    int64_t* row_ptr = nullptr; int32_t* col = nullptr; int32_t* w = nullptr;
+    int32_t* outdeg = nullptr;
+    int64_t bytes = 0;
+};
+
+struct DevWork;  // defined in dg_kernels.cu
+
+struct RunState {
+    int algo = -1, mode = 0;
+    int64_t source = 0;
+    double eps = 0, param = 0;
+    int64_t round = 0;
+    dg_run_stats stats{};
+};
+
+// Kernel-side entry points (dg_kernels.cu).  All return 0 or DG_E*.
+int dev_select(int device, std::string& err);
+int dev_upload_csr(DevLayout& D, const HostCSR& g, std::string& err);
+int dev_upload_layout(DevLayout& D, const HostLayout& L, std::string& err);
+void dev_free_layout(DevLayout& D, bool csr_too);
+int dev_set_vertex_params(DevWork*& W, const DevLayout& D, const double* p_inj, const double* p_cont,
+                          const double* inj, std::string& err);
+int dev_run(DevWork*& W, const DevLayout& D, RunState& S, int64_t max_rounds, std::string& err);
+int dev_run_begin(DevWork*& W, const DevLayout& D, RunState& S, std::string& err);
+int dev_rounds(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, int64_t* active, std::string& err);
+int dev_boundary_pack(DevWork* W, const DevLayout& D, RunState& S, void* buf, std::string& err);
+int dev_boundary_unpack(DevWork* W, const DevLayout& D, RunState& S, const void* buf, int64_t* active, std::string& err);
+int dev_run_end(DevWork* W, const DevLayout& D, RunState& S, std::string& err);
+int dev_get_states(DevWork* W, const DevLayout& D, const RunState& S, void* out, int64_t n, int out_is_device,
+                   std::string& err);
+void dev_free_work(DevWork*& W);
+
+}  // namespace dg

@@ -1,0 +1,423 @@
+// Host-side preprocessing rows of DiGraph (sec. 3.2.1 / 3.2.3):
+//   (1) Algorithm 1 path decomposition per subgraph (OpenMP), short-path
+//       merging, hot/cold classification;
+//   (2) path dependency graph, Tarjan SCC condensation (DAG sketch),
+//       layering, priority Pri(p), partitions and vertex->partition maps;
+//   (5) multi-rank path partitioning and the boundary (replica) vertex set.
+// Deterministic for a given dg_path_params (independent of the number of
+// OpenMP threads): subgraph outputs are concatenated in subgraph order.
+#include <omp.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cstring>
+#include <numeric>
+#include <stdexcept>
+
+#include "dg_internal.h"
+
+namespace dg {
+namespace {
+
+struct SubOut {
+    std::vector<int32_t> pv;     // path vertices, concatenated
+    std::vector<int32_t> pw;     // weight of the edge into each path vertex (0 at heads)
+    std::vector<int64_t> start;  // path starts into pv (+ final size)
+};
+
+// ---------------------------------------------------------------------------
+// Algorithm 1 on one subgraph [lo, hi).
+// An expansion of v visits *all* of v's local edges (the for loop of lines
+// 6-17 runs to completion and only expansions of v visit v's edges), so
+// "v has unvisited local edges" == "v is local, has out-edges and was never
+// expanded"; no per-edge visited flags are needed.
+// ---------------------------------------------------------------------------
+struct Decomposer {
+    const HostCSR& g;
+    const std::vector<int32_t>& scol;   // successors of each row, sorted (line 5)
+    const std::vector<int32_t>& sw;     // their weights
+    const std::vector<int64_t>& deg;
+    std::vector<uint8_t>& expanded;     // global, disjoint per subgraph
+    std::vector<uint8_t>& inner;        // global (line 13), benign byte races
+    std::vector<uint32_t>& visited;     // per thread, stamp = subgraph id + 1
+    uint32_t stamp;
+    int64_t lo, hi;
+    int d_max;
+    SubOut& out;
+    bool open = false;
+
+    void new_path() {  // lines 14 / 19: close the current path
+        if (open) { out.start.push_back((int64_t)out.pv.size()); open = false; }
+    }
+    void insert(int32_t u, int32_t v, int32_t w) {  // line 9
+        if (!open) { out.pv.push_back(u); out.pw.push_back(0); open = true; }
+        out.pv.push_back(v); out.pw.push_back(w);
+    }
+    bool has_unvisited(int64_t v) const {
+        return v >= lo && v < hi && !expanded[v] && g.row_ptr[v + 1] > g.row_ptr[v];
+    }
+    void graphp(int32_t v_root, int d) {
+        visited[v_root] = stamp;                                    // line 2
+        if (has_unvisited(v_root) && d < d_max) {                   // line 3
+            expanded[v_root] = 1;
+            for (int64_t e = g.row_ptr[v_root]; e < g.row_ptr[v_root + 1]; e++) {  // lines 4-6
+                int32_t v = scol[e];
+                insert(v_root, v, sw[e]);                           // lines 7-9
+                if (visited[v] != stamp) {                          // line 10
+                    graphp(v, d + 1);                               // line 11
+                } else {
+                    __atomic_store_n(&inner[v], (uint8_t)1, __ATOMIC_RELAXED);  // line 13
+                    new_path();                                     // line 14
+                }
+            }
+        } else {
+            new_path();                                             // line 19
+        }
+    }
+};
+
+// Iterative Tarjan over a CSR graph; comp[v] = SCC id in completion order
+// (reverse topological order of the condensation).
+int64_t tarjan(int64_t N, const std::vector<int64_t>& ptr, const std::vector<int64_t>& adj,
+               std::vector<int64_t>& comp) {
+    std::vector<int64_t> index(N, -1), low(N, 0), it(N, 0);
+    std::vector<uint8_t> onst(N, 0);
+    std::vector<int64_t> st, work;
+    st.reserve(1024); work.reserve(1024);
+    comp.assign(N, -1);
+    int64_t counter = 0, ncomp = 0;
+    for (int64_t r = 0; r < N; r++) {
+        if (index[r] != -1) continue;
+        index[r] = low[r] = counter++;
+        st.push_back(r); onst[r] = 1; it[r] = ptr[r];
+        work.push_back(r);
+        while (!work.empty()) {
+            int64_t v = work.back();
+            if (it[v] < ptr[v + 1]) {
+                int64_t u = adj[it[v]++];
+                if (index[u] == -1) {
+                    index[u] = low[u] = counter++;
+                    st.push_back(u); onst[u] = 1; it[u] = ptr[u];
+                    work.push_back(u);
+                } else if (onst[u]) {
+                    low[v] = std::min(low[v], index[u]);
+                }
+            } else {
+                work.pop_back();
+                if (!work.empty()) { int64_t p = work.back(); low[p] = std::min(low[p], low[v]); }
+                if (low[v] == index[v]) {
+                    while (true) {
+                        int64_t x = st.back(); st.pop_back(); onst[x] = 0;
+                        comp[x] = ncomp;
+                        if (x == v) break;
+                    }
+                    ncomp++;
+                }
+            }
+        }
+    }
+    return ncomp;
+}
+
+}  // namespace
+
+void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
+    auto t0 = std::chrono::steady_clock::now();
+    const int64_t n = g.n, m = g.m;
+    L = HostLayout();
+    L.params = p;
+    std::vector<int64_t> deg(n);
+    for (int64_t v = 0; v < n; v++) deg[v] = (int64_t)g.indeg[v] + g.outdeg[v];
+
+    // ---- line 5: successors sorted by (degree desc, id asc), stable in CSR order
+    std::vector<int32_t> scol(g.col), sw(m);
+    if (g.has_w) sw = g.w; else std::fill(sw.begin(), sw.end(), 1);
+    #pragma omp parallel for schedule(dynamic, 4096)
+    for (int64_t v = 0; v < n; v++) {
+        int64_t b = g.row_ptr[v], e = g.row_ptr[v + 1];
+        if (e - b < 2) continue;
+        std::vector<std::pair<int32_t, int32_t>> tmp(e - b);
+        for (int64_t i = b; i < e; i++) tmp[i - b] = {scol[i], sw[i]};
+        if (p.order == 0)
+            std::stable_sort(tmp.begin(), tmp.end(), [&](const auto& x, const auto& y) {
+                if (deg[x.first] != deg[y.first]) return deg[x.first] > deg[y.first];
+                return x.first < y.first;
+            });
+        else
+            std::stable_sort(tmp.begin(), tmp.end(),
+                             [](const auto& x, const auto& y) { return x.first < y.first; });
+        for (int64_t i = b; i < e; i++) { scol[i] = tmp[i - b].first; sw[i] = tmp[i - b].second; }
+    }
+
+    // ---- subgraphs: contiguous vertex ranges of ~m/T out-edges (reading R-SUB)
+    const int T = std::max(1, p.n_sub);
+    std::vector<int64_t> bounds(T + 1, 0);
+    for (int k = 1; k < T; k++) {
+        int64_t target = (int64_t)(((__int128)k * m) / T);
+        int64_t v = std::lower_bound(g.row_ptr.begin(), g.row_ptr.begin() + n + 1, target) - g.row_ptr.begin();
+        bounds[k] = std::max(bounds[k - 1], std::min(v, n));
+    }
+    bounds[T] = n;
+
+    // ---- Algorithm 1 on every subgraph (parallel over subgraphs)
+    std::vector<SubOut> subs(T);
+    std::vector<uint8_t> expanded(n, 0), inner(n, 0);
+    const int nthr = omp_get_max_threads();
+    std::vector<std::vector<uint32_t>> vis(nthr);
+    #pragma omp parallel for schedule(dynamic, 1)
+    for (int k = 0; k < T; k++) {
+        auto& visited = vis[omp_get_thread_num()];
+        if (visited.empty()) visited.assign(n, 0);
+        int64_t lo = bounds[k], hi = bounds[k + 1];
+        SubOut& out = subs[k];
+        out.start.push_back(0);
+        Decomposer D{g, scol, sw, deg, expanded, inner, visited, (uint32_t)(k + 1), lo, hi, p.d_max, out};
+        std::vector<int32_t> roots(hi - lo);
+        std::iota(roots.begin(), roots.end(), (int32_t)lo);
+        if (p.order == 0)
+            std::stable_sort(roots.begin(), roots.end(),
+                             [&](int32_t a, int32_t b) { return deg[a] > deg[b]; });
+        for (int32_t r : roots)
+            if (D.has_unvisited(r)) D.graphp(r, 0);
+        D.new_path();
+    }
+
+    // ---- concatenate (subgraph order)
+    std::vector<int64_t> poff{0};
+    std::vector<int32_t> pv, pw;
+    {
+        int64_t tot = 0;
+        for (auto& s : subs) tot += (int64_t)s.pv.size();
+        pv.reserve(tot); pw.reserve(tot);
+        for (auto& s : subs) {
+            int64_t base = (int64_t)pv.size();
+            pv.insert(pv.end(), s.pv.begin(), s.pv.end());
+            pw.insert(pw.end(), s.pw.begin(), s.pw.end());
+            for (size_t i = 1; i < s.start.size(); i++) poff.push_back(base + s.start[i]);
+            SubOut().pv.swap(s.pv);
+        }
+    }
+    const int64_t P0 = (int64_t)poff.size() - 1;
+    L.paths_before_merge = P0;
+
+    // ---- short-path merging (reading R-MERGE)
+    std::vector<int64_t> nxt(P0, -1), last(P0), clen(P0);
+    std::vector<uint8_t> absorbed(P0, 0);
+    for (int64_t i = 0; i < P0; i++) { last[i] = i; clen[i] = poff[i + 1] - poff[i] - 1; }
+    if (p.l_merge > 0 && P0 > 1) {
+        std::vector<int64_t> hptr(n + 1, 0), hlist(P0), cursor(n);
+        for (int64_t i = 0; i < P0; i++) hptr[pv[poff[i]] + 1]++;
+        for (int64_t v = 0; v < n; v++) hptr[v + 1] += hptr[v];
+        for (int64_t v = 0; v < n; v++) cursor[v] = hptr[v];
+        {
+            std::vector<int64_t> fill(hptr.begin(), hptr.end() - 1);
+            for (int64_t i = 0; i < P0; i++) hlist[fill[pv[poff[i]]]++] = i;
+        }
+        for (int64_t i = 0; i < P0; i++) {
+            if (absorbed[i]) continue;
+            while (true) {
+                int64_t lp = last[i];
+                int32_t x = pv[poff[lp + 1] - 1];
+                if (g.indeg[x] > 1 && g.outdeg[x] > 1 && inner[x]) break;
+                int64_t pick = -1;
+                while (cursor[x] < hptr[x + 1] && absorbed[hlist[cursor[x]]]) cursor[x]++;
+                for (int64_t k = cursor[x]; k < hptr[x + 1]; k++) {
+                    int64_t j = hlist[k];
+                    if (j == i || absorbed[j]) continue;
+                    if (clen[i] + clen[j] <= p.l_merge) { pick = j; break; }
+                }
+                if (pick < 0) break;
+                nxt[last[i]] = pick;
+                last[i] = last[pick];
+                clen[i] += clen[pick];
+                absorbed[pick] = 1;
+            }
+        }
+    }
+    // materialise merged paths (merge order)
+    std::vector<int64_t> moff{0};
+    std::vector<int32_t> mv, mw;
+    mv.reserve(pv.size()); mw.reserve(pv.size());
+    for (int64_t i = 0; i < P0; i++) {
+        if (absorbed[i]) continue;
+        bool first = true;
+        for (int64_t c = i; c >= 0; c = nxt[c]) {
+            for (int64_t k = poff[c] + (first ? 0 : 1); k < poff[c + 1]; k++) {
+                mv.push_back(pv[k]); mw.push_back(pw[k]);
+            }
+            first = false;
+        }
+        moff.push_back((int64_t)mv.size());
+    }
+    { std::vector<int32_t>().swap(pv); std::vector<int32_t>().swap(pw); }
+    const int64_t P = (int64_t)moff.size() - 1;
+
+    // ---- path statistics (reading R-HOT)
+    std::vector<double> dbar(P);
+    std::vector<int64_t> nvert(P);
+    std::vector<uint8_t> hot(P);
+    const double mean_deg = n ? 2.0 * (double)m / (double)n : 0.0;
+    #pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < P; i++) {
+        double s = 0;
+        for (int64_t k = moff[i]; k < moff[i + 1]; k++) s += (double)deg[mv[k]];
+        nvert[i] = moff[i + 1] - moff[i];
+        dbar[i] = s / (double)nvert[i];
+        hot[i] = dbar[i] >= (double)p.hot_factor * mean_deg;
+    }
+
+    // ---- dependency graph G' as a bipartite path/vertex graph (reading R-DEP):
+    // path node i -> vertex node P+x for every x entered by an edge of i;
+    // vertex node P+x -> path node j for every x left by an edge of j.
+    // Reachability between path nodes equals reachability in G'.
+    const int64_t N = P + n;
+    std::vector<int64_t> aptr(N + 1, 0), adj;
+    std::vector<int64_t> layer_of_path(P, 0), scc_label(P, 0);
+    int64_t n_layers = 0, n_dep_sccs = 0, giant = 0;
+    {
+        for (int64_t i = 0; i < P; i++) {
+            int64_t len = moff[i + 1] - moff[i];
+            aptr[i + 1] += len - 1;                                   // entered vertices
+            for (int64_t k = moff[i]; k < moff[i + 1] - 1; k++) aptr[P + mv[k] + 1]++;  // left vertices
+        }
+        for (int64_t x = 0; x < N; x++) aptr[x + 1] += aptr[x];
+        adj.resize(aptr[N]);
+        std::vector<int64_t> fill(aptr.begin(), aptr.end() - 1);
+        for (int64_t i = 0; i < P; i++) {
+            for (int64_t k = moff[i] + 1; k < moff[i + 1]; k++) adj[fill[i]++] = P + mv[k];
+            for (int64_t k = moff[i]; k < moff[i + 1] - 1; k++) adj[fill[P + mv[k]]++] = i;
+        }
+        std::vector<int64_t> comp;
+        int64_t nc = tarjan(N, aptr, adj, comp);
+        // group nodes by comp; comps are numbered in reverse topological order
+        std::vector<int64_t> cptr(nc + 1, 0), cnodes(N);
+        for (int64_t x = 0; x < N; x++) cptr[comp[x] + 1]++;
+        for (int64_t c = 0; c < nc; c++) cptr[c + 1] += cptr[c];
+        {
+            std::vector<int64_t> fill2(cptr.begin(), cptr.end() - 1);
+            for (int64_t x = 0; x < N; x++) cnodes[fill2[comp[x]]++] = x;
+        }
+        std::vector<int64_t> f(nc, 0), minpath(nc, INT64_MAX), npaths(nc, 0);
+        for (int64_t i = 0; i < P; i++) {
+            minpath[comp[i]] = std::min(minpath[comp[i]], i);
+            npaths[comp[i]]++;
+        }
+        // topological order = decreasing comp id (sources first)
+        for (int64_t c = nc - 1; c >= 0; c--) {
+            int64_t add = npaths[c] > 0 ? 1 : 0;
+            for (int64_t q = cptr[c]; q < cptr[c + 1]; q++) {
+                int64_t x = cnodes[q];
+                for (int64_t e = aptr[x]; e < aptr[x + 1]; e++) {
+                    int64_t d = comp[adj[e]];
+                    if (d != c) f[d] = std::max(f[d], f[c] + add);
+                }
+            }
+        }
+        for (int64_t i = 0; i < P; i++) {
+            layer_of_path[i] = f[comp[i]];
+            scc_label[i] = minpath[comp[i]];
+            n_layers = std::max(n_layers, f[comp[i]] + 1);
+        }
+        for (int64_t c = 0; c < nc; c++)
+            if (npaths[c] > 0) { n_dep_sccs++; giant = std::max(giant, npaths[c]); }
+    }
+    { std::vector<int64_t>().swap(adj); std::vector<int64_t>().swap(aptr); }
+
+    // ---- priority Pri(p) = alpha*D(p)*N(p) - L(p)
+    double dmax = 0; int64_t nmax = 0;
+    for (int64_t i = 0; i < P; i++) { dmax = std::max(dmax, dbar[i]); nmax = std::max(nmax, nvert[i]); }
+    const double alpha = (dmax > 0 && nmax > 0) ? 1.0 / (dmax * (double)nmax) : 0.0;
+    std::vector<double> pri(P);
+    for (int64_t i = 0; i < P; i++) pri[i] = alpha * dbar[i] * (double)nvert[i] - (double)layer_of_path[i];
+    std::vector<int64_t> order(P);
+    std::iota(order.begin(), order.end(), 0);
+    std::stable_sort(order.begin(), order.end(), [&](int64_t a, int64_t b) { return pri[a] > pri[b]; });
+
+    // ---- partitions over the priority order (greedy, whole paths)
+    const int64_t target = std::max<int32_t>(1, p.part_entries);
+    std::vector<int64_t> gpart_first{0};  // global partition -> first index in `order`
+    {
+        int64_t acc = 0;
+        for (int64_t r = 0; r < P; r++) {
+            if (acc >= target) { gpart_first.push_back(r); acc = 0; }
+            acc += nvert[order[r]];
+        }
+        gpart_first.push_back(P);
+        if (P == 0) gpart_first.assign(1, 0);
+    }
+    const int64_t G = (int64_t)gpart_first.size() - 1;
+    const int world = std::max(1, p.world), rank = p.rank;
+
+    // ---- boundary vertices: present in partitions of >1 rank (round-robin owner q % world)
+    if (world > 1) {
+        std::vector<uint64_t> mask(n, 0);
+        for (int64_t q = 0; q < G; q++) {
+            uint64_t bit = 1ull << ((q % world) & 63);
+            for (int64_t r = gpart_first[q]; r < gpart_first[q + 1]; r++) {
+                int64_t i = order[r];
+                for (int64_t k = moff[i]; k < moff[i + 1]; k++) mask[mv[k]] |= bit;
+            }
+        }
+        for (int64_t v = 0; v < n; v++)
+            if (__builtin_popcountll(mask[v]) > 1) L.boundary.push_back((int32_t)v);
+    }
+
+    // ---- this rank's layout
+    L.part_off.push_back(0);
+    L.path_off.push_back(0);
+    for (int64_t q = rank; q < G; q += world) {
+        for (int64_t r = gpart_first[q]; r < gpart_first[q + 1]; r++) {
+            int64_t i = order[r];
+            for (int64_t k = moff[i]; k < moff[i + 1]; k++) {
+                uint32_t code = (uint32_t)mv[k];
+                if (k == moff[i]) code |= kHead;
+                if (k == moff[i + 1] - 1) code |= kTail;
+                L.e_idx.push_back(code);
+                L.e_w.push_back(mw[k]);
+            }
+            L.path_off.push_back((int64_t)L.e_idx.size());
+            L.layer.push_back((int32_t)layer_of_path[i]);
+            L.scc.push_back(scc_label[i]);
+            L.merged_index.push_back(i);
+            L.hot.push_back(hot[i]);
+            L.n_hot += hot[i];
+        }
+        L.part_off.push_back((int64_t)L.e_idx.size());
+    }
+    const int64_t npart = (int64_t)L.part_off.size() - 1;
+
+    // ---- vertex -> partitions (distinct), source (non-tail) and destination (non-head) occurrences
+    auto build_map = [&](uint32_t skip_flag, std::vector<int64_t>& ptr, std::vector<int32_t>& lst) {
+        ptr.assign(n + 1, 0);
+        std::vector<int32_t> lastp(n, -1);
+        for (int64_t q = 0; q < npart; q++)
+            for (int64_t k = L.part_off[q]; k < L.part_off[q + 1]; k++) {
+                uint32_t c = L.e_idx[k];
+                if (c & skip_flag) continue;
+                int32_t v = (int32_t)(c & kVMask);
+                if (lastp[v] != (int32_t)q) { lastp[v] = (int32_t)q; ptr[v + 1]++; }
+            }
+        for (int64_t v = 0; v < n; v++) ptr[v + 1] += ptr[v];
+        lst.resize(ptr[n]);
+        std::vector<int64_t> fill(ptr.begin(), ptr.end() - 1);
+        std::fill(lastp.begin(), lastp.end(), -1);
+        for (int64_t q = 0; q < npart; q++)
+            for (int64_t k = L.part_off[q]; k < L.part_off[q + 1]; k++) {
+                uint32_t c = L.e_idx[k];
+                if (c & skip_flag) continue;
+                int32_t v = (int32_t)(c & kVMask);
+                if (lastp[v] != (int32_t)q) { lastp[v] = (int32_t)q; lst[fill[v]++] = (int32_t)q; }
+            }
+    };
+    build_map(kTail, L.vsrc_ptr, L.vsrc);
+    build_map(kHead, L.vdst_ptr, L.vdst);
+
+    L.n_layers = n_layers;
+    L.n_dep_sccs = n_dep_sccs;
+    L.giant = giant;
+    L.built = true;
+    L.preprocess_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+}
+
+}  // namespace dg

@@ -1,0 +1,156 @@
+"""-m "not gpu": the C-ABI library loads and exports every symbol of
+include/digraph.h, and its host preprocessing rows (Algorithm 1, merging,
+dependency DAG, layers, priority order, partitions) agree exactly with the
+oracle -- the product and the oracle share no code."""
+import itertools
+import os
+import re
+
+import numpy as np
+import pytest
+
+import inputs
+from oracle import paths as OP
+from paper_conf_asplos_zhangl0hlg19_b200 import _abi, DiGraph, DGError
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_library_exports_every_header_symbol():
+    hdr = open(os.path.join(ROOT, "include", "digraph.h")).read()
+    declared = sorted(set(re.findall(r"^\s*(?:int|void|const char \*)\s*\*?\s*(dg_\w+)\s*\(", hdr, re.M)))
+    assert declared, "no declarations parsed"
+    L = _abi.lib()
+    for name in declared:
+        assert hasattr(L, name), name
+    assert sorted(_abi.EXPORTS) == declared
+
+
+def oracle_layout(g, d_max, n_sub, order, l_merge):
+    src, dst, _ = g.edges()
+    paths, inner = OP.graphp_decompose(g.n, g.row_ptr, g.col, d_max=d_max, n_sub=n_sub, order=order)
+    merged = OP.merge_short_paths(g.n, src, dst, paths, inner, l_max=l_merge) if l_merge else paths
+    dep = OP.dependency_graph(merged)
+    scc, layer = OP.condense_and_layer(len(merged), dep)
+    dbar, nv, hot = OP.path_stats(g.n, src, dst, merged, hot_factor=2.0)
+    pri = OP.priority(dbar, nv, layer)
+    return paths, merged, scc, layer, hot, pri
+
+
+def product_layout(g, d_max, n_sub, order, l_merge, part_entries=64):
+    dg = DiGraph()
+    dg.load_graph(g)
+    dg.build_paths(d_max=d_max, l_merge=l_merge, n_sub=n_sub, order=order, part_entries=part_entries)
+    return dg, dg.export_paths(), dg.layout_info()
+
+
+def split(ex):
+    off, v = ex["path_off"], ex["vertices"]
+    return [v[off[i]:off[i + 1]].tolist() for i in range(len(off) - 1)]
+
+
+def fig4_graph():
+    edges = [(0, 1), (1, 2), (2, 3), (3, 4), (4, 5), (3, 6), (6, 7), (7, 8), (8, 9), (8, 10),
+             (10, 11), (11, 12), (7, 13), (13, 14), (14, 6)]
+    return inputs.from_edges(15, [e[0] for e in edges], [e[1] for e in edges], [1] * len(edges))
+
+
+def test_product_reproduces_figure4_layout():
+    g = fig4_graph()
+    dg, ex, info = product_layout(g, 16, 1, "id", 0)
+    paths = split(ex)
+    by_merge = [p for _, p in sorted(zip(ex["merged_index"].tolist(), paths))]
+    assert by_merge == [[0, 1, 2, 3, 4, 5], [3, 6, 7, 8, 9], [8, 10, 11, 12], [7, 13, 14, 6]]
+    lay = dict(zip(ex["merged_index"].tolist(), ex["layer"].tolist()))
+    assert [lay[i] for i in range(4)] == [0, 1, 2, 1]
+    scc = dict(zip(ex["merged_index"].tolist(), ex["scc"].tolist()))
+    assert [scc[i] for i in range(4)] == [0, 1, 2, 1]
+    # priority order: layer 0 first, layer 2 last
+    assert ex["layer"].tolist() == sorted(ex["layer"].tolist())
+    assert info["n_layers"] == 3 and info["n_dep_sccs"] == 3 and info["giant_scc_paths"] == 2
+
+
+CASES = list(itertools.product([0, 1, 2], [1, 3], ["degree", "id"], [0, 64], [16, 3]))
+
+
+@pytest.mark.parametrize("seed,n_sub,order,l_merge,d_max", CASES)
+def test_product_preprocessing_matches_oracle(seed, n_sub, order, l_merge, d_max):
+    g = inputs.rmat(9, 400, 2500, seed=seed, weights=(1, 9)) if seed != 2 else \
+        inputs.uniform(300, 1200, seed=seed, weights=(1, 9))
+    o_paths, o_merged, o_scc, o_layer, o_hot, o_pri = oracle_layout(g, d_max, n_sub, order, l_merge)
+    dg, ex, info = product_layout(g, d_max, n_sub, order, l_merge)
+    assert info["paths_before_merge"] == len(o_paths)
+    paths = split(ex)
+    midx = ex["merged_index"]
+    assert sorted(midx.tolist()) == list(range(len(o_merged)))
+    for p, i in zip(paths, midx.tolist()):
+        assert p == o_merged[i]
+    # dependency SCC labels and layers
+    assert np.array_equal(ex["scc"], o_scc[midx])
+    assert np.array_equal(ex["layer"], o_layer[midx])
+    assert np.array_equal(ex["hot"], o_hot[midx])
+    # priority order = stable sort by Pri desc
+    assert midx.tolist() == np.argsort(-o_pri, kind="stable").tolist()
+    # partitions cover whole paths in order
+    po = ex["part_off"]
+    assert po[0] == 0 and po[-1] == ex["path_off"][-1]
+    assert set(po.tolist()) <= set(ex["path_off"].tolist())
+
+
+def test_edge_weights_follow_paths():
+    g = inputs.rmat(8, 256, 1500, seed=5, weights=(1, 255))
+    dg, ex, info = product_layout(g, 16, 2, "degree", 64)
+    # every path edge is a graph edge; weights are the graph's
+    wmap = {}
+    src, dst, w = g.edges()
+    for a, b, c in zip(src.tolist(), dst.tolist(), w.tolist()):
+        wmap[(a, b)] = c
+    cover = []
+    for p in split(ex):
+        cover += list(zip(p[:-1], p[1:]))
+    assert sorted(cover) == sorted(zip(src.tolist(), dst.tolist()))
+
+
+def test_multirank_partitioning_is_a_disjoint_cover():
+    g = inputs.rmat(10, 1000, 8000, seed=3)
+    world = 3
+    covers, bnd_sets, presence = [], [], []
+    for r in range(world):
+        dg = DiGraph()
+        dg.load_graph(g)
+        dg.build_paths(part_entries=128, rank=r, world=world)
+        ex = dg.export_paths()
+        cov = []
+        for p in split(ex):
+            cov += list(zip(p[:-1], p[1:]))
+        covers.append(cov)
+        bnd_sets.append(dg.boundary_vertices().tolist())
+        presence.append(set(ex["vertices"].tolist()))
+    src, dst, _ = g.edges()
+    assert sorted(sum(covers, [])) == sorted(zip(src.tolist(), dst.tolist()))
+    assert bnd_sets[0] == bnd_sets[1] == bnd_sets[2]
+    multi = sorted(v for v in range(g.n) if sum(v in s for s in presence) > 1)
+    assert bnd_sets[0] == multi
+    sizes = [len(c) for c in covers]
+    assert max(sizes) - min(sizes) <= 0.2 * max(sizes)       # balanced
+
+
+def test_run_without_cuda_fails_loudly():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("CUDA present")
+    dg = DiGraph()
+    dg.load_graph(fig4_graph())
+    dg.build_paths()
+    with pytest.raises(DGError, match="DG_ENOCUDA"):
+        dg.run("sssp", source=0)
+
+
+def test_bad_arguments_are_rejected():
+    dg = DiGraph()
+    with pytest.raises(DGError, match="DG_EINVAL"):
+        dg.build_paths()
+    with pytest.raises(DGError, match="DG_EINVAL"):
+        dg.load_csr(3, np.array([0, 1, 2, 9]), np.array([1, 2, 0]))
+    with pytest.raises(DGError, match="DG_EINVAL"):
+        dg.load_csr(3, np.array([0, 1, 2, 3]), np.array([1, 2, 7]))
