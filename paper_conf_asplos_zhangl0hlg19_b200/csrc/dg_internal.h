@@ -40,8 +40,14 @@ struct HostLayout {
     // vertex -> partitions maps
     std::vector<int64_t> vsrc_ptr;  std::vector<int32_t> vsrc;   // non-tail occurrences
     std::vector<int64_t> vdst_ptr;  std::vector<int32_t> vdst;   // non-head occurrences
+    // home partition of each vertex: first (highest-priority) local partition
+    // holding it, -1 if none; PageRank/Adsorption activate it when the
+    // vertex's delta crosses eps
+    std::vector<int32_t> hpart;
     // multi-rank
     std::vector<int32_t> boundary;      // vertices present on >1 rank (ascending)
+    std::vector<uint8_t> bnd_owner;     // this rank owns boundary[k] (lowest rank holding it)
+    std::vector<uint8_t> vown;          // this rank owns vertex v (lowest rank holding it; rank 0 if none)
     // stats
     int64_t n_layers = 0, n_dep_sccs = 0, giant = 0, paths_before_merge = 0, n_hot = 0;
     double preprocess_ms = 0;
@@ -58,6 +64,9 @@ struct DevLayout {
     int64_t* vsrc_ptr = nullptr; int32_t* vsrc = nullptr;
     int64_t* vdst_ptr = nullptr; int32_t* vdst = nullptr;
     int32_t* bnd = nullptr;
+    uint8_t* bnd_owner = nullptr;
+    int32_t* hpart = nullptr;
+    uint8_t* vown = nullptr;
     // CSR (for the vertex-centric ablation and per-vertex coefficients)
     int64_t* row_ptr = nullptr; int32_t* col = nullptr; int32_t* w = nullptr;
     int32_t* outdeg = nullptr;

@@ -60,7 +60,6 @@ struct DevWork {
     int grid_path = 0, grid_vertex = 0;
     uint2* vs_u = nullptr;      // {value, stamp}: SSSP/BFS dist, WCC label
     float4* vs_f = nullptr;     // {T, coef, sigma|delta, stamp}: PR / Adsorption
-    float* s_val = nullptr;     // per-entry mirror value S_val (Fig. 4)
     float* e_coef = nullptr;    // Adsorption: coefficient of the path edge out of each entry
     float* ads_base = nullptr;  // Adsorption: p_inj * I per vertex
     float* ads_pcont = nullptr; // Adsorption: p_cont per vertex
@@ -69,7 +68,6 @@ struct DevWork {
     int32_t* vlist[2] = {nullptr, nullptr};
     int32_t* blockcnt = nullptr;
     Counters* ctr = nullptr;
-    float* bnd_base = nullptr;
     double* dsum = nullptr;
     int32_t* scc_color = nullptr;
     int32_t* scc_label = nullptr;
@@ -88,13 +86,13 @@ struct KParams {
     const int32_t* vsrc;
     const int64_t* vdst_ptr;
     const int32_t* vdst;
+    const int32_t* hpart;
     const int64_t* row_ptr;
     const int32_t* col;
     const int32_t* w;
     int64_t n_part, n;
     uint2* vs_u;
     float4* vs_f;
-    float* s_val;
     const float* e_coef;
     uint8_t* part_flag;
     int32_t* plist0;
@@ -272,29 +270,39 @@ __device__ void walk_minplus(const KParams& P, int64_t beg, int64_t end, int rou
     }
 }
 
-// Accumulative walk (PageRank / Adsorption), Fig. 4 S_val as the
-// per-entry mirror: the path edge out of entry i pushes
-//   a_i = c_i * (pend_i + p_i),  pend_i = T_i - S_val[i] if >= eps else 0,
-// where p_i = a_{i-1} is what the path predecessor pushed in this walk (used
-// immediately: PAPER.md line 96), T_i the gathered master total and c_i the
-// edge coefficient (d/outdeg for PageRank).  S_val[i] += pend_i + p_i.
-template <bool EDGE_COEF>
-__device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round, Acc& acc) {
-    const int lane = threadIdx.x & 31;
+// Accumulative walk (PageRank / Adsorption).
+// Vertex state {r, g, delta, stamp}: r = accumulated value, delta = pending
+// (fp32, small magnitudes -> no cancellation), g = per-vertex push factor
+// (d/outdeg for PageRank, p_cont/W(u) for Adsorption).  Walking a path in
+// order, entry i fires f_i = delta_i + p_i where delta_i is claimed from the
+// master when >= eps (the per-vertex stop rule) and p_i = c_(i-1) * f_(i-1)
+// is what its path predecessor just fired along the path edge -- used in the
+// same round (Observation 1).  The in-window recurrence is
+// the affine scan q_i = c_i * (delta_i + q_(i-1)).  A firing vertex adds f_i
+// to r and pushes g*w*f_i to all its out-neighbours' deltas through the CSR
+// (warp-cooperative, load-balanced); the amount p_i it already received
+// in-register is debited from its own delta ("borrowed"), so mass is
+// conserved exactly.  A delta crossing eps activates the vertex's home
+// partition.
+template <bool ADS>
+__device__ void walk_delta(const KParams& P, int64_t beg, int64_t end, Acc& acc) {
+    __shared__ int32_t s_v[kWarps][128];
+    __shared__ float s_amt[kWarps][128];
+    __shared__ int64_t s_row[kWarps][128];
+    __shared__ int32_t s_off[kWarps][129];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const float eps = P.eps;
-    float carry = 0.f;
     for (int64_t base = beg & ~(int64_t)3; base < end; base += 128) {
         const int64_t i0 = base + 4 * lane;
         uint4 code = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
-        float4 s4 = make_float4(0.f, 0.f, 0.f, 0.f), c4 = s4;
+        float4 c4 = make_float4(0.f, 0.f, 0.f, 0.f);
         if (i0 < end) {
             code = ld_stream_u4(P.e_idx + i0);
-            s4 = ld_stream_f4(P.s_val + i0);
-            if (EDGE_COEF) c4 = ld_stream_f4(P.e_coef + i0);
+            if (ADS) c4 = ld_stream_f4(P.e_coef + i0);
         }
-        float T0[4], al[4], be[4], pend[4], sv[4];
+        float al[4], be[4], dl[4], gf[4];
         uint32_t vtx[4];
-        bool hd[4], tl[4], valid[4];
+        bool hd[4], valid[4];
 #pragma unroll
         for (int k = 0; k < 4; k++) {
             const int64_t i = i0 + k;
@@ -302,17 +310,19 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round
             uint32_t c = u4get(code, k);
             vtx[k] = c & kVMask;
             hd[k] = !valid[k] || (c & kHead);
-            tl[k] = !valid[k] || (c & kTail);
+            bool tl = !valid[k] || (c & kTail);
             float4 st = valid[k] ? P.vs_f[vtx[k]] : make_float4(0.f, 0.f, 0.f, 0.f);
-            T0[k] = st.x;
-            sv[k] = f4get(s4, k);
-            float coef = EDGE_COEF ? f4get(c4, k) : st.y;
-            float pd = T0[k] - sv[k];
-            pend[k] = (!tl[k] && pd >= eps) ? pd : 0.f;
-            al[k] = tl[k] ? 0.f : coef * pend[k];
-            be[k] = (tl[k] || hd[k]) ? 0.f : coef;
+            float d = 0.f;
+            if (valid[k] && st.z >= eps) {
+                d = atomicExch(&P.vs_f[vtx[k]].z, 0.f);
+                if (d < 0.f) { atomicAdd(&P.vs_f[vtx[k]].z, d); d = 0.f; }
+            }
+            dl[k] = d;
+            gf[k] = st.y;
+            float cout = tl ? 0.f : (ADS ? f4get(c4, k) : st.y);
+            al[k] = cout * d;
+            be[k] = (tl || hd[k]) ? 0.f : cout;
         }
-        // lane aggregate of f_k(x) = al + be * x
         float Al = 0.f, Be = 1.f;
 #pragma unroll
         for (int k = 0; k < 4; k++) { Al = al[k] + be[k] * Al; Be = be[k] * Be; }
@@ -322,45 +332,83 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round
             float Bp = __shfl_up_sync(0xffffffffu, Be, off);
             if (lane >= off) { Al = Al + Be * Ap; Be = Be * Bp; }
         }
-        float Ae = __shfl_up_sync(0xffffffffu, Al, 1);
-        float Bx = __shfl_up_sync(0xffffffffu, Be, 1);
-        if (lane == 0) { Ae = 0.f; Bx = 1.f; }
-        float prev = Ae + Bx * carry;
-        float pin[4];
+        float prev = __shfl_up_sync(0xffffffffu, Al, 1);
+        if (lane == 0) prev = 0.f;  // no carry across windows: earlier windows pushed through memory
+        float f[4];
+        bool fire[4];
 #pragma unroll
         for (int k = 0; k < 4; k++) {
-            pin[k] = hd[k] ? 0.f : prev;
+            float pin = hd[k] ? 0.f : prev;
             prev = al[k] + be[k] * prev;
-        }
-        carry = __shfl_sync(0xffffffffu, prev, 31);
-        bool sig[4];
-        float tnew[4];
-#pragma unroll
-        for (int k = 0; k < 4; k++) {
-            sig[k] = false;
-            tnew[k] = 0.f;
-            if (!valid[k]) continue;
-            if (!hd[k]) acc.edges++;
-            const float p = pin[k];
-            if (p > 0.f) {
-                float old = atomicAdd(&P.vs_f[vtx[k]].x, p);
-                tnew[k] = old + p;
+            f[k] = dl[k] + pin;
+            fire[k] = valid[k] && f[k] > 0.f;
+            if (valid[k] && !hd[k]) acc.edges++;
+            if (fire[k]) {
+                atomicAdd(&P.vs_f[vtx[k]].x, f[k]);
+                if (pin > 0.f) atomicAdd(&P.vs_f[vtx[k]].z, -pin);  // borrowed from the CSR push below
                 acc.upd++;
-                float sigma = P.vs_f[vtx[k]].z;
-                if (tnew[k] - sigma >= eps)
-                    sig[k] = atomicExch(reinterpret_cast<int*>(&P.vs_f[vtx[k]].w), round + 1) != round + 1;
-                if (sig[k]) P.vs_f[vtx[k]].z = tnew[k];
-            }
-            if (!tl[k]) {
-                float ns = sv[k] + pend[k] + p;
-                if (ns != sv[k]) P.s_val[i0 + k] = ns;
             }
         }
+        // gather the fired vertices of the window (<= 128) and expand their CSR rows
+        int nit = 0;
 #pragma unroll
         for (int k = 0; k < 4; k++) {
-            uint32_t m = __ballot_sync(0xffffffffu, sig[k]);
-            if (m) flag_partitions(m, (int)vtx[k], P.vsrc_ptr, P.vsrc, P.part_flag);
+            uint32_t m = __ballot_sync(0xffffffffu, fire[k]);
+            if (fire[k]) {
+                int pos = nit + __popc(m & ((1u << lane) - 1));
+                s_v[wid][pos] = (int32_t)vtx[k];
+                s_amt[wid][pos] = f[k] * gf[k];
+            }
+            nit += __popc(m);
         }
+        __syncwarp();
+        if (nit == 0) continue;
+        int dsum = 0, dg4[4];
+#pragma unroll
+        for (int t = 0; t < 4; t++) {
+            int it = lane * 4 + t;
+            dg4[t] = 0;
+            if (it < nit) {
+                int v = s_v[wid][it];
+                int64_t r0 = P.row_ptr[v];
+                dg4[t] = (int)(P.row_ptr[v + 1] - r0);
+                s_row[wid][it] = r0;
+            }
+            dsum += dg4[t];
+        }
+        int inc = dsum;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            int y = __shfl_up_sync(0xffffffffu, inc, off);
+            if (lane >= off) inc += y;
+        }
+        int run = inc - dsum;
+#pragma unroll
+        for (int t = 0; t < 4; t++) {
+            int it = lane * 4 + t;
+            if (it <= nit) s_off[wid][it] = run;
+            run += dg4[t];
+        }
+        if (lane == 31 && nit == 128) s_off[wid][128] = inc;
+        __syncwarp();
+        const int total = s_off[wid][nit];
+        for (int j = lane; j < total; j += 32) {
+            int lo = 0, hi = nit - 1;  // owner: largest o with s_off[o] <= j
+            while (lo < hi) {
+                int mid = (lo + hi + 1) >> 1;
+                if (s_off[wid][mid] <= j) lo = mid; else hi = mid - 1;
+            }
+            const int64_t e = s_row[wid][lo] + (j - s_off[wid][lo]);
+            const int x = P.col[e];
+            const float add = ADS ? s_amt[wid][lo] * (float)P.w[e] : s_amt[wid][lo];
+            const float old = atomicAdd(&P.vs_f[x].z, add);
+            if (old < eps && old + add >= eps) {
+                const int hp = P.hpart[x];
+                if (hp >= 0) P.part_flag[hp] = 1;  // -1: x lives on another rank (multi-GPU sync delivers it)
+            }
+            acc.edges++;
+        }
+        __syncwarp();
     }
 }
 
@@ -599,8 +647,8 @@ __global__ void __launch_bounds__(kBlock) path_kernel(KParams P) {
             if (ALGO == DG_SSSP) walk_minplus<0>(P, beg, end, round, acc);
             else if (ALGO == DG_BFS) walk_minplus<1>(P, beg, end, round, acc);
             else if (ALGO == DG_WCC) walk_minplus<2>(P, beg, end, round, acc);
-            else if (ALGO == DG_PAGERANK) walk_accum<false>(P, beg, end, round, acc);
-            else if (ALGO == DG_ADSORPTION) walk_accum<true>(P, beg, end, round, acc);
+            else if (ALGO == DG_PAGERANK) walk_delta<false>(P, beg, end, acc);
+            else if (ALGO == DG_ADSORPTION) walk_delta<true>(P, beg, end, acc);
             else if (ALGO == 100) walk_scc_fwd(P, beg, end, round, acc);
             else if (ALGO == 101) walk_scc_bwd(P, beg, end, round, acc);
         }
@@ -733,16 +781,23 @@ __global__ void init_u_kernel(uint2* vs, int64_t n, int algo, int64_t source) {
         vs[v] = make_uint2(val, 0u);
     }
 }
-__global__ void init_pr_kernel(float4* vs, const int32_t* outdeg, int64_t n, float d, int vertex_mode) {
+// {r, g, delta, stamp}: r = 0, delta = 1-d (unnormalised PageRank, reading R-PR)
+// With several ranks only the vertex's owner rank starts with the delta, so
+// per-rank contributions add up (multi-GPU gather = sum).
+__global__ void init_pr_kernel(float4* vs, const int32_t* outdeg, const uint8_t* vown, int64_t n, float d) {
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
         float c = outdeg[v] > 0 ? d / (float)outdeg[v] : 0.f;
-        // path mode: T = 1-d, sigma = T.  vertex mode: r = 0, delta = 1-d.
-        vs[v] = vertex_mode ? make_float4(0.f, c, 1.f - d, 0.f) : make_float4(1.f - d, c, 1.f - d, 0.f);
+        vs[v] = make_float4(0.f, c, vown[v] ? 1.f - d : 0.f, 0.f);
     }
 }
-__global__ void init_ads_kernel(float4* vs, const float* base, int64_t n) {
+// Adsorption: r = 0, delta = p_inj * I, g = p_cont / W(u)
+__global__ void init_ads_kernel(float4* vs, const float* base, const float* gfac, const uint8_t* vown, int64_t n) {
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
-        vs[v] = make_float4(base[v], 0.f, base[v], 0.f);
+        vs[v] = make_float4(0.f, gfac[v], vown[v] ? base[v] : 0.f, 0.f);
+}
+__global__ void gfac_kernel(float* pcont_to_g, const float* wsum, int64_t n) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x)
+        pcont_to_g[v] = wsum[v] > 0.f ? pcont_to_g[v] / wsum[v] : 0.f;
 }
 __global__ void fill_iota_kernel(int32_t* a, int64_t n) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
@@ -769,21 +824,20 @@ __global__ void wsum_kernel(float* wsum, const int64_t* row_ptr, const int32_t* 
         wsum[v] = (float)s;
     }
 }
-__global__ void sum_T_kernel(const float4* vs, int64_t n, int vertex_mode, double* out) {
+__global__ void sum_T_kernel(const float4* vs, int64_t n, double* out) {
     double s = 0;
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
         float4 x = vs[v];
-        s += vertex_mode ? (double)x.x + (double)x.z : (double)x.x;
+        s += (double)x.x + (double)x.z;
     }
     for (int off = 16; off; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
     if ((threadIdx.x & 31) == 0) atomicAdd(out, s);
 }
-__global__ void out_pr_kernel(const float4* vs, int64_t n, int vertex_mode, const double* sum, float* out, int normalize) {
+__global__ void out_pr_kernel(const float4* vs, int64_t n, const double* sum, float* out, int normalize) {
     const double inv = normalize ? 1.0 / *sum : 1.0;
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n; v += (int64_t)gridDim.x * blockDim.x) {
         float4 x = vs[v];
-        double t = vertex_mode ? (double)x.x + (double)x.z : (double)x.x;
-        out[v] = (float)(t * inv);
+        out[v] = (float)(((double)x.x + (double)x.z) * inv);
     }
 }
 __global__ void out_u_kernel(const uint2* vs, int64_t n, uint32_t* out) {
@@ -846,27 +900,21 @@ __global__ void unpack_min_kernel(uint2* vs, const int32_t* bnd, int64_t nb, con
         }
     }
 }
-__global__ void pack_sum_kernel(const float4* vs, const int32_t* bnd, int64_t nb, const float* base, float* buf) {
+// SUM algorithms exchange the pending deltas of boundary vertices: every
+// rank contributes its local delta, the owner rank receives the total
+// ("each mirror always sends its new state to its master").
+__global__ void pack_sum_kernel(const float4* vs, const int32_t* bnd, int64_t nb, float* buf) {
     for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nb; k += (int64_t)gridDim.x * blockDim.x)
-        buf[k] = vs[bnd[k]].x - base[k];
+        buf[k] = vs[bnd[k]].z;
 }
-__global__ void unpack_sum_kernel(float4* vs, const int32_t* bnd, int64_t nb, float* base, const float* buf, float eps,
-                                  int round, const int64_t* ptr, const int32_t* lst, uint8_t* flag) {
+__global__ void unpack_sum_kernel(float4* vs, const int32_t* bnd, const uint8_t* owner, int64_t nb, const float* buf,
+                                  float eps, const int32_t* hpart, uint8_t* flag) {
     for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nb; k += (int64_t)gridDim.x * blockDim.x) {
         int v = bnd[k];
-        float t = base[k] + buf[k];
-        base[k] = t;
-        vs[v].x = t;
-        if (t - vs[v].z >= eps) {
-            vs[v].z = t;
-            vs[v].w = __int_as_float(round + 1);
-            for (int64_t j = ptr[v]; j < ptr[v + 1]; j++) flag[lst[j]] = 1;
-        }
+        float t = owner[k] ? buf[k] : 0.f;
+        vs[v].z = t;
+        if (t >= eps && hpart[v] >= 0) flag[hpart[v]] = 1;
     }
-}
-__global__ void init_base_kernel(const float4* vs, const int32_t* bnd, int64_t nb, float* base) {
-    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < nb; k += (int64_t)gridDim.x * blockDim.x)
-        base[k] = vs[bnd[k]].x;
 }
 // single-block ordered compaction of part_flag (outside the persistent kernel)
 __global__ void compact_flags_kernel(uint8_t* flag, int64_t n_part, int32_t* out, Counters* ctr, int slot) {
@@ -925,10 +973,10 @@ int grid_1d(int64_t n) {
 KParams make_params(const DevLayout& D, DevWork* W) {
     KParams P{};
     P.e_idx = D.e_idx; P.e_w = D.e_w; P.part_off = D.part_off;
-    P.vsrc_ptr = D.vsrc_ptr; P.vsrc = D.vsrc; P.vdst_ptr = D.vdst_ptr; P.vdst = D.vdst;
+    P.vsrc_ptr = D.vsrc_ptr; P.vsrc = D.vsrc; P.vdst_ptr = D.vdst_ptr; P.vdst = D.vdst; P.hpart = D.hpart;
     P.row_ptr = D.row_ptr; P.col = D.col; P.w = D.w;
     P.n_part = D.n_part; P.n = D.n;
-    P.vs_u = W->vs_u; P.vs_f = W->vs_f; P.s_val = W->s_val; P.e_coef = W->e_coef;
+    P.vs_u = W->vs_u; P.vs_f = W->vs_f; P.e_coef = W->e_coef;
     P.part_flag = W->part_flag; P.plist0 = W->plist[0]; P.plist1 = W->plist[1];
     P.vlist0 = W->vlist[0]; P.vlist1 = W->vlist[1];
     P.ctr = W->ctr; P.blockcnt = W->blockcnt;
@@ -943,7 +991,6 @@ int ensure_work(DevWork*& W, const DevLayout& D, std::string& err) {
     int rc;
     if ((rc = dalloc(&W->vs_u, D.n, bytes, err))) return rc;
     if ((rc = dalloc(&W->vs_f, D.n, bytes, err))) return rc;
-    if ((rc = dalloc(&W->s_val, D.M + kPad, bytes, err))) return rc;
     if ((rc = dalloc(&W->part_flag, D.n_part + 1, bytes, err))) return rc;
     if ((rc = dalloc(&W->plist[0], std::max<int64_t>(D.n_part, D.n) + 1, bytes, err))) return rc;
     if ((rc = dalloc(&W->plist[1], std::max<int64_t>(D.n_part, D.n) + 1, bytes, err))) return rc;
@@ -951,9 +998,7 @@ int ensure_work(DevWork*& W, const DevLayout& D, std::string& err) {
     if ((rc = dalloc(&W->blockcnt, 148 * 64, bytes, err))) return rc;
     if ((rc = dalloc(&W->ctr, 1, bytes, err))) return rc;
     if ((rc = dalloc(&W->dsum, 1, bytes, err))) return rc;
-    if ((rc = dalloc(&W->bnd_base, D.n_bnd + 1, bytes, err))) return rc;
     CK(cudaMemset(W->part_flag, 0, D.n_part + 1));
-    CK(cudaMemset(W->s_val, 0, sizeof(float) * (D.M + kPad)));
     CK(cudaEventCreate(&W->ev0));
     CK(cudaEventCreate(&W->ev1));
     return DG_OK;
@@ -1026,7 +1071,7 @@ int init_states(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
     if (S.mode == DG_MODE_VERTEX) {
         // frontier: the source (SSSP/BFS) or every vertex (PageRank)
         if (algo == DG_PAGERANK) {
-            init_pr_kernel<<<g, 256>>>(W->vs_f, D.outdeg, D.n, (float)S.param, 1);
+            init_pr_kernel<<<g, 256>>>(W->vs_f, D.outdeg, D.vown, D.n, (float)S.param);
             fill_iota_kernel<<<g, 256>>>(W->vlist[0], D.n);
             int nn = (int)D.n;
             CK(cudaMemcpy(&W->ctr->n_cur[0], &nn, sizeof(int), cudaMemcpyHostToDevice));
@@ -1054,9 +1099,8 @@ int init_states(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
         CK(cudaMemcpy(&W->ctr->n_cur[0], &np, sizeof(int), cudaMemcpyHostToDevice));
         S.stats.kernel_launches += 2;
     } else if (algo == DG_PAGERANK || algo == DG_ADSORPTION) {
-        if (algo == DG_PAGERANK) init_pr_kernel<<<g, 256>>>(W->vs_f, D.outdeg, D.n, (float)S.param, 0);
-        else init_ads_kernel<<<g, 256>>>(W->vs_f, W->ads_base, D.n);
-        CK(cudaMemsetAsync(W->s_val, 0, sizeof(float) * (D.M + kPad)));
+        if (algo == DG_PAGERANK) init_pr_kernel<<<g, 256>>>(W->vs_f, D.outdeg, D.vown, D.n, (float)S.param);
+        else init_ads_kernel<<<g, 256>>>(W->vs_f, W->ads_base, W->ads_pcont, D.vown, D.n);
         fill_iota_kernel<<<grid_1d(D.n_part), 256>>>(W->plist[0], D.n_part);
         int np = (int)D.n_part;
         CK(cudaMemcpy(&W->ctr->n_cur[0], &np, sizeof(int), cudaMemcpyHostToDevice));
@@ -1193,6 +1237,12 @@ int dev_upload_layout(DevLayout& D, const HostLayout& L, std::string& err) {
     if ((rc = dalloc(&D.vdst_ptr, D.n + 1, D.bytes, err))) return rc;
     if ((rc = dalloc(&D.vdst, L.vdst.size(), D.bytes, err))) return rc;
     if ((rc = dalloc(&D.bnd, D.n_bnd + 1, D.bytes, err))) return rc;
+    if ((rc = dalloc(&D.bnd_owner, D.n_bnd + 1, D.bytes, err))) return rc;
+    if ((rc = dalloc(&D.hpart, D.n + 1, D.bytes, err))) return rc;
+    if ((rc = dalloc(&D.vown, D.n + 1, D.bytes, err))) return rc;
+    if ((rc = h2d(D.bnd_owner, L.bnd_owner.data(), D.n_bnd, err))) return rc;
+    if ((rc = h2d(D.hpart, L.hpart.data(), D.n, err))) return rc;
+    if ((rc = h2d(D.vown, L.vown.data(), D.n, err))) return rc;
     CK(cudaMemset(D.e_idx + D.M, 0, sizeof(uint32_t) * kPad));
     CK(cudaMemset(D.e_w + D.M, 0, sizeof(int32_t) * kPad));
     if ((rc = h2d(D.e_idx, L.e_idx.data(), D.M, err))) return rc;
@@ -1210,6 +1260,7 @@ int dev_upload_layout(DevLayout& D, const HostLayout& L, std::string& err) {
 void dev_free_layout(DevLayout& D, bool csr_too) {
     dfree(D.e_idx); dfree(D.e_w); dfree(D.part_off);
     dfree(D.vsrc_ptr); dfree(D.vsrc); dfree(D.vdst_ptr); dfree(D.vdst); dfree(D.bnd);
+    dfree(D.bnd_owner); dfree(D.hpart); dfree(D.vown);
     if (csr_too) { dfree(D.row_ptr); dfree(D.col); dfree(D.w); dfree(D.outdeg); }
     D.bytes = 0;
     D.M = D.n_part = D.n_bnd = 0;
@@ -1217,9 +1268,9 @@ void dev_free_layout(DevLayout& D, bool csr_too) {
 
 void dev_free_work(DevWork*& W) {
     if (!W) return;
-    dfree(W->vs_u); dfree(W->vs_f); dfree(W->s_val); dfree(W->e_coef); dfree(W->ads_base); dfree(W->ads_pcont);
+    dfree(W->vs_u); dfree(W->vs_f); dfree(W->e_coef); dfree(W->ads_base); dfree(W->ads_pcont);
     dfree(W->part_flag); dfree(W->plist[0]); dfree(W->plist[1]); dfree(W->blockcnt); dfree(W->ctr);
-    dfree(W->bnd_base); dfree(W->dsum); dfree(W->scc_color); dfree(W->scc_label); dfree(W->scc_mark);
+    dfree(W->dsum); dfree(W->scc_color); dfree(W->scc_label); dfree(W->scc_mark);
     dfree(W->remaining);
     if (W->ev0) cudaEventDestroy(W->ev0);
     if (W->ev1) cudaEventDestroy(W->ev1);
@@ -1247,6 +1298,7 @@ int dev_set_vertex_params(DevWork*& W, const DevLayout& D, const double* p_inj, 
     CK(cudaMemset(W->e_coef, 0, sizeof(float) * (D.M + kPad)));
     if (D.w) {
         ads_coef_kernel<<<grid_1d(D.M), 256>>>(W->e_coef, D.e_idx, D.e_w, W->ads_pcont, wsum, D.M);
+        gfac_kernel<<<grid_1d(D.n), 256>>>(W->ads_pcont, wsum, D.n);
     } else {
         err = "Adsorption needs edge weights (load the CSR with weights)";
         cudaFree(wsum);
@@ -1300,8 +1352,6 @@ int dev_run_begin(DevWork*& W, const DevLayout& D, RunState& S, std::string& err
     if ((rc = ensure_work(W, D, err))) return rc;
     if (S.algo == DG_ADSORPTION && !W->have_params) { err = "Adsorption needs dg_set_vertex_params first"; return DG_EINVAL; }
     if ((rc = init_states(W, D, S, err))) return rc;
-    if ((S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION) && D.n_bnd)
-        init_base_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_f, D.bnd, D.n_bnd, W->bnd_base);
     CK(cudaGetLastError());
     CK(cudaEventRecord(W->ev0));
     return DG_OK;
@@ -1319,7 +1369,7 @@ int dev_rounds(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, 
 int dev_boundary_pack(DevWork* W, const DevLayout& D, RunState& S, void* buf, std::string& err) {
     if (!D.n_bnd) return DG_OK;
     if (S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION)
-        pack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_f, D.bnd, D.n_bnd, W->bnd_base, (float*)buf);
+        pack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_f, D.bnd, D.n_bnd, (float*)buf);
     else
         pack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, D.bnd, D.n_bnd, (uint32_t*)buf);
     S.stats.kernel_launches++;
@@ -1336,8 +1386,8 @@ int dev_boundary_unpack(DevWork* W, const DevLayout& D, RunState& S, const void*
     const int round = c.round;  // stamps of the next local round
     if (D.n_bnd) {
         if (S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION)
-            unpack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_f, D.bnd, D.n_bnd, W->bnd_base, (const float*)buf,
-                                                         (float)S.eps, round, D.vsrc_ptr, D.vsrc, W->part_flag);
+            unpack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_f, D.bnd, D.bnd_owner, D.n_bnd, (const float*)buf,
+                                                         (float)S.eps, D.hpart, W->part_flag);
         else
             unpack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, D.bnd, D.n_bnd, (const uint32_t*)buf, round,
                                                          D.vsrc_ptr, D.vsrc,
@@ -1376,10 +1426,9 @@ int dev_get_states(DevWork* W, const DevLayout& D, const RunState& S, void* out,
     }
     const int g = grid_1d(n);
     if (S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION) {
-        int vm = S.mode == DG_MODE_VERTEX;
         CK(cudaMemset(W->dsum, 0, sizeof(double)));
-        if (S.algo == DG_PAGERANK) sum_T_kernel<<<g, 256>>>(W->vs_f, n, vm, W->dsum);
-        out_pr_kernel<<<g, 256>>>(W->vs_f, n, vm, W->dsum, (float*)dst, S.algo == DG_PAGERANK);
+        if (S.algo == DG_PAGERANK) sum_T_kernel<<<g, 256>>>(W->vs_f, n, W->dsum);
+        out_pr_kernel<<<g, 256>>>(W->vs_f, n, W->dsum, (float*)dst, S.algo == DG_PAGERANK);
     } else if (S.algo == DG_SCC) {
         CK(cudaMemcpy(dst, W->scc_label, 4 * (size_t)n, cudaMemcpyDeviceToDevice));
     } else {

@@ -349,18 +349,33 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     const int64_t G = (int64_t)gpart_first.size() - 1;
     const int world = std::max(1, p.world), rank = p.rank;
 
-    // ---- boundary vertices: present in partitions of >1 rank (round-robin owner q % world)
+    // ---- boundary vertices: present in partitions of >1 rank (round-robin owner q % world);
+    // owner of a vertex = lowest rank holding it (rank 0 for vertices on no path)
+    L.vown.assign(n, world > 1 ? 0 : 1);
     if (world > 1) {
-        std::vector<uint64_t> mask(n, 0);
+        // present[v]: ranks whose partitions hold v.  touched[v]: ranks that can
+        // write v's state -- present, or (PageRank/Adsorption) an out-neighbour of
+        // a present vertex, since a firing vertex pushes along all its CSR edges.
+        std::vector<uint64_t> present(n, 0), touched;
         for (int64_t q = 0; q < G; q++) {
             uint64_t bit = 1ull << ((q % world) & 63);
             for (int64_t r = gpart_first[q]; r < gpart_first[q + 1]; r++) {
                 int64_t i = order[r];
-                for (int64_t k = moff[i]; k < moff[i + 1]; k++) mask[mv[k]] |= bit;
+                for (int64_t k = moff[i]; k < moff[i + 1]; k++) present[mv[k]] |= bit;
             }
         }
-        for (int64_t v = 0; v < n; v++)
-            if (__builtin_popcountll(mask[v]) > 1) L.boundary.push_back((int32_t)v);
+        touched = present;
+        for (int64_t u = 0; u < n; u++)
+            if (present[u])
+                for (int64_t e = g.row_ptr[u]; e < g.row_ptr[u + 1]; e++) touched[g.col[e]] |= present[u];
+        for (int64_t v = 0; v < n; v++) {
+            int owner = present[v] ? __builtin_ctzll(present[v]) : 0;
+            L.vown[v] = owner == rank;
+            if (__builtin_popcountll(touched[v]) > 1) {
+                L.boundary.push_back((int32_t)v);
+                L.bnd_owner.push_back(owner == rank);
+            }
+        }
     }
 
     // ---- this rank's layout
@@ -412,6 +427,9 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     };
     build_map(kTail, L.vsrc_ptr, L.vsrc);
     build_map(kHead, L.vdst_ptr, L.vdst);
+    L.hpart.assign(n, -1);
+    for (int64_t q = npart - 1; q >= 0; q--)
+        for (int64_t k = L.part_off[q]; k < L.part_off[q + 1]; k++) L.hpart[L.e_idx[k] & kVMask] = (int32_t)q;
 
     L.n_layers = n_layers;
     L.n_dep_sccs = n_dep_sccs;

@@ -1,0 +1,191 @@
+"""-m gpu: the CUDA path (through the C ABI) against the oracle, element by
+element, on the same seeded inputs.
+
+Bars (BASELINE.json north_star): SSSP / BFS / WCC / SCC bit-exact;
+PageRank (d = 0.85, fp32 states, per-vertex stop at delta < 1e-7) within
+L1 <= 1e-4 and per-vertex relative error <= 1e-3 of the oracle converged to
+residual 1e-12; Adsorption to the same bar.
+"""
+import numpy as np
+import pytest
+
+import inputs
+from oracle import algorithms as OA
+from paper_conf_asplos_zhangl0hlg19_b200 import DiGraph
+
+pytestmark = pytest.mark.gpu
+
+PR_L1, PR_REL = 1e-4, 1e-3
+
+
+@pytest.fixture(autouse=True)
+def _cuda(cuda_required):
+    pass
+
+
+def graphs_small():
+    return {
+        "rmat12": inputs.rmat(12, 4096, 40000, seed=11),
+        "uniform_dup": inputs.uniform(3000, 9000, seed=12, dedupe=False, drop_self=False),
+        "chains": inputs.chains(20000, 26000, chain_len=700, seed=13),
+        "rmat14": inputs.rmat(14, 1 << 14, 200000, seed=14),
+    }
+
+
+_G = {}
+
+
+def G(name):
+    if name not in _G:
+        if name == "rmat16":
+            _G[name] = inputs.make("rmat16")
+        else:
+            _G[name] = graphs_small()[name]
+    return _G[name]
+
+
+def engine(g, **kw):
+    dg = DiGraph()
+    dg.load_graph(g)
+    dg.build_paths(**kw)
+    return dg
+
+
+SSSP_CASES = [("rmat16", 0, {}), ("rmat12", 0, {}), ("rmat12", 77, {"part_entries": 64}),
+              ("uniform_dup", 5, {"l_merge": 0}), ("chains", 0, {"d_max": 64, "l_merge": 4096}),
+              ("rmat14", 0, {"order": "id", "n_sub": 7})]
+
+
+@pytest.mark.parametrize("name,source,kw", SSSP_CASES)
+@pytest.mark.parametrize("mode", ["path", "vertex"])
+def test_sssp_bit_exact(name, source, kw, mode):
+    g = G(name)
+    dg = engine(g, **kw)
+    st = dg.run("sssp", source=source, mode=mode)
+    got = dg.get_states().astype(np.int64)
+    src, dst, w = g.edges()
+    exp, _ = OA.sssp_bellman_ford(g.n, src, dst, w, source)
+    assert np.array_equal(got, exp), f"{np.sum(got != exp)} mismatches"
+    assert st["converged"]
+    assert (st["vertex_updates"] > 0) == bool((exp < OA.UNREACHED).sum() > 1)
+
+
+@pytest.mark.parametrize("name", ["rmat12", "chains"])
+@pytest.mark.parametrize("mode", ["path", "vertex"])
+def test_bfs_bit_exact(name, mode):
+    g = G(name)
+    dg = engine(g)
+    dg.run("bfs", source=0, mode=mode)
+    got = dg.get_states().astype(np.int64)
+    src, dst, _ = g.edges()
+    assert np.array_equal(got, OA.bfs_levels(g.n, src, dst, 0))
+
+
+def check_pr(got, exp):
+    l1 = np.abs(got.astype(np.float64) - exp).sum()
+    rel = np.abs(got.astype(np.float64) - exp) / exp
+    assert l1 <= PR_L1, l1
+    assert rel.max() <= PR_REL, rel.max()
+    return l1, rel.max()
+
+
+@pytest.mark.parametrize("name,kw", [("rmat12", {}), ("rmat14", {}), ("uniform_dup", {"part_entries": 100}),
+                                     ("chains", {"d_max": 64, "l_merge": 4096})])
+@pytest.mark.parametrize("mode", ["path", "vertex"])
+def test_pagerank_within_tolerance(name, kw, mode):
+    g = G(name)
+    dg = engine(g, **kw)
+    st = dg.run("pagerank", epsilon=1e-7, damping=0.85, mode=mode)
+    got = dg.get_states()
+    src, dst, _ = g.edges()
+    exp, _ = OA.pagerank_power(g.n, src, dst, d=0.85, tol=1e-12)
+    check_pr(got, exp)
+    assert abs(got.astype(np.float64).sum() - 1.0) < 1e-5
+    assert st["converged"]
+
+
+@pytest.mark.parametrize("name", ["rmat12", "uniform_dup", "chains"])
+def test_wcc_bit_exact(name):
+    g = G(name)
+    dg = engine(g)
+    dg.run("wcc")
+    got = dg.get_states().astype(np.int64)
+    src, dst, _ = g.edges()
+    exp, _ = OA.wcc_label_propagation(g.n, src, dst)
+    assert np.array_equal(got, exp)
+
+
+@pytest.mark.parametrize("name", ["rmat12", "uniform_dup", "chains"])
+def test_scc_bit_exact(name):
+    g = G(name)
+    dg = engine(g)
+    st = dg.run("scc")
+    got = dg.get_states().astype(np.int64)
+    src, dst, _ = g.edges()
+    exp = OA.scc_tarjan(g.n, src, dst)
+    assert np.array_equal(got, exp), f"{np.sum(got != exp)} mismatches"
+    assert st["outer_iterations"] >= 1
+
+
+@pytest.mark.parametrize("name", ["rmat12", "chains"])
+def test_adsorption_within_tolerance(name):
+    g = G(name)
+    dg = engine(g)
+    p_inj, p_cont, inj = inputs.adsorption_params(g.n, seed=3)
+    dg.set_vertex_params(p_inj, p_cont, inj)
+    dg.run("adsorption", epsilon=1e-7)
+    got = dg.get_states().astype(np.float64)
+    src, dst, w = g.edges()
+    exp, _ = OA.adsorption_jacobi(g.n, src, dst, w, p_inj, p_cont, inj, tol=1e-12)
+    scale = np.abs(exp).sum()
+    assert np.abs(got - exp).sum() / scale <= PR_L1
+    big = exp > 1e-3 * exp.mean()
+    assert (np.abs(got - exp)[big] / exp[big]).max() <= PR_REL
+
+
+def test_edge_cases():
+    # empty edge set, single vertex, self loop only, source with no out-edges
+    for n, e in [(1, []), (5, []), (3, [(1, 1)]), (4, [(1, 2), (2, 3)])]:
+        g = inputs.from_edges(n, [a for a, _ in e], [b for _, b in e], [3] * len(e))
+        dg = engine(g)
+        dg.run("sssp", source=0)
+        got = dg.get_states().astype(np.int64)
+        exp, _ = OA.sssp_bellman_ford(n, [a for a, _ in e], [b for _, b in e], [3] * len(e), 0)
+        assert np.array_equal(got, exp)
+        dg.run("pagerank")
+        pr = dg.get_states()
+        exp_pr, _ = OA.pagerank_power(n, np.array([a for a, _ in e], np.int64), np.array([b for _, b in e], np.int64))
+        assert np.abs(pr - exp_pr).sum() <= PR_L1
+        dg.run("wcc")
+        assert np.array_equal(dg.get_states(), OA.wcc_label_propagation(
+            n, np.array([a for a, _ in e], np.int64), np.array([b for _, b in e], np.int64))[0])
+
+
+def test_path_model_needs_fewer_updates_than_vertex_ablation():
+    g = G("rmat14")
+    dg = engine(g)
+    sp = dg.run("sssp", source=0, mode="path")
+    sv = dg.run("sssp", source=0, mode="vertex")
+    assert sp["vertex_updates"] <= sv["vertex_updates"], (sp, sv)
+
+
+def test_repeated_runs_are_independent():
+    g = G("rmat12")
+    dg = engine(g)
+    dg.run("pagerank")
+    a = dg.get_states().copy()
+    dg.run("sssp", source=3)
+    dg.run("pagerank")
+    b = dg.get_states()
+    check_pr(b, a.astype(np.float64))
+
+
+def test_states_into_device_buffer():
+    import torch
+    g = G("rmat12")
+    dg = engine(g)
+    dg.run("sssp", source=0)
+    host = dg.get_states()
+    dev = torch.empty(g.n, dtype=torch.int32, device="cuda")
+    dg.get_states(dev)
+    assert np.array_equal(dev.cpu().numpy().view(np.uint32), host)
