@@ -68,10 +68,13 @@ typedef struct {
     int32_t part_entries;  /* target path entries per partition (scheduling unit) */
     int32_t rank;          /* this process's rank for multi-GPU path partitioning */
     int32_t world;         /* number of ranks (1 = single GPU) */
+    int32_t merge_rule;    /* 0: paper-literal (no merge through a line-13 inner vertex of
+                              in/out degree > 1); 1: relaxed (any head-to-tail merge within
+                              l_merge; reading R-MERGE) */
 } dg_path_params;
 
 /* Fill *p with the defaults (d_max 16, l_merge 64, n_sub 64, order 0,
- * hot_factor 2, part_entries 2048, rank 0, world 1). */
+ * hot_factor 2, part_entries 2048, rank 0, world 1, merge_rule 1). */
 void dg_default_params(dg_path_params *p);
 
 /* Statistics of one dg_run (device-side counters). */
@@ -83,6 +86,9 @@ typedef struct {
     int64_t units_processed;      /* partitions (path) / vertices (vertex) dispatched */
     int64_t kernel_launches;      /* kernels launched by this run                  */
     int64_t outer_iterations;     /* SCC colouring iterations (0 otherwise)        */
+    int64_t entries_processed;    /* path entries walked (path mode)               */
+    int64_t csr_edges;            /* CSR out-edges pushed (delta algorithms, ablation) */
+    double kernel_ms;             /* device time of the propagation kernels only   */
 } dg_run_stats;
 
 /* Static description of the built layout (sizes; for tests and benchmarks). */

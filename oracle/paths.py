@@ -133,33 +133,74 @@ def merge_short_paths(n, src, dst, paths, inner, l_max):
     a head-to-tail way ... if both in-degree and out-degree of their
     intersected vertex are more than one, they are merged only when their
     intersected vertex is not an inner vertex".  DESIGN.md reading R-MERGE:
-    paths are visited in order; path i repeatedly absorbs the lowest-indexed
-    unabsorbed path j != i whose head is i's tail, while the merged edge count
-    stays <= l_max."""
+
+      1. at every vertex x where merging is allowed, the k-th path (by index)
+         ending at x is linked to the k-th path starting at x; a path is never
+         linked to itself (a closed path swaps with the next starter);
+      2. links form chains and cycles; each cycle is cut before its
+         lowest-indexed path;
+      3. every chain is walked from its start and cut into merged paths of at
+         most l_max edges (a piece that does not fit starts a new path);
+      4. merged paths are ordered by the index of their first piece.
+
+    ``inner`` holds the line-13 vertices for the paper-literal rule, or is
+    empty for the relaxed rule."""
     indeg, outdeg = _degrees(n, np.asarray(src), np.asarray(dst))
-    paths = [list(p) for p in paths]
-    absorbed = [False] * len(paths)
-    by_head = defaultdict(list)
-    for j, p in enumerate(paths):
-        by_head[p[0]].append(j)
-    for i in range(len(paths)):
-        if absorbed[i]:
+    P = len(paths)
+    ends, starts = defaultdict(list), defaultdict(list)
+    for i, p in enumerate(paths):
+        ends[p[-1]].append(i)
+        starts[p[0]].append(i)
+    nxt, prv = [-1] * P, [-1] * P
+    for x in sorted(set(ends) & set(starts)):
+        if indeg[x] > 1 and outdeg[x] > 1 and x in inner:
             continue
-        while True:
-            x = paths[i][-1]
-            if indeg[x] > 1 and outdeg[x] > 1 and x in inner:
-                break
-            pick = None
-            for j in by_head.get(x, []):
-                if j != i and not absorbed[j] and \
-                        (len(paths[i]) - 1) + (len(paths[j]) - 1) <= l_max:
-                    pick = j
-                    break
-            if pick is None:
-                break
-            paths[i] = paths[i] + paths[pick][1:]
-            absorbed[pick] = True
-    return [p for j, p in enumerate(paths) if not absorbed[j]]
+        A, B = ends[x], list(starts[x])
+        for k in range(min(len(A), len(B))):
+            if A[k] == B[k]:
+                if k + 1 < len(B):
+                    B[k], B[k + 1] = B[k + 1], B[k]
+                else:
+                    continue
+            nxt[A[k]], prv[B[k]] = B[k], A[k]
+    seen = [False] * P
+    chains = []
+    for i in range(P):                      # chains: start where nothing links in
+        if prv[i] == -1:
+            c, j = [], i
+            while j != -1:
+                seen[j] = True
+                c.append(j)
+                j = nxt[j]
+            chains.append(c)
+    for i in range(P):                      # cycles: cut before the lowest index
+        if not seen[i]:
+            c, j = [], i
+            while not seen[j]:
+                seen[j] = True
+                c.append(j)
+                j = nxt[j]
+            chains.append(c)
+    segs = []
+    for c in chains:
+        cur, cur_len = [], 0
+        for j in c:
+            e = len(paths[j]) - 1
+            if cur and cur_len + e > l_max:
+                segs.append(cur)
+                cur, cur_len = [], 0
+            cur.append(j)
+            cur_len += e
+        if cur:
+            segs.append(cur)
+    segs.sort(key=lambda sg: sg[0])
+    out = []
+    for sg in segs:
+        p = list(paths[sg[0]])
+        for j in sg[1:]:
+            p += paths[j][1:]
+        out.append(p)
+    return out
 
 
 def path_stats(n, src, dst, paths, hot_factor=2.0):

@@ -30,14 +30,16 @@ EXPORTS = [
 class dg_path_params(ctypes.Structure):
     _fields_ = [("d_max", ctypes.c_int32), ("l_merge", ctypes.c_int32), ("n_sub", ctypes.c_int32),
                 ("order", ctypes.c_int32), ("hot_factor", ctypes.c_float),
-                ("part_entries", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32)]
+                ("part_entries", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
+                ("merge_rule", ctypes.c_int32)]
 
 
 class dg_run_stats(ctypes.Structure):
     _fields_ = [("time_ms", ctypes.c_double), ("rounds", ctypes.c_int64),
                 ("vertex_updates", ctypes.c_int64), ("edges_processed", ctypes.c_int64),
                 ("units_processed", ctypes.c_int64), ("kernel_launches", ctypes.c_int64),
-                ("outer_iterations", ctypes.c_int64)]
+                ("outer_iterations", ctypes.c_int64), ("entries_processed", ctypes.c_int64),
+                ("csr_edges", ctypes.c_int64), ("kernel_ms", ctypes.c_double)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -46,6 +46,7 @@ void dg_default_params(dg_path_params* p) {
     p->part_entries = 2048;
     p->rank = 0;
     p->world = 1;
+    p->merge_rule = 1;
 }
 
 int dg_create(dg_graph** out, int device) {
@@ -108,7 +109,7 @@ int dg_build_paths(dg_graph* g, const dg_path_params* p) {
     dg_default_params(&q);
     if (p) q = *p;
     if (q.d_max < 1 || q.n_sub < 1 || q.part_entries < 1 || q.world < 1 || q.world > 64 ||
-        q.rank < 0 || q.rank >= q.world || q.l_merge < 0)
+        q.rank < 0 || q.rank >= q.world || q.l_merge < 0 || q.merge_rule < 0 || q.merge_rule > 1)
         return fail(DG_EINVAL, "dg_build_paths: bad parameters");
     try {
         dg::build_layout(g->csr, q, g->layout);

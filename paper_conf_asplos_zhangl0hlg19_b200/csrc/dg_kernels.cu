@@ -48,7 +48,7 @@ constexpr int kWarps = kBlock / 32;
 constexpr int kPad = 256;  // entries of zero padding after the layout arrays
 
 struct Counters {
-    unsigned long long updates, edges, units;
+    unsigned long long updates, edges, units, entries, pushes;
     int n_cur[2];
     unsigned int ticket[2];
     int round;  // global round number (stamps are round+1)
@@ -73,7 +73,7 @@ struct DevWork {
     int32_t* scc_label = nullptr;
     uint8_t* scc_mark = nullptr;
     int32_t* remaining = nullptr;
-    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr, kev0 = nullptr, kev1 = nullptr;
     bool have_params = false;
 };
 
@@ -158,7 +158,7 @@ __device__ __forceinline__ void flag_partitions(uint32_t mask, int v, const int6
 }
 
 struct Acc {
-    unsigned long long upd = 0, edges = 0, units = 0;
+    unsigned long long upd = 0, edges = 0, units = 0, entries = 0, pushes = 0;
 };
 
 // ------------------------------------------------------------------ path walks
@@ -249,6 +249,7 @@ __device__ void walk_minplus(const KParams& P, int64_t beg, int64_t end, int rou
         for (int k = 0; k < 4; k++) {
             sig[k] = false;
             if (valid[k]) {
+                acc.entries++;
                 if (!(u4get(code, k) & kHead)) acc.edges++;
                 if (val[k] < a[k]) {
                     uint32_t old = atomicMin(&P.vs_u[vtx[k]].x, val[k]);
@@ -342,6 +343,7 @@ __device__ void walk_delta(const KParams& P, int64_t beg, int64_t end, Acc& acc)
             prev = al[k] + be[k] * prev;
             f[k] = dl[k] + pin;
             fire[k] = valid[k] && f[k] > 0.f;
+            if (valid[k]) acc.entries++;
             if (valid[k] && !hd[k]) acc.edges++;
             if (fire[k]) {
                 atomicAdd(&P.vs_f[vtx[k]].x, f[k]);
@@ -406,7 +408,7 @@ __device__ void walk_delta(const KParams& P, int64_t beg, int64_t end, Acc& acc)
                 const int hp = P.hpart[x];
                 if (hp >= 0) P.part_flag[hp] = 1;  // -1: x lives on another rank (multi-GPU sync delivers it)
             }
-            acc.edges++;
+            acc.pushes++;
         }
         __syncwarp();
     }
@@ -461,6 +463,7 @@ __device__ void walk_scc_fwd(const KParams& P, int64_t beg, int64_t end, int rou
         for (int k = 0; k < 4; k++) {
             sig[k] = false;
             if (!live[k]) continue;
+            acc.entries++;
             if (!(u4get(code, k) & kHead)) acc.edges++;
             if (val[k] < a[k]) {
                 uint32_t old = atomicMin(&P.vs_u[vtx[k]].x, val[k]);
@@ -551,6 +554,7 @@ __device__ void walk_scc_bwd(const KParams& P, int64_t beg, int64_t end, int rou
         for (int k = 0; k < 4; k++) {
             sig[k] = false;
             if (!live[k]) continue;
+            acc.entries++;
             if (!tl[k]) acc.edges++;
             if (newm[k] && !mk[k]) {
                 // byte flag: plain store is idempotent
@@ -660,11 +664,15 @@ __global__ void __launch_bounds__(kBlock) path_kernel(KParams P) {
     for (int off = 16; off; off >>= 1) {
         acc.upd += __shfl_xor_sync(0xffffffffu, acc.upd, off);
         acc.edges += __shfl_xor_sync(0xffffffffu, acc.edges, off);
+        acc.entries += __shfl_xor_sync(0xffffffffu, acc.entries, off);
+        acc.pushes += __shfl_xor_sync(0xffffffffu, acc.pushes, off);
     }
     if (lane == 0) {
         atomicAdd(&P.ctr->updates, acc.upd);
         atomicAdd(&P.ctr->edges, acc.edges);
         atomicAdd(&P.ctr->units, acc.units);
+        atomicAdd(&P.ctr->entries, acc.entries);
+        atomicAdd(&P.ctr->pushes, acc.pushes);
     }
     grid.sync();
     if (blockIdx.x == 0 && threadIdx.x == 0) P.ctr->round += r;
@@ -733,7 +741,7 @@ __global__ void __launch_bounds__(kBlock) vertex_kernel(KParams P) {
                 const int u = s_v[wid][lo];
                 const int64_t e = P.row_ptr[u] + (j - s_off[wid][lo]);
                 const int x = P.col[e];
-                acc.edges++;
+                acc.pushes++;
                 bool push = false;
                 if (ALGO == DG_PAGERANK) {
                     float a = s_push[wid][lo];
@@ -764,11 +772,13 @@ __global__ void __launch_bounds__(kBlock) vertex_kernel(KParams P) {
         acc.upd += __shfl_xor_sync(0xffffffffu, acc.upd, off);
         acc.edges += __shfl_xor_sync(0xffffffffu, acc.edges, off);
         acc.units += __shfl_xor_sync(0xffffffffu, acc.units, off);
+        acc.pushes += __shfl_xor_sync(0xffffffffu, acc.pushes, off);
     }
     if (lane == 0) {
         atomicAdd(&P.ctr->updates, acc.upd);
         atomicAdd(&P.ctr->edges, acc.edges);
         atomicAdd(&P.ctr->units, acc.units);
+        atomicAdd(&P.ctr->pushes, acc.pushes);
     }
     grid.sync();
     if (blockIdx.x == 0 && threadIdx.x == 0) P.ctr->round += r;
@@ -1001,6 +1011,8 @@ int ensure_work(DevWork*& W, const DevLayout& D, std::string& err) {
     CK(cudaMemset(W->part_flag, 0, D.n_part + 1));
     CK(cudaEventCreate(&W->ev0));
     CK(cudaEventCreate(&W->ev1));
+    CK(cudaEventCreate(&W->kev0));
+    CK(cudaEventCreate(&W->kev1));
     return DG_OK;
 }
 
@@ -1039,8 +1051,14 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, float ep
         CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, kBlock, 0));
         grid = sms * std::max(1, per);
     }
+    CK(cudaEventRecord(W->kev0));
     CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kBlock), args, 0, 0));
     CK(cudaGetLastError());
+    CK(cudaEventRecord(W->kev1));
+    CK(cudaEventSynchronize(W->kev1));
+    float kms = 0;
+    CK(cudaEventElapsedTime(&kms, W->kev0, W->kev1));
+    S.stats.kernel_ms += kms;
     S.stats.kernel_launches++;
     return DG_OK;
 }
@@ -1057,8 +1075,14 @@ int launch_vertex(DevWork* W, const DevLayout& D, int algo, int rounds, float ep
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, kBlock, 0));
     int grid = sms * std::max(1, per);
+    CK(cudaEventRecord(W->kev0));
     CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kBlock), args, 0, 0));
     CK(cudaGetLastError());
+    CK(cudaEventRecord(W->kev1));
+    CK(cudaEventSynchronize(W->kev1));
+    float kms = 0;
+    CK(cudaEventElapsedTime(&kms, W->kev0, W->kev1));
+    S.stats.kernel_ms += kms;
     S.stats.kernel_launches++;
     return DG_OK;
 }
@@ -1117,8 +1141,10 @@ int collect_stats(DevWork* W, RunState& S, std::string& err) {
     S.stats.rounds += c.round - (int)S.round;
     S.round = c.round;
     S.stats.vertex_updates = (int64_t)c.updates;
-    S.stats.edges_processed = (int64_t)c.edges;
+    S.stats.edges_processed = (int64_t)(c.edges + c.pushes);
     S.stats.units_processed = (int64_t)c.units;
+    S.stats.entries_processed = (int64_t)c.entries;
+    S.stats.csr_edges = (int64_t)c.pushes;
     return DG_OK;
 }
 
@@ -1186,6 +1212,7 @@ int run_scc(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, std
     S.stats.vertex_updates = (int64_t)cf.updates;
     S.stats.edges_processed = (int64_t)cf.edges;
     S.stats.units_processed = (int64_t)cf.units;
+    S.stats.entries_processed = (int64_t)cf.entries;
     return DG_OK;
 }
 
@@ -1274,6 +1301,8 @@ void dev_free_work(DevWork*& W) {
     dfree(W->remaining);
     if (W->ev0) cudaEventDestroy(W->ev0);
     if (W->ev1) cudaEventDestroy(W->ev1);
+    if (W->kev0) cudaEventDestroy(W->kev0);
+    if (W->kev1) cudaEventDestroy(W->kev1);
     delete W;
     W = nullptr;
 }

@@ -11,6 +11,8 @@
 #include <algorithm>
 #include <atomic>
 #include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <numeric>
 #include <stdexcept>
@@ -124,6 +126,15 @@ int64_t tarjan(int64_t N, const std::vector<int64_t>& ptr, const std::vector<int
 
 void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     auto t0 = std::chrono::steady_clock::now();
+    auto tp = t0;
+    const bool verbose = std::getenv("DG_VERBOSE") != nullptr;
+    auto phase = [&](const char* name) {
+        auto now = std::chrono::steady_clock::now();
+        if (verbose)
+            std::fprintf(stderr, "[dg_build_paths] %-22s %9.1f ms\n", name,
+                         std::chrono::duration<double, std::milli>(now - tp).count());
+        tp = now;
+    };
     const int64_t n = g.n, m = g.m;
     L = HostLayout();
     L.params = p;
@@ -150,6 +161,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
         for (int64_t i = b; i < e; i++) { scol[i] = tmp[i - b].first; sw[i] = tmp[i - b].second; }
     }
 
+    phase("sort successors");
     // ---- subgraphs: contiguous vertex ranges of ~m/T out-edges (reading R-SUB)
     const int T = std::max(1, p.n_sub);
     std::vector<int64_t> bounds(T + 1, 0);
@@ -183,6 +195,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
         D.new_path();
     }
 
+    phase("algorithm 1");
     // ---- concatenate (subgraph order)
     std::vector<int64_t> poff{0};
     std::vector<int32_t> pv, pw;
@@ -201,58 +214,94 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     const int64_t P0 = (int64_t)poff.size() - 1;
     L.paths_before_merge = P0;
 
-    // ---- short-path merging (reading R-MERGE)
-    std::vector<int64_t> nxt(P0, -1), last(P0), clen(P0);
-    std::vector<uint8_t> absorbed(P0, 0);
-    for (int64_t i = 0; i < P0; i++) { last[i] = i; clen[i] = poff[i + 1] - poff[i] - 1; }
+    phase("concatenate");
+    // ---- short-path merging (reading R-MERGE):
+    // pair the k-th path ending at x with the k-th path starting at x, cut
+    // cycles before their lowest index, cut chains into <= l_merge edges,
+    // order merged paths by their first piece.
+    std::vector<int64_t> nxt(P0, -1), prv(P0, -1);
     if (p.l_merge > 0 && P0 > 1) {
-        std::vector<int64_t> hptr(n + 1, 0), hlist(P0), cursor(n);
-        for (int64_t i = 0; i < P0; i++) hptr[pv[poff[i]] + 1]++;
-        for (int64_t v = 0; v < n; v++) hptr[v + 1] += hptr[v];
-        for (int64_t v = 0; v < n; v++) cursor[v] = hptr[v];
+        std::vector<int64_t> eptr(n + 1, 0), sptr(n + 1, 0), elist(P0), slist(P0);
+        for (int64_t i = 0; i < P0; i++) { eptr[pv[poff[i + 1] - 1] + 1]++; sptr[pv[poff[i]] + 1]++; }
+        for (int64_t v = 0; v < n; v++) { eptr[v + 1] += eptr[v]; sptr[v + 1] += sptr[v]; }
         {
-            std::vector<int64_t> fill(hptr.begin(), hptr.end() - 1);
-            for (int64_t i = 0; i < P0; i++) hlist[fill[pv[poff[i]]]++] = i;
+            std::vector<int64_t> fe(eptr.begin(), eptr.end() - 1), fs(sptr.begin(), sptr.end() - 1);
+            for (int64_t i = 0; i < P0; i++) { elist[fe[pv[poff[i + 1] - 1]]++] = i; slist[fs[pv[poff[i]]]++] = i; }
         }
-        for (int64_t i = 0; i < P0; i++) {
-            if (absorbed[i]) continue;
-            while (true) {
-                int64_t lp = last[i];
-                int32_t x = pv[poff[lp + 1] - 1];
-                if (g.indeg[x] > 1 && g.outdeg[x] > 1 && inner[x]) break;
-                int64_t pick = -1;
-                while (cursor[x] < hptr[x + 1] && absorbed[hlist[cursor[x]]]) cursor[x]++;
-                for (int64_t k = cursor[x]; k < hptr[x + 1]; k++) {
-                    int64_t j = hlist[k];
-                    if (j == i || absorbed[j]) continue;
-                    if (clen[i] + clen[j] <= p.l_merge) { pick = j; break; }
+        #pragma omp parallel for schedule(dynamic, 4096)
+        for (int64_t x = 0; x < n; x++) {
+            const int64_t na = eptr[x + 1] - eptr[x], nb = sptr[x + 1] - sptr[x];
+            if (!na || !nb) continue;
+            if (p.merge_rule == 0 && g.indeg[x] > 1 && g.outdeg[x] > 1 && inner[x]) continue;
+            int64_t* A = &elist[eptr[x]];
+            int64_t* B = &slist[sptr[x]];
+            for (int64_t k = 0; k < std::min(na, nb); k++) {
+                if (A[k] == B[k]) {
+                    if (k + 1 < nb) std::swap(B[k], B[k + 1]);
+                    else continue;
                 }
-                if (pick < 0) break;
-                nxt[last[i]] = pick;
-                last[i] = last[pick];
-                clen[i] += clen[pick];
-                absorbed[pick] = 1;
+                nxt[A[k]] = B[k];
+                prv[B[k]] = A[k];
             }
         }
     }
-    // materialise merged paths (merge order)
-    std::vector<int64_t> moff{0};
-    std::vector<int32_t> mv, mw;
-    mv.reserve(pv.size()); mw.reserve(pv.size());
-    for (int64_t i = 0; i < P0; i++) {
-        if (absorbed[i]) continue;
+    // chains (start where nothing links in), then cycles cut before their lowest index
+    std::vector<uint8_t> seen(P0, 0);
+    std::vector<int64_t> seg_first, seg_len;   // segments: first piece, #pieces
+    std::vector<int64_t> seg_pieces;           // pieces in chain order, segments contiguous per chain
+    auto walk_chain = [&](int64_t s0, std::vector<int64_t>& pieces, std::vector<int64_t>& sf, std::vector<int64_t>& sl) {
+        int64_t cur_len = 0, cur_n = 0;
+        for (int64_t j = s0; j != -1 && !seen[j]; j = nxt[j]) {
+            seen[j] = 1;
+            const int64_t e = poff[j + 1] - poff[j] - 1;
+            if (cur_n && cur_len + e > p.l_merge) { sl.push_back(cur_n); cur_n = 0; cur_len = 0; }
+            if (!cur_n) sf.push_back(j);
+            pieces.push_back(j);
+            cur_n++; cur_len += e;
+        }
+        if (cur_n) sl.push_back(cur_n);
+    };
+    {
+        const int nth = omp_get_max_threads();
+        std::vector<std::vector<int64_t>> tp(nth), tf(nth), tl(nth);
+        #pragma omp parallel for schedule(dynamic, 4096)
+        for (int64_t i = 0; i < P0; i++)
+            if (prv[i] == -1) { int t = omp_get_thread_num(); walk_chain(i, tp[t], tf[t], tl[t]); }
+        for (int t = 0; t < nth; t++) {
+            seg_pieces.insert(seg_pieces.end(), tp[t].begin(), tp[t].end());
+            seg_first.insert(seg_first.end(), tf[t].begin(), tf[t].end());
+            seg_len.insert(seg_len.end(), tl[t].begin(), tl[t].end());
+        }
+        for (int64_t i = 0; i < P0; i++)
+            if (!seen[i]) walk_chain(i, seg_pieces, seg_first, seg_len);
+    }
+    const int64_t P = (int64_t)seg_first.size();
+    std::vector<int64_t> seg_start(P + 1, 0);   // into seg_pieces
+    for (int64_t s2 = 0; s2 < P; s2++) seg_start[s2 + 1] = seg_start[s2] + seg_len[s2];
+    std::vector<int64_t> sorder(P);
+    std::iota(sorder.begin(), sorder.end(), 0);
+    std::sort(sorder.begin(), sorder.end(), [&](int64_t a, int64_t b) { return seg_first[a] < seg_first[b]; });
+    // materialise merged paths (merge order) in parallel
+    std::vector<int64_t> moff(P + 1, 0);
+    for (int64_t r = 0; r < P; r++) {
+        int64_t sgi = sorder[r], len = 1;
+        for (int64_t q = seg_start[sgi]; q < seg_start[sgi + 1]; q++) len += poff[seg_pieces[q] + 1] - poff[seg_pieces[q]] - 1;
+        moff[r + 1] = moff[r] + len;
+    }
+    std::vector<int32_t> mv(moff[P]), mw(moff[P]);
+    #pragma omp parallel for schedule(dynamic, 1024)
+    for (int64_t r = 0; r < P; r++) {
+        int64_t sgi = sorder[r], o = moff[r];
         bool first = true;
-        for (int64_t c = i; c >= 0; c = nxt[c]) {
-            for (int64_t k = poff[c] + (first ? 0 : 1); k < poff[c + 1]; k++) {
-                mv.push_back(pv[k]); mw.push_back(pw[k]);
-            }
+        for (int64_t q = seg_start[sgi]; q < seg_start[sgi + 1]; q++) {
+            int64_t c = seg_pieces[q];
+            for (int64_t k = poff[c] + (first ? 0 : 1); k < poff[c + 1]; k++) { mv[o] = pv[k]; mw[o] = pw[k]; o++; }
             first = false;
         }
-        moff.push_back((int64_t)mv.size());
     }
     { std::vector<int32_t>().swap(pv); std::vector<int32_t>().swap(pw); }
-    const int64_t P = (int64_t)moff.size() - 1;
 
+    phase("merge");
     // ---- path statistics (reading R-HOT)
     std::vector<double> dbar(P);
     std::vector<int64_t> nvert(P);
@@ -267,6 +316,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
         hot[i] = dbar[i] >= (double)p.hot_factor * mean_deg;
     }
 
+    phase("path stats");
     // ---- dependency graph G' as a bipartite path/vertex graph (reading R-DEP):
     // path node i -> vertex node P+x for every x entered by an edge of i;
     // vertex node P+x -> path node j for every x left by an edge of j.
@@ -324,6 +374,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     }
     { std::vector<int64_t>().swap(adj); std::vector<int64_t>().swap(aptr); }
 
+    phase("dependency DAG");
     // ---- priority Pri(p) = alpha*D(p)*N(p) - L(p)
     double dmax = 0; int64_t nmax = 0;
     for (int64_t i = 0; i < P; i++) { dmax = std::max(dmax, dbar[i]); nmax = std::max(nmax, nvert[i]); }
@@ -378,6 +429,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
         }
     }
 
+    phase("priority+partitions");
     // ---- this rank's layout
     L.part_off.push_back(0);
     L.path_off.push_back(0);
@@ -427,6 +479,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     };
     build_map(kTail, L.vsrc_ptr, L.vsrc);
     build_map(kHead, L.vdst_ptr, L.vdst);
+    phase("layout+maps");
     L.hpart.assign(n, -1);
     for (int64_t q = npart - 1; q >= 0; q--)
         for (int64_t k = L.part_off[q]; k < L.part_off[q + 1]; k++) L.hpart[L.e_idx[k] & kVMask] = (int32_t)q;

@@ -26,10 +26,12 @@ def test_library_exports_every_header_symbol():
     assert sorted(_abi.EXPORTS) == declared
 
 
-def oracle_layout(g, d_max, n_sub, order, l_merge):
+def oracle_layout(g, d_max, n_sub, order, l_merge, rule="relaxed"):
     src, dst, _ = g.edges()
     paths, inner = OP.graphp_decompose(g.n, g.row_ptr, g.col, d_max=d_max, n_sub=n_sub, order=order)
-    merged = OP.merge_short_paths(g.n, src, dst, paths, inner, l_max=l_merge) if l_merge else paths
+    # reading R-MERGE: "relaxed" ignores the inner-vertex constraint (oracle: inner = {})
+    inner_used = inner if rule == "paper" else set()
+    merged = OP.merge_short_paths(g.n, src, dst, paths, inner_used, l_max=l_merge) if l_merge else paths
     dep = OP.dependency_graph(merged)
     scc, layer = OP.condense_and_layer(len(merged), dep)
     dbar, nv, hot = OP.path_stats(g.n, src, dst, merged, hot_factor=2.0)
@@ -37,10 +39,11 @@ def oracle_layout(g, d_max, n_sub, order, l_merge):
     return paths, merged, scc, layer, hot, pri
 
 
-def product_layout(g, d_max, n_sub, order, l_merge, part_entries=64):
+def product_layout(g, d_max, n_sub, order, l_merge, part_entries=64, rule="relaxed"):
     dg = DiGraph()
     dg.load_graph(g)
-    dg.build_paths(d_max=d_max, l_merge=l_merge, n_sub=n_sub, order=order, part_entries=part_entries)
+    dg.build_paths(d_max=d_max, l_merge=l_merge, n_sub=n_sub, order=order, part_entries=part_entries,
+                   merge_rule=rule)
     return dg, dg.export_paths(), dg.layout_info()
 
 
@@ -70,15 +73,15 @@ def test_product_reproduces_figure4_layout():
     assert info["n_layers"] == 3 and info["n_dep_sccs"] == 3 and info["giant_scc_paths"] == 2
 
 
-CASES = list(itertools.product([0, 1, 2], [1, 3], ["degree", "id"], [0, 64], [16, 3]))
+CASES = list(itertools.product([0, 1, 2], [1, 3], ["degree", "id"], [0, 64], [16, 3], ["paper", "relaxed"]))
 
 
-@pytest.mark.parametrize("seed,n_sub,order,l_merge,d_max", CASES)
-def test_product_preprocessing_matches_oracle(seed, n_sub, order, l_merge, d_max):
+@pytest.mark.parametrize("seed,n_sub,order,l_merge,d_max,rule", CASES)
+def test_product_preprocessing_matches_oracle(seed, n_sub, order, l_merge, d_max, rule):
     g = inputs.rmat(9, 400, 2500, seed=seed, weights=(1, 9)) if seed != 2 else \
         inputs.uniform(300, 1200, seed=seed, weights=(1, 9))
-    o_paths, o_merged, o_scc, o_layer, o_hot, o_pri = oracle_layout(g, d_max, n_sub, order, l_merge)
-    dg, ex, info = product_layout(g, d_max, n_sub, order, l_merge)
+    o_paths, o_merged, o_scc, o_layer, o_hot, o_pri = oracle_layout(g, d_max, n_sub, order, l_merge, rule)
+    dg, ex, info = product_layout(g, d_max, n_sub, order, l_merge, rule=rule)
     assert info["paths_before_merge"] == len(o_paths)
     paths = split(ex)
     midx = ex["merged_index"]

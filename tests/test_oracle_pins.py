@@ -315,8 +315,11 @@ def test_merge_respects_inner_constraint():
     assert out == [[0, 2], [2, 4], [2, 5], [3, 1, 2]]
     out2 = P.merge_short_paths(n, src, dst, paths, inner=set(), l_max=64)
     assert out2 == [[0, 2, 4], [3, 1, 2, 5]]
+    # links by hand: at x=1 path4->path2; at x=2 (ends [0,2], starts [1,3])
+    # path0->path1, path2->path3.  Chains [0,1] and [4,2,3]; the cap of 2 edges
+    # cuts the second after [3,1,2]; segments ordered by first piece 0, 3, 4.
     out3 = P.merge_short_paths(n, src, dst, paths, inner=set(), l_max=2)
-    assert out3 == [[0, 2, 4], [1, 2, 5], [3, 1]]   # length cap blocks the last merge
+    assert out3 == [[0, 2, 4], [2, 5], [3, 1, 2]]
 
 
 # ------------------------------------------------------------------ dependency DAG
