@@ -83,7 +83,7 @@ typedef struct {
     int64_t rounds;               /* rounds until the active counter reached zero  */
     int64_t vertex_updates;       /* master-state changes (successful relax/fold)  */
     int64_t edges_processed;      /* path edges (or CSR edges) walked              */
-    int64_t units_processed;      /* partitions (path) / vertices (vertex) dispatched */
+    int64_t units_processed;      /* 128-entry windows walked (path) / vertices expanded (vertex) */
     int64_t kernel_launches;      /* kernels launched by this run                  */
     int64_t outer_iterations;     /* SCC colouring iterations (0 otherwise)        */
     int64_t entries_processed;    /* path entries walked (path mode)               */
@@ -105,6 +105,7 @@ typedef struct {
     int64_t paths_before_merge;   /* paths produced by Algorithm 1                  */
     double preprocess_ms;         /* host time of dg_build_paths                    */
     int64_t device_bytes;         /* device memory held by the layout               */
+    int64_t h2d_bytes;            /* bytes the last dg_upload copied host -> device */
 } dg_layout_info;
 
 /* Create an empty graph bound to CUDA device `device` (cudaSetDevice is
@@ -166,11 +167,18 @@ int dg_run(dg_graph *g, int algo, int64_t source, double epsilon, double param,
 
 /* Copy the final states of the last dg_run into `out` (n elements):
  *   SSSP/BFS      uint32 distances (DG_INF unreachable)
- *   PAGERANK      float32 ranks normalised to sum 1 (reading R-PR)
+ *   PAGERANK      float32 ranks normalised to sum 1 (reading R-PR);
+ *                 after a multi-rank run (world > 1): this rank's unnormalised
+ *                 totals -- take the MAX over ranks (totals grow monotonically
+ *                 from the same initial value), then dg_normalize_states
  *   ADSORPTION    float32 scores x_v
  *   WCC / SCC     int32 label = smallest vertex id of the component
  *   out_is_device 0: `out` is HOST memory; 1: DEVICE memory. */
 int dg_get_states(dg_graph *g, void *out, int64_t n, int out_is_device);
+
+/* Normalise a DEVICE float32[n] buffer in place to sum 1 (the last step of a
+ * multi-rank PageRank after the contributions were summed over ranks). */
+int dg_normalize_states(dg_graph *g, void *buf, int64_t n);
 
 /* Layout sizes / preprocessing time. */
 int dg_get_layout_info(const dg_graph *g, dg_layout_info *info);
@@ -194,8 +202,9 @@ int dg_export_paths(const dg_graph *g, int64_t *path_off, int32_t *vertices, int
  * PageRank/Adsorption); dg_boundary_unpack } until the all-reduced active
  * count is zero; dg_run_end. */
 
-/* Number of boundary vertices and the buffer element type of this rank:
- * *elem_bytes = 4 (uint32 for MIN algorithms, float32 for SUM algorithms). */
+/* Number of boundary vertices (vertices on more than one rank's paths).
+ * Buffer elements: uint32 (as int32) for MIN algorithms, uint64 fixed-point
+ * (2^-32 units, as int64) for SUM algorithms. */
 int dg_boundary_size(const dg_graph *g, int64_t *n_boundary);
 
 /* Export the boundary vertex ids (HOST int32[n_boundary], ascending). */
@@ -207,10 +216,10 @@ int dg_run_begin(dg_graph *g, int algo, int64_t source, double epsilon, double p
 /* Run up to max_rounds local rounds; *active = partitions still active. */
 int dg_rounds(dg_graph *g, int64_t max_rounds, int64_t *active);
 
-/* Pack boundary states into DEVICE buffer `buf` (n_boundary x 4 bytes):
- * MIN algorithms: the current states; SUM algorithms: the increments since
- * the last unpack ("each mirror always sends its new state
- * to its master"). */
+/* Pack boundary states into DEVICE buffer `buf` (n_boundary elements, see
+ * dg_boundary_size): MIN algorithms: the current states; SUM algorithms: the
+ * growth of each total since the last unpack ("each mirror
+ * always sends its new state to its master"). */
 int dg_boundary_pack(dg_graph *g, void *buf);
 
 /* Apply the all-reduced DEVICE buffer; vertices whose state changed

@@ -24,6 +24,7 @@ EXPORTS = [
     "dg_build_paths", "dg_upload", "dg_set_vertex_params", "dg_run", "dg_get_states",
     "dg_get_layout_info", "dg_export_paths", "dg_boundary_size", "dg_boundary_vertices",
     "dg_run_begin", "dg_rounds", "dg_boundary_pack", "dg_boundary_unpack", "dg_run_end",
+    "dg_normalize_states",
 ]
 
 
@@ -51,7 +52,8 @@ class dg_layout_info(ctypes.Structure):
                 ("n_hot_paths", ctypes.c_int64), ("n_layers", ctypes.c_int64),
                 ("n_dep_sccs", ctypes.c_int64), ("giant_scc_paths", ctypes.c_int64),
                 ("n_boundary", ctypes.c_int64), ("paths_before_merge", ctypes.c_int64),
-                ("preprocess_ms", ctypes.c_double), ("device_bytes", ctypes.c_int64)]
+                ("preprocess_ms", ctypes.c_double), ("device_bytes", ctypes.c_int64),
+                ("h2d_bytes", ctypes.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -93,6 +95,7 @@ def lib():
         "dg_boundary_pack": (i32, [P, P]),
         "dg_boundary_unpack": (i32, [P, P, pp(i64)]),
         "dg_run_end": (i32, [P, pp(dg_run_stats)]),
+        "dg_normalize_states": (i32, [P, P, i64]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)

@@ -64,6 +64,7 @@ void dg_destroy(dg_graph* g) {
     if (!g) return;
     dg::dev_free_work(g->work);
     dg::dev_free_layout(g->dev, true);
+    dg::dev_unpin_all(g->dev);
     delete g;
 }
 
@@ -73,6 +74,10 @@ int dg_load_csr(dg_graph* g, int64_t n, int64_t m, const int64_t* row_ptr, const
     if (n < 0 || n >= (int64_t)dg::kVMask || m < 0) return fail(DG_EINVAL, "dg_load_csr: bad n or m");
     if (!row_ptr || (m > 0 && !col)) return fail(DG_EINVAL, "dg_load_csr: NULL row_ptr/col");
     if (row_ptr[0] != 0 || row_ptr[n] != m) return fail(DG_EINVAL, "dg_load_csr: row_ptr[0] != 0 or row_ptr[n] != m");
+    dg::dev_free_work(g->work);
+    dg::dev_free_layout(g->dev, true);
+    dg::dev_unpin_all(g->dev);
+    g->uploaded = false;
     try {
         dg::HostCSR& c = g->csr;
         c = dg::HostCSR();
@@ -111,6 +116,10 @@ int dg_build_paths(dg_graph* g, const dg_path_params* p) {
     if (q.d_max < 1 || q.n_sub < 1 || q.part_entries < 1 || q.world < 1 || q.world > 64 ||
         q.rank < 0 || q.rank >= q.world || q.l_merge < 0 || q.merge_rule < 0 || q.merge_rule > 1)
         return fail(DG_EINVAL, "dg_build_paths: bad parameters");
+    dg::dev_free_work(g->work);
+    dg::dev_free_layout(g->dev, true);
+    dg::dev_unpin_all(g->dev);
+    g->uploaded = false;
     try {
         dg::build_layout(g->csr, q, g->layout);
     } catch (const std::bad_alloc&) {
@@ -201,6 +210,14 @@ int dg_get_states(dg_graph* g, void* out, int64_t n, int out_is_device) {
     return rc ? fail(rc, err) : DG_OK;
 }
 
+int dg_normalize_states(dg_graph* g, void* buf, int64_t n) {
+    if (!g || !buf || n < 0) return fail(DG_EINVAL, "dg_normalize_states: bad argument");
+    if (int rc0 = select_dev(g)) return rc0;
+    std::string err;
+    int rc = dg::dev_normalize(buf, n, err);
+    return rc ? fail(rc, err) : DG_OK;
+}
+
 int dg_get_layout_info(const dg_graph* g, dg_layout_info* info) {
     if (!g || !info) return fail(DG_EINVAL, "dg_get_layout_info: NULL argument");
     std::memset(info, 0, sizeof(*info));
@@ -219,6 +236,7 @@ int dg_get_layout_info(const dg_graph* g, dg_layout_info* info) {
     info->paths_before_merge = L.paths_before_merge;
     info->preprocess_ms = L.preprocess_ms;
     info->device_bytes = g->dev.bytes;
+    info->h2d_bytes = g->dev.h2d_bytes;
     return DG_OK;
 }
 
@@ -259,6 +277,7 @@ int dg_run_begin(dg_graph* g, int algo, int64_t source, double epsilon, double p
     g->run = dg::RunState();
     g->run.algo = algo; g->run.mode = DG_MODE_PATH; g->run.source = source;
     g->run.eps = epsilon; g->run.param = param;
+    g->run.raw_states = g->layout.params.world > 1;
     std::string err;
     rc = dg::dev_run_begin(g->work, g->dev, g->run, err);
     if (rc) return fail(rc, err);

@@ -37,17 +37,8 @@ struct HostLayout {
     std::vector<uint32_t> e_idx;        // vertex | head | tail
     std::vector<int32_t> e_w;           // weight of the path edge INTO this entry (0 at heads)
     std::vector<int64_t> part_off;      // n_part+1
-    // vertex -> partitions maps
-    std::vector<int64_t> vsrc_ptr;  std::vector<int32_t> vsrc;   // non-tail occurrences
-    std::vector<int64_t> vdst_ptr;  std::vector<int32_t> vdst;   // non-head occurrences
-    // home partition of each vertex: first (highest-priority) local partition
-    // holding it, -1 if none; PageRank/Adsorption activate it when the
-    // vertex's delta crosses eps
-    std::vector<int32_t> hpart;
     // multi-rank
     std::vector<int32_t> boundary;      // vertices present on >1 rank (ascending)
-    std::vector<uint8_t> bnd_owner;     // this rank owns boundary[k] (lowest rank holding it)
-    std::vector<uint8_t> vown;          // this rank owns vertex v (lowest rank holding it; rank 0 if none)
     // stats
     int64_t n_layers = 0, n_dep_sccs = 0, giant = 0, paths_before_merge = 0, n_hot = 0;
     double preprocess_ms = 0;
@@ -61,17 +52,15 @@ struct DevLayout {
     uint32_t* e_idx = nullptr;
     int32_t* e_w = nullptr;
     int64_t* part_off = nullptr;
-    int64_t* vsrc_ptr = nullptr; int32_t* vsrc = nullptr;
-    int64_t* vdst_ptr = nullptr; int32_t* vdst = nullptr;
     int32_t* bnd = nullptr;
-    uint8_t* bnd_owner = nullptr;
-    int32_t* hpart = nullptr;
-    uint8_t* vown = nullptr;
     // CSR (for the vertex-centric ablation and per-vertex coefficients)
     int64_t* row_ptr = nullptr; int32_t* col = nullptr; int32_t* w = nullptr;
     int32_t* outdeg = nullptr;
-    int64_t bytes = 0;
+    int64_t bytes = 0;      // device bytes allocated
+    int64_t h2d_bytes = 0;  // bytes copied host -> device by the last upload
+    std::vector<void*> pinned;  // host buffers page-locked with cudaHostRegister
 };
+void dev_unpin_all(DevLayout& D);
 
 struct DevWork;  // defined in dg_kernels.cu
 
@@ -80,6 +69,7 @@ struct RunState {
     int64_t source = 0;
     double eps = 0, param = 0;
     int64_t round = 0;
+    bool raw_states = false;  // multi-rank: per-rank additive contributions, not normalised
     dg_run_stats stats{};
 };
 
@@ -96,6 +86,7 @@ int dev_rounds(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, 
 int dev_boundary_pack(DevWork* W, const DevLayout& D, RunState& S, void* buf, std::string& err);
 int dev_boundary_unpack(DevWork* W, const DevLayout& D, RunState& S, const void* buf, int64_t* active, std::string& err);
 int dev_run_end(DevWork* W, const DevLayout& D, RunState& S, std::string& err);
+int dev_normalize(void* buf, int64_t n, std::string& err);
 int dev_get_states(DevWork* W, const DevLayout& D, const RunState& S, void* out, int64_t n, int out_is_device,
                    std::string& err);
 void dev_free_work(DevWork*& W);

@@ -402,12 +402,8 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
 
     // ---- boundary vertices: present in partitions of >1 rank (round-robin owner q % world);
     // owner of a vertex = lowest rank holding it (rank 0 for vertices on no path)
-    L.vown.assign(n, world > 1 ? 0 : 1);
     if (world > 1) {
-        // present[v]: ranks whose partitions hold v.  touched[v]: ranks that can
-        // write v's state -- present, or (PageRank/Adsorption) an out-neighbour of
-        // a present vertex, since a firing vertex pushes along all its CSR edges.
-        std::vector<uint64_t> present(n, 0), touched;
+        std::vector<uint64_t> present(n, 0);  // ranks whose partitions hold v
         for (int64_t q = 0; q < G; q++) {
             uint64_t bit = 1ull << ((q % world) & 63);
             for (int64_t r = gpart_first[q]; r < gpart_first[q + 1]; r++) {
@@ -415,18 +411,8 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
                 for (int64_t k = moff[i]; k < moff[i + 1]; k++) present[mv[k]] |= bit;
             }
         }
-        touched = present;
-        for (int64_t u = 0; u < n; u++)
-            if (present[u])
-                for (int64_t e = g.row_ptr[u]; e < g.row_ptr[u + 1]; e++) touched[g.col[e]] |= present[u];
-        for (int64_t v = 0; v < n; v++) {
-            int owner = present[v] ? __builtin_ctzll(present[v]) : 0;
-            L.vown[v] = owner == rank;
-            if (__builtin_popcountll(touched[v]) > 1) {
-                L.boundary.push_back((int32_t)v);
-                L.bnd_owner.push_back(owner == rank);
-            }
-        }
+        for (int64_t v = 0; v < n; v++)
+            if (__builtin_popcountll(present[v]) > 1) L.boundary.push_back((int32_t)v);
     }
 
     phase("priority+partitions");
@@ -452,38 +438,8 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
         }
         L.part_off.push_back((int64_t)L.e_idx.size());
     }
-    const int64_t npart = (int64_t)L.part_off.size() - 1;
 
-    // ---- vertex -> partitions (distinct), source (non-tail) and destination (non-head) occurrences
-    auto build_map = [&](uint32_t skip_flag, std::vector<int64_t>& ptr, std::vector<int32_t>& lst) {
-        ptr.assign(n + 1, 0);
-        std::vector<int32_t> lastp(n, -1);
-        for (int64_t q = 0; q < npart; q++)
-            for (int64_t k = L.part_off[q]; k < L.part_off[q + 1]; k++) {
-                uint32_t c = L.e_idx[k];
-                if (c & skip_flag) continue;
-                int32_t v = (int32_t)(c & kVMask);
-                if (lastp[v] != (int32_t)q) { lastp[v] = (int32_t)q; ptr[v + 1]++; }
-            }
-        for (int64_t v = 0; v < n; v++) ptr[v + 1] += ptr[v];
-        lst.resize(ptr[n]);
-        std::vector<int64_t> fill(ptr.begin(), ptr.end() - 1);
-        std::fill(lastp.begin(), lastp.end(), -1);
-        for (int64_t q = 0; q < npart; q++)
-            for (int64_t k = L.part_off[q]; k < L.part_off[q + 1]; k++) {
-                uint32_t c = L.e_idx[k];
-                if (c & skip_flag) continue;
-                int32_t v = (int32_t)(c & kVMask);
-                if (lastp[v] != (int32_t)q) { lastp[v] = (int32_t)q; lst[fill[v]++] = (int32_t)q; }
-            }
-    };
-    build_map(kTail, L.vsrc_ptr, L.vsrc);
-    build_map(kHead, L.vdst_ptr, L.vdst);
-    phase("layout+maps");
-    L.hpart.assign(n, -1);
-    for (int64_t q = npart - 1; q >= 0; q--)
-        for (int64_t k = L.part_off[q]; k < L.part_off[q + 1]; k++) L.hpart[L.e_idx[k] & kVMask] = (int32_t)q;
-
+    phase("layout");
     L.n_layers = n_layers;
     L.n_dep_sccs = n_dep_sccs;
     L.giant = giant;

@@ -159,6 +159,11 @@ class DiGraph:
               "dg_boundary_unpack")
         return a.value
 
+    def normalize_states(self, buf):
+        check(self._L.dg_normalize_states(self._h, ctypes.c_void_p(buf.data_ptr()), buf.numel()),
+              "dg_normalize_states")
+        return buf
+
     def run_end(self):
         st = _abi.dg_run_stats()
         check(self._L.dg_run_end(self._h, ctypes.byref(st)), "dg_run_end")

@@ -132,16 +132,8 @@ def test_multirank_partitioning_is_a_disjoint_cover():
     src, dst, _ = g.edges()
     assert sorted(sum(covers, [])) == sorted(zip(src.tolist(), dst.tolist()))
     assert bnd_sets[0] == bnd_sets[1] == bnd_sets[2]
-    # boundary = vertices whose state more than one rank can write: present in a
-    # rank's paths, or an out-neighbour of a present vertex (delta pushes)
-    src, dst, _ = g.edges()
-    touched = []
-    for s_ in presence:
-        t = set(s_)
-        pres = np.zeros(g.n, bool); pres[list(s_)] = True
-        t |= set(dst[pres[src]].tolist())
-        touched.append(t)
-    multi = sorted(v for v in range(g.n) if sum(v in t for t in touched) > 1)
+    # boundary = vertices replicated on more than one rank's paths
+    multi = sorted(v for v in range(g.n) if sum(v in s_ for s_ in presence) > 1)
     assert bnd_sets[0] == multi
     sizes = [len(c) for c in covers]
     assert max(sizes) - min(sizes) <= 0.2 * max(sizes)       # balanced
