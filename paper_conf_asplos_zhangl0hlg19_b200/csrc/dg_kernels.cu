@@ -140,6 +140,47 @@ __device__ __forceinline__ void ld_stream_u64x4(const unsigned long long* p, uns
     asm volatile("ld.global.L1::no_allocate.v2.u64 {%0,%1}, [%2];" : "=l"(o[0]), "=l"(o[1]) : "l"(p));
     asm volatile("ld.global.L1::no_allocate.v2.u64 {%0,%1}, [%2];" : "=l"(o[2]), "=l"(o[3]) : "l"(p + 2));
 }
+// L2 eviction policies: streamed path arrays are evict-first so they do not
+// push the (re-used) vertex states out of the 126 MB L2; states are evict-last.
+__device__ __forceinline__ unsigned long long policy_evict_first() {
+    unsigned long long p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ unsigned long long policy_evict_last() {
+    unsigned long long p;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint4 ld_stream_u4_h(const uint32_t* p, unsigned long long pol) {
+    uint4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ float4 ld_stream_f4_h(const float* p, unsigned long long pol) {
+    float4 r;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p), "l"(pol));
+    return r;
+}
+__device__ __forceinline__ void ld_stream_u64x4_h(const unsigned long long* p, unsigned long long (&o)[4],
+                                                  unsigned long long pol) {
+    asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;"
+                 : "=l"(o[0]), "=l"(o[1]) : "l"(p), "l"(pol));
+    asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;"
+                 : "=l"(o[2]), "=l"(o[3]) : "l"(p + 2), "l"(pol));
+}
+__device__ __forceinline__ void st_stream_u64_h(unsigned long long* p, unsigned long long v, unsigned long long pol) {
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(pol));
+}
+// 16-byte master-state gather kept in L2 (evict-last)
+__device__ __forceinline__ void ld_state_h(const void* p, unsigned long long& t, float& coef, unsigned long long pol) {
+    unsigned long long a, b;
+    asm volatile("ld.global.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;" : "=l"(a), "=l"(b) : "l"(p), "l"(pol));
+    t = a;
+    coef = __uint_as_float((unsigned)(b & 0xffffffffull));
+}
 __device__ __forceinline__ uint32_t u4get(const uint4& v, int k) {
     return k == 0 ? v.x : k == 1 ? v.y : k == 2 ? v.z : v.w;
 }
@@ -310,15 +351,15 @@ __device__ __forceinline__ unsigned long long fx_from(float x) { return x > 0.f 
 __device__ __forceinline__ float fx_to(unsigned long long v) { return __ull2float_rn(v) * kFxInv; }
 
 template <bool ADS>
-__device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, const uint32_t* bcur, uint32_t* bnxt,
-                           Acc& acc) {
+__device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, const uint32_t* bcur, Acc& acc,
+                           unsigned long long pol_stream, unsigned long long pol_keep) {
     const int lane = threadIdx.x & 31;
     const unsigned long long eps = P.eps_fx;
     float carry = 0.f;
     for (int64_t base = beg & ~(int64_t)3; base < end; base += 128) {
         const int64_t i0 = base + 4 * lane;
         uint4 code = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
-        if (i0 < end) code = ld_stream_u4(P.e_idx + i0);
+        if (i0 < end) code = ld_stream_u4_h(P.e_idx + i0, pol_stream);
         uint32_t vtx[4];
         bool valid[4], any_act = false;
 #pragma unroll
@@ -333,8 +374,8 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, const uin
         unsigned long long sv[4] = {0ull, 0ull, 0ull, 0ull};
         float4 c4 = make_float4(0.f, 0.f, 0.f, 0.f);
         if (i0 < end) {
-            ld_stream_u64x4(P.s_val + i0, sv);
-            if (ADS) c4 = ld_stream_f4(P.e_coef + i0);
+            ld_stream_u64x4_h(P.s_val + i0, sv, pol_stream);
+            if (ADS) c4 = ld_stream_f4_h(P.e_coef + i0, pol_stream);
         }
         float al[4], be[4];
         unsigned long long pend[4];
@@ -344,10 +385,12 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, const uin
             const uint32_t c = u4get(code, k);
             hd[k] = !valid[k] || (c & kHead);
             tl[k] = !valid[k] || (c & kTail);
-            AccState st = valid[k] ? P.vs_a[vtx[k]] : AccState{0ull, 0.f, 0};
-            const unsigned long long pd = st.T > sv[k] ? st.T - sv[k] : 0ull;
+            unsigned long long T = 0ull;
+            float coef = 0.f;
+            if (valid[k]) ld_state_h(&P.vs_a[vtx[k]], T, coef, pol_keep);
+            const unsigned long long pd = T > sv[k] ? T - sv[k] : 0ull;
             pend[k] = (!tl[k] && pd >= eps) ? pd : 0ull;
-            const float coef = ADS ? f4get(c4, k) : st.coef;
+            if (ADS) coef = f4get(c4, k);
             al[k] = tl[k] ? 0.f : coef * fx_to(pend[k]);
             be[k] = (tl[k] || hd[k]) ? 0.f : coef;
         }
@@ -378,15 +421,32 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, const uin
             if (!hd[k]) acc.edges++;
             const unsigned long long p = fx_from(pin[k]);
             if (p) {
-                const unsigned long long tn = atomicAdd(&P.vs_a[vtx[k]].T, p) + p;
+                atomicAdd(&P.vs_a[vtx[k]].T, p);  // no return value used: REDG
                 acc.upd++;
-                if (tn - P.sigma[vtx[k]] >= eps && signal_vertex(bnxt, vtx[k])) {
-                    P.sigma[vtx[k]] = tn;
-                    acc.sig++;
-                }
             }
-            if (!tl[k] && (pend[k] | p)) P.s_val[i0 + k] = sv[k] + pend[k] + p;
+            if (!tl[k] && (pend[k] | p)) st_stream_u64_h(P.s_val + i0 + k, sv[k] + pend[k] + p, pol_stream);
         }
+    }
+}
+
+// End-of-round vertex sweep of the accumulative algorithms: a vertex whose
+// total grew by >= eps since its last signal is signalled for the next round
+// (the per-vertex stop rule at delta < eps).  One warp per 32 vertices writes
+// one bitmap word (the next bitmap is empty at this point).
+__device__ void accum_sweep(const KParams& P, uint32_t* bnxt, unsigned& cnt) {
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int64_t words = (P.n + 31) >> 5;
+    for (int64_t w = gw; w < words; w += nwarps) {
+        const int64_t v = w * 32 + lane;
+        bool s = false;
+        if (v < P.n) {
+            const unsigned long long T = P.vs_a[v].T;
+            if (T - P.sigma[v] >= P.eps_fx) { P.sigma[v] = T; s = true; }
+        }
+        const unsigned m = __ballot_sync(0xffffffffu, s);
+        if (lane == 0) { bnxt[w] = m; cnt += __popc(m); }
     }
 }
 
@@ -483,9 +543,11 @@ __device__ void walk_scc_bwd(const KParams& P, int64_t beg, int64_t end, const u
 
 // ------------------------------------------------------------------ persistent round driver
 template <int ALGO>
-__global__ void __launch_bounds__(kBlock) path_kernel(KParams P) {
+__global__ void __launch_bounds__(kBlock, 3) path_kernel(KParams P) {
     cg::grid_group grid = cg::this_grid();
     const int lane = threadIdx.x & 31;
+    constexpr bool kAccum = ALGO == DG_PAGERANK || ALGO == DG_ADSORPTION;
+    const unsigned long long pol_stream = policy_evict_first(), pol_keep = policy_evict_last();
     Acc acc;
     int r = 0;
     for (; r < P.max_rounds; r++) {
@@ -505,8 +567,12 @@ __global__ void __launch_bounds__(kBlock) path_kernel(KParams P) {
             else if (ALGO == DG_WCC) walk_minplus<2>(P, beg, end, bcur, bnxt, acc);
             else if (ALGO == 100) walk_minplus<3>(P, beg, end, bcur, bnxt, acc);
             else if (ALGO == 101) walk_scc_bwd(P, beg, end, bcur, bnxt, acc);
-            else if (ALGO == DG_PAGERANK) walk_accum<false>(P, beg, end, bcur, bnxt, acc);
-            else if (ALGO == DG_ADSORPTION) walk_accum<true>(P, beg, end, bcur, bnxt, acc);
+            else if (ALGO == DG_PAGERANK) walk_accum<false>(P, beg, end, bcur, acc, pol_stream, pol_keep);
+            else if (ALGO == DG_ADSORPTION) walk_accum<true>(P, beg, end, bcur, acc, pol_stream, pol_keep);
+        }
+        if (kAccum) {
+            grid.sync();  // all pushes of the round landed
+            accum_sweep(P, bnxt, acc.sig);
         }
         // publish this round's newly signalled vertices (the device active counter)
         unsigned s = acc.sig;
