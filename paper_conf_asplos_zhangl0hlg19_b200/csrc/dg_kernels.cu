@@ -64,7 +64,7 @@ struct Counters {
 struct __align__(16) AccState {
     unsigned long long T;
     float coef;
-    int pad;
+    int stamp;  // the round this vertex was last signalled for (activity of the path walk)
 };
 
 struct DevWork {
@@ -174,12 +174,14 @@ __device__ __forceinline__ void ld_stream_u64x4_h(const unsigned long long* p, u
 __device__ __forceinline__ void st_stream_u64_h(unsigned long long* p, unsigned long long v, unsigned long long pol) {
     asm volatile("st.global.L1::no_allocate.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(pol));
 }
-// 16-byte master-state gather kept in L2 (evict-last)
-__device__ __forceinline__ void ld_state_h(const void* p, unsigned long long& t, float& coef, unsigned long long pol) {
+// 16-byte master-state gather kept in L2 (evict-last): {T, coef, stamp}
+__device__ __forceinline__ void ld_state_h(const void* p, unsigned long long& t, float& coef, int& stamp,
+                                           unsigned long long pol) {
     unsigned long long a, b;
     asm volatile("ld.global.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;" : "=l"(a), "=l"(b) : "l"(p), "l"(pol));
     t = a;
     coef = __uint_as_float((unsigned)(b & 0xffffffffull));
+    stamp = (int)(b >> 32);
 }
 __device__ __forceinline__ uint32_t u4get(const uint4& v, int k) {
     return k == 0 ? v.x : k == 1 ? v.y : k == 2 ? v.z : v.w;
@@ -351,32 +353,45 @@ __device__ __forceinline__ unsigned long long fx_from(float x) { return x > 0.f 
 __device__ __forceinline__ float fx_to(unsigned long long v) { return __ull2float_rn(v) * kFxInv; }
 
 template <bool ADS>
-__device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, const uint32_t* bcur, Acc& acc,
+__device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round, Acc& acc,
                            unsigned long long pol_stream, unsigned long long pol_keep) {
     const int lane = threadIdx.x & 31;
     const unsigned long long eps = P.eps_fx;
     float carry = 0.f;
-    for (int64_t base = beg & ~(int64_t)3; base < end; base += 128) {
+    const int64_t first = beg & ~(int64_t)3;
+    // software pipeline: the next window's indices are in flight while this one is walked
+    uint4 code_nx = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
+    if (first + 4 * lane < end) code_nx = ld_stream_u4_h(P.e_idx + first + 4 * lane, pol_stream);
+    for (int64_t base = first; base < end; base += 128) {
         const int64_t i0 = base + 4 * lane;
-        uint4 code = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
-        if (i0 < end) code = ld_stream_u4_h(P.e_idx + i0, pol_stream);
-        uint32_t vtx[4];
-        bool valid[4], any_act = false;
-#pragma unroll
-        for (int k = 0; k < 4; k++) {
-            const int64_t i = i0 + k;
-            valid[k] = i >= beg && i < end;
-            vtx[k] = u4get(code, k) & kVMask;
-            any_act |= valid[k] && test_bit(bcur, vtx[k]);
-        }
-        if (!__any_sync(0xffffffffu, any_act) && carry == 0.f) continue;
-        acc.units++;
+        const uint4 code = code_nx;
+        if (i0 + 128 < end) code_nx = ld_stream_u4_h(P.e_idx + i0 + 128, pol_stream);
+        // masters (with their signal stamps) and mirrors are fetched together;
+        // a window none of whose vertices was signalled and that receives no
+        // carry is skipped after the fetch (PageRank keeps most windows active)
         unsigned long long sv[4] = {0ull, 0ull, 0ull, 0ull};
         float4 c4 = make_float4(0.f, 0.f, 0.f, 0.f);
         if (i0 < end) {
             ld_stream_u64x4_h(P.s_val + i0, sv, pol_stream);
             if (ADS) c4 = ld_stream_f4_h(P.e_coef + i0, pol_stream);
         }
+        uint32_t vtx[4];
+        unsigned long long T[4];
+        float cf[4];
+        bool valid[4], any_act = false;
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            const int64_t i = i0 + k;
+            valid[k] = i >= beg && i < end;
+            vtx[k] = u4get(code, k) & kVMask;
+            T[k] = 0ull;
+            cf[k] = 0.f;
+            int stamp = -1;
+            if (valid[k]) ld_state_h(&P.vs_a[vtx[k]], T[k], cf[k], stamp, pol_keep);
+            any_act |= stamp == round;
+        }
+        if (!__any_sync(0xffffffffu, any_act) && carry == 0.f) continue;
+        acc.units++;
         float al[4], be[4];
         unsigned long long pend[4];
         bool hd[4], tl[4];
@@ -385,12 +400,9 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, const uin
             const uint32_t c = u4get(code, k);
             hd[k] = !valid[k] || (c & kHead);
             tl[k] = !valid[k] || (c & kTail);
-            unsigned long long T = 0ull;
-            float coef = 0.f;
-            if (valid[k]) ld_state_h(&P.vs_a[vtx[k]], T, coef, pol_keep);
-            const unsigned long long pd = T > sv[k] ? T - sv[k] : 0ull;
+            const unsigned long long pd = T[k] > sv[k] ? T[k] - sv[k] : 0ull;
             pend[k] = (!tl[k] && pd >= eps) ? pd : 0ull;
-            if (ADS) coef = f4get(c4, k);
+            const float coef = ADS ? f4get(c4, k) : cf[k];
             al[k] = tl[k] ? 0.f : coef * fx_to(pend[k]);
             be[k] = (tl[k] || hd[k]) ? 0.f : coef;
         }
@@ -431,22 +443,16 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, const uin
 
 // End-of-round vertex sweep of the accumulative algorithms: a vertex whose
 // total grew by >= eps since its last signal is signalled for the next round
-// (the per-vertex stop rule at delta < eps).  One warp per 32 vertices writes
-// one bitmap word (the next bitmap is empty at this point).
-__device__ void accum_sweep(const KParams& P, uint32_t* bnxt, unsigned& cnt) {
-    const int lane = threadIdx.x & 31;
-    const int64_t gw = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    const int64_t words = (P.n + 31) >> 5;
-    for (int64_t w = gw; w < words; w += nwarps) {
-        const int64_t v = w * 32 + lane;
-        bool s = false;
-        if (v < P.n) {
-            const unsigned long long T = P.vs_a[v].T;
-            if (T - P.sigma[v] >= P.eps_fx) { P.sigma[v] = T; s = true; }
+// (the per-vertex stop rule at delta < eps): its stamp is set to that round,
+// which the next walk reads together with the total.
+__device__ void accum_sweep(const KParams& P, int next_round, unsigned& cnt) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < P.n; v += (int64_t)gridDim.x * blockDim.x) {
+        const unsigned long long T = P.vs_a[v].T;
+        if (T - P.sigma[v] >= P.eps_fx) {
+            P.sigma[v] = T;
+            P.vs_a[v].stamp = next_round;
+            cnt++;
         }
-        const unsigned m = __ballot_sync(0xffffffffu, s);
-        if (lane == 0) { bnxt[w] = m; cnt += __popc(m); }
     }
 }
 
@@ -567,12 +573,12 @@ __global__ void __launch_bounds__(kBlock, 3) path_kernel(KParams P) {
             else if (ALGO == DG_WCC) walk_minplus<2>(P, beg, end, bcur, bnxt, acc);
             else if (ALGO == 100) walk_minplus<3>(P, beg, end, bcur, bnxt, acc);
             else if (ALGO == 101) walk_scc_bwd(P, beg, end, bcur, bnxt, acc);
-            else if (ALGO == DG_PAGERANK) walk_accum<false>(P, beg, end, bcur, acc, pol_stream, pol_keep);
-            else if (ALGO == DG_ADSORPTION) walk_accum<true>(P, beg, end, bcur, acc, pol_stream, pol_keep);
+            else if (ALGO == DG_PAGERANK) walk_accum<false>(P, beg, end, round, acc, pol_stream, pol_keep);
+            else if (ALGO == DG_ADSORPTION) walk_accum<true>(P, beg, end, round, acc, pol_stream, pol_keep);
         }
         if (kAccum) {
             grid.sync();  // all pushes of the round landed
-            accum_sweep(P, bnxt, acc.sig);
+            accum_sweep(P, round + 1, acc.sig);
         }
         // publish this round's newly signalled vertices (the device active counter)
         unsigned s = acc.sig;
@@ -733,7 +739,7 @@ __global__ void init_acc_kernel(AccState* vs, unsigned long long* sigma, const i
         const float t0 = base ? base[v] : 1.f - d;
         const unsigned long long T = (unsigned long long)((double)t0 * 4294967296.0);
         const float c = (!base && outdeg[v] > 0) ? d / (float)outdeg[v] : 0.f;
-        vs[v] = AccState{T, c, 0};
+        vs[v] = AccState{T, c, 0};  // stamp 0: active in round 0
         sigma[v] = T;
     }
 }
@@ -858,7 +864,7 @@ __global__ void pack_sum_kernel(const AccState* vs, const int32_t* bnd, int64_t 
 }
 __global__ void unpack_sum_kernel(AccState* vs, unsigned long long* sigma, const int32_t* bnd, int64_t nb,
                                   unsigned long long* base, const unsigned long long* buf, unsigned long long eps,
-                                  uint32_t* b, Counters* ctr, int slot) {
+                                  int round, Counters* ctr, int slot) {
     unsigned cnt = 0;
     GRID_STRIDE(k, nb) {
         const int v = bnd[k];
@@ -867,7 +873,8 @@ __global__ void unpack_sum_kernel(AccState* vs, unsigned long long* sigma, const
         vs[v].T = t;
         if (t - sigma[v] >= eps) {
             sigma[v] = t;
-            cnt += signal_vertex(b, (uint32_t)v);
+            cnt += vs[v].stamp != round;
+            vs[v].stamp = round;
         }
     }
     for (int off = 16; off; off >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, off);
@@ -1323,7 +1330,8 @@ int dev_boundary_unpack(DevWork* W, const DevLayout& D, RunState& S, const void*
         if (S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION)
             unpack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_a, W->sigma, D.bnd, D.n_bnd, W->bnd_base,
                                                          (const unsigned long long*)buf,
-                                                         (unsigned long long)(S.eps * 4294967296.0), b, W->ctr, slot);
+                                                         (unsigned long long)(S.eps * 4294967296.0), c.round, W->ctr,
+                                                         slot);
         else
             unpack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, D.bnd, D.n_bnd, (const uint32_t*)buf, b, W->ctr,
                                                          slot);
