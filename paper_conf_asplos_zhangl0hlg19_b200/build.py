@@ -42,7 +42,8 @@ def build(force=False, verbose=False):
     for s in srcs:
         o = os.path.join(BUILD, os.path.basename(s) + ".o")
         if s.endswith(".cu"):
-            cmd = ["nvcc", *NVCC_FLAGS, "-c", s, "-o", o]
+            extra = os.environ.get("DG_NVCC_EXTRA", "").split()  # developer experiments only
+            cmd = ["nvcc", *NVCC_FLAGS, *extra, "-c", s, "-o", o]
         else:
             cmd = ["g++", *CXX_FLAGS, "-I", "/usr/local/cuda/include", "-c", s, "-o", o]
         r = subprocess.run(cmd, capture_output=True, text=True)

@@ -49,6 +49,9 @@ constexpr uint32_t INF = DG_INF;
 constexpr int kBlock = 256;
 constexpr int kWarps = kBlock / 32;
 constexpr int kPad = 256;  // zero entries after every per-entry array
+#ifndef DG_PATH_MINB
+#define DG_PATH_MINB 3  // resident CTAs per SM requested for the path kernel
+#endif
 
 // device counters of a run
 struct Counters {
@@ -549,7 +552,7 @@ __device__ void walk_scc_bwd(const KParams& P, int64_t beg, int64_t end, const u
 
 // ------------------------------------------------------------------ persistent round driver
 template <int ALGO>
-__global__ void __launch_bounds__(kBlock, 3) path_kernel(KParams P) {
+__global__ void __launch_bounds__(kBlock, DG_PATH_MINB) path_kernel(KParams P) {
     cg::grid_group grid = cg::this_grid();
     const int lane = threadIdx.x & 31;
     constexpr bool kAccum = ALGO == DG_PAGERANK || ALGO == DG_ADSORPTION;

@@ -1,0 +1,201 @@
+"""Multi-GPU host logic on CPU (-m "not gpu"): world-size-2 gloo runs of the
+real multi-rank preprocessing (dg_build_paths with rank/world: path
+partitioning and boundary set) and of the real driver protocol
+(`parallel.run_distributed` / `gather_states`), with a test-only CPU engine
+that walks the rank's exported paths with the kernel's semantics.  The
+product itself has no CPU path; this engine exists only in the tests.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import inputs
+from oracle import algorithms as OA
+
+FX = 1 << 32
+
+
+class CpuPathEngine:
+    """Mimics libdigraph's per-rank semantics on the rank's own paths."""
+
+    def __init__(self, g, rank, world):
+        from paper_conf_asplos_zhangl0hlg19_b200 import DiGraph
+        dg = DiGraph()
+        dg.load_graph(g)
+        dg.build_paths(part_entries=64, rank=rank, world=world)
+        ex = dg.export_paths()
+        self.bnd = dg.boundary_vertices().astype(np.int64)
+        off, v = ex["path_off"], ex["vertices"].astype(np.int64)
+        self.paths = [v[off[i]:off[i + 1]] for i in range(len(off) - 1)]
+        src, dst, w = g.edges()
+        self.wmap = {}
+        for a, b, c in zip(src.tolist(), dst.tolist(), w.tolist()):
+            self.wmap.setdefault((a, b), []).append(c)
+        self.n = g.n
+        self.outdeg = np.diff(g.row_ptr)
+        # per-path weights / mirrors
+        self.pw = []
+        used = {}
+        for p in self.paths:
+            ws = []
+            for a, b in zip(p[:-1].tolist(), p[1:].tolist()):
+                k = used.get((a, b), 0)
+                ws.append(self.wmap[(a, b)][k])
+                used[(a, b)] = k + 1
+            self.pw.append(ws)
+
+    def boundary_vertices(self):
+        return self.bnd
+
+    def run_begin(self, algo, source=0, epsilon=1e-7, damping=0.85):
+        self.algo = algo
+        if algo in ("sssp", "wcc"):
+            self.x = np.full(self.n, OA.UNREACHED, np.int64)
+            if algo == "sssp":
+                self.x[source] = 0
+            else:
+                self.x = np.arange(self.n, dtype=np.int64)
+        else:
+            self.eps = int(epsilon * FX)
+            self.T = np.full(self.n, int((1 - damping) * FX), np.int64)
+            self.coef = np.where(self.outdeg > 0, damping / np.maximum(self.outdeg, 1), 0.0)
+            self.S = [np.zeros(len(p), np.int64) for p in self.paths]
+            self.base = self.T[self.bnd].copy()
+
+    def _walk_min(self):
+        changed = 0
+        for p, ws in zip(self.paths, self.pw):
+            cur = None
+            for t, v in enumerate(p.tolist()):
+                a = self.x[v]
+                if cur is not None:
+                    cand = cur + (ws[t - 1] if self.algo == "sssp" else 0)
+                    if cand < a:
+                        self.x[v] = cand
+                        changed += 1
+                        a = cand
+                cur = a
+            if self.algo == "wcc":  # backward along the path
+                cur = None
+                for v in p[::-1].tolist():
+                    a = self.x[v]
+                    if cur is not None and cur < a:
+                        self.x[v] = cur
+                        changed += 1
+                        a = cur
+                    cur = a
+        return changed
+
+    def _walk_accum(self):
+        pushed = 0
+        for p, S in zip(self.paths, self.S):
+            carry = 0.0
+            for t, v in enumerate(p.tolist()):
+                pin = carry if t > 0 else 0.0
+                pfx = int(pin * FX)
+                if pfx:
+                    self.T[v] += pfx
+                    pushed += 1
+                if t < len(p) - 1:
+                    pend = (self.T[v] - pfx) - S[t]      # the total before this walk's push
+                    pend = pend if pend >= self.eps else 0
+                    carry = self.coef[v] * ((pend / FX) + pin)
+                    S[t] += pend + pfx
+                else:
+                    carry = 0.0
+        return pushed
+
+    def rounds(self, k):
+        for _ in range(100000):
+            if (self._walk_min() if self.algo in ("sssp", "wcc") else self._walk_accum()) == 0:
+                return 0
+        raise RuntimeError("local rounds did not converge")
+
+    def boundary_pack(self, buf):
+        if self.algo in ("sssp", "wcc"):
+            buf.copy_(torch.from_numpy(self.x[self.bnd].astype(np.int32)))
+        else:
+            buf.copy_(torch.from_numpy(self.T[self.bnd] - self.base))
+
+    def boundary_unpack(self, buf):
+        if len(self.bnd) == 0:
+            return 0
+        b = buf.numpy().astype(np.int64)
+        if self.algo in ("sssp", "wcc"):
+            new = np.minimum(self.x[self.bnd], b)
+            act = int((new < self.x[self.bnd]).sum())
+            self.x[self.bnd] = new
+            return act
+        t = self.base + b
+        act = int(((t - self.T[self.bnd]) > 0).sum())
+        self.T[self.bnd] = t
+        self.base = t.copy()
+        return act
+
+    def run_end(self):
+        return {}
+
+    def get_states(self, out):
+        if self.algo in ("sssp", "wcc"):
+            out.copy_(torch.from_numpy(self.x.astype(np.int32)))
+        else:
+            out.copy_(torch.from_numpy((self.T / FX).astype(np.float32)))
+        return out
+
+    def normalize_states(self, buf):
+        buf /= buf.sum()
+        return buf
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def _worker(rank, world, port, algo, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_asplos_zhangl0hlg19_b200 import parallel
+    g = inputs.rmat(10, 1024, 6000, seed=21, weights=(1, 20))
+    eng = CpuPathEngine(g, rank, world)
+    stats, info = parallel.run_distributed(eng, algo, source=0, epsilon=1e-7, device=torch.device("cpu"))
+    out = parallel.gather_states(eng, algo, g.n, device=torch.device("cpu"))
+    if rank == 0:
+        q.put((out.numpy().copy(), info))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("algo", ["sssp", "wcc", "pagerank"])
+def test_two_rank_protocol_matches_oracle(algo):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, algo, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    got, info = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    g = inputs.rmat(10, 1024, 6000, seed=21, weights=(1, 20))
+    src, dst, w = g.edges()
+    assert info["boundary"] > 0 and info["syncs"] >= 1
+    if algo == "sssp":
+        exp, _ = OA.sssp_bellman_ford(g.n, src, dst, w, 0)
+        assert np.array_equal(got.astype(np.int64), exp)
+    elif algo == "wcc":
+        exp, _ = OA.wcc_label_propagation(g.n, src, dst)
+        assert np.array_equal(got.astype(np.int64), exp)
+    else:
+        exp, _ = OA.pagerank_power(g.n, src, dst)
+        assert np.abs(got - exp).sum() <= 1e-4
+        assert (np.abs(got - exp) / exp).max() <= 1e-3
