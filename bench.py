@@ -200,8 +200,9 @@ def main():
     ap.add_argument("--mode", default="path", choices=["path", "vertex"])
     ap.add_argument("--seed", type=int, default=1)
     ap.add_argument("--eps", type=float, default=1e-7)
-    ap.add_argument("--part-entries", type=int, default=2048)
+    ap.add_argument("--part-entries", type=int, default=0)
     ap.add_argument("--merge-rule", default="relaxed")
+    ap.add_argument("--n-proxy", type=int, default=2048)
     ap.add_argument("--l2-flush-mb", type=int, default=512)
     ap.add_argument("--no-extras", action="store_true", help="skip ablation/e2e/cpu baseline (profiling runs)")
     args = ap.parse_args()
@@ -231,7 +232,8 @@ def main():
     dg = DiGraph(device=local)
     dg.load_graph(g)
     t0 = time.time()
-    dg.build_paths(part_entries=args.part_entries, rank=rank, world=world, merge_rule=args.merge_rule)
+    dg.build_paths(part_entries=args.part_entries, rank=rank, world=world, merge_rule=args.merge_rule,
+                   n_proxy=args.n_proxy)
     t_pre = time.time() - t0
     dg.upload()
     info = dg.layout_info()

@@ -65,16 +65,20 @@ typedef struct {
     int32_t n_sub;         /* number of subgraphs Algorithm 1 runs on in parallel (line 114) */
     int32_t order;         /* successor/root order: 0 = degree desc (line 5), 1 = vertex id */
     float hot_factor;      /* hot path iff avg degree >= hot_factor * mean degree (R-HOT) */
-    int32_t part_entries;  /* target path entries per partition (scheduling unit) */
+    int32_t part_entries;  /* target path entries per partition (scheduling unit); 0 = auto
+                              (about 16K partitions, 128..2048 entries each) */
     int32_t rank;          /* this process's rank for multi-GPU path partitioning */
     int32_t world;         /* number of ranks (1 = single GPU) */
     int32_t merge_rule;    /* 0: paper-literal (no merge through a line-13 inner vertex of
                               in/out degree > 1); 1: relaxed (any head-to-tail merge within
                               l_merge; reading R-MERGE) */
+    int32_t n_proxy;       /* highest-degree vertices kept as shared-memory proxies by the
+                              PageRank/Adsorption walk; 0 = none */
 } dg_path_params;
 
 /* Fill *p with the defaults (d_max 16, l_merge 64, n_sub 64, order 0,
- * hot_factor 2, part_entries 2048, rank 0, world 1, merge_rule 1). */
+ * hot_factor 2, part_entries 0 (auto), rank 0, world 1, merge_rule 1,
+ * n_proxy 2048). */
 void dg_default_params(dg_path_params *p);
 
 /* Statistics of one dg_run (device-side counters). */

@@ -1,7 +1,9 @@
 // C ABI of libdigraph.so (include/digraph.h): argument checking, lifecycle
 // and dispatch to the host preprocessing (dg_preprocess.cpp) and the CUDA
 // kernels (dg_kernels.cu).  No computation step of dg_run happens here.
+#include <algorithm>
 #include <cstring>
+#include <vector>
 #include <exception>
 #include <new>
 #include <string>
@@ -43,10 +45,11 @@ void dg_default_params(dg_path_params* p) {
     p->n_sub = 64;
     p->order = 0;
     p->hot_factor = 2.0f;
-    p->part_entries = 2048;
+    p->part_entries = 0;
     p->rank = 0;
     p->world = 1;
     p->merge_rule = 1;
+    p->n_proxy = 2048;
 }
 
 int dg_create(dg_graph** out, int device) {
@@ -113,8 +116,9 @@ int dg_build_paths(dg_graph* g, const dg_path_params* p) {
     dg_path_params q;
     dg_default_params(&q);
     if (p) q = *p;
-    if (q.d_max < 1 || q.n_sub < 1 || q.part_entries < 1 || q.world < 1 || q.world > 64 ||
-        q.rank < 0 || q.rank >= q.world || q.l_merge < 0 || q.merge_rule < 0 || q.merge_rule > 1)
+    if (q.d_max < 1 || q.n_sub < 1 || q.part_entries < 0 || q.world < 1 || q.world > 64 ||
+        q.rank < 0 || q.rank >= q.world || q.l_merge < 0 || q.merge_rule < 0 || q.merge_rule > 1 ||
+        q.n_proxy < 0 || q.n_proxy > 16384)
         return fail(DG_EINVAL, "dg_build_paths: bad parameters");
     dg::dev_free_work(g->work);
     dg::dev_free_layout(g->dev, true);
@@ -138,10 +142,9 @@ int dg_upload(dg_graph* g) {
     if (!g || !g->layout.built) return fail(DG_EINVAL, "dg_upload: no layout built");
     if (int rc0 = select_dev(g)) return rc0;
     std::string err;
-    dg::dev_free_work(g->work);
-    dg::dev_free_layout(g->dev, true);
-    g->uploaded = false;
-    int rc = dg::dev_upload_csr(g->dev, g->csr, err);
+    // a re-upload of the same layout copies into the existing device buffers
+    // (and keeps the work buffers); a new layout was freed by dg_build_paths
+    int rc = dg::dev_upload_csr(g->dev, g->csr, g->layout, err);
     if (!rc) rc = dg::dev_upload_layout(g->dev, g->layout, err);
     if (rc) { dg::dev_free_layout(g->dev, true); return fail(rc, err); }
     g->uploaded = true;
@@ -163,8 +166,13 @@ int dg_set_vertex_params(dg_graph* g, const double* p_inj, const double* p_cont,
     for (int64_t v = 0; v < g->csr.n; v++)
         if (!(p_cont[v] >= 0 && p_cont[v] < 1 && p_inj[v] >= 0))
             return fail(DG_EINVAL, "dg_set_vertex_params: need 0 <= p_cont < 1 and p_inj >= 0");
+    // to internal vertex ids
+    const auto& orig = g->layout.orig;
+    const int64_t n = g->csr.n;
+    std::vector<double> a(n), b(n), c(n);
+    for (int64_t u = 0; u < n; u++) { a[u] = p_inj[orig[u]]; b[u] = p_cont[orig[u]]; c[u] = inj[orig[u]]; }
     std::string err;
-    int rc = dg::dev_set_vertex_params(g->work, g->dev, p_inj, p_cont, inj, err);
+    int rc = dg::dev_set_vertex_params(g->work, g->dev, a.data(), b.data(), c.data(), err);
     return rc ? fail(rc, err) : DG_OK;
 }
 
@@ -191,7 +199,8 @@ int dg_run(dg_graph* g, int algo, int64_t source, double epsilon, double param, 
     if ((rc = select_dev(g))) return rc;
     if ((rc = ensure_uploaded(g))) return rc;
     g->run = dg::RunState();
-    g->run.algo = algo; g->run.mode = mode; g->run.source = source;
+    g->run.algo = algo; g->run.mode = mode;
+    g->run.source = (algo == DG_SSSP || algo == DG_BFS) ? g->layout.new_id[source] : 0;
     g->run.eps = epsilon; g->run.param = param;
     std::string err;
     rc = dg::dev_run(g->work, g->dev, g->run, max_rounds <= 0 ? 1000000 : max_rounds, err);
@@ -247,7 +256,7 @@ int dg_export_paths(const dg_graph* g, int64_t* path_off, int32_t* vertices, int
     const size_t P = L.path_off.size() - 1;
     if (path_off) std::memcpy(path_off, L.path_off.data(), sizeof(int64_t) * (P + 1));
     if (vertices)
-        for (size_t k = 0; k < L.e_idx.size(); k++) vertices[k] = (int32_t)(L.e_idx[k] & dg::kVMask);
+        for (size_t k = 0; k < L.e_idx.size(); k++) vertices[k] = L.orig[L.e_idx[k] & dg::kVMask];
     if (layer) std::memcpy(layer, L.layer.data(), sizeof(int32_t) * P);
     if (scc) std::memcpy(scc, L.scc.data(), sizeof(int64_t) * P);
     if (merged_index) std::memcpy(merged_index, L.merged_index.data(), sizeof(int64_t) * P);
@@ -264,7 +273,10 @@ int dg_boundary_size(const dg_graph* g, int64_t* n_boundary) {
 
 int dg_boundary_vertices(const dg_graph* g, int32_t* out) {
     if (!g || !g->layout.built || !out) return fail(DG_EINVAL, "dg_boundary_vertices: no layout built");
-    std::memcpy(out, g->layout.boundary.data(), sizeof(int32_t) * g->layout.boundary.size());
+    std::vector<int32_t> b(g->layout.boundary.size());
+    for (size_t k = 0; k < b.size(); k++) b[k] = g->layout.orig[g->layout.boundary[k]];
+    std::sort(b.begin(), b.end());
+    std::memcpy(out, b.data(), sizeof(int32_t) * b.size());
     return DG_OK;
 }
 
@@ -275,7 +287,8 @@ int dg_run_begin(dg_graph* g, int algo, int64_t source, double epsilon, double p
     if ((rc = select_dev(g))) return rc;
     if ((rc = ensure_uploaded(g))) return rc;
     g->run = dg::RunState();
-    g->run.algo = algo; g->run.mode = DG_MODE_PATH; g->run.source = source;
+    g->run.algo = algo; g->run.mode = DG_MODE_PATH;
+    g->run.source = (algo == DG_SSSP || algo == DG_BFS) ? g->layout.new_id[source] : 0;
     g->run.eps = epsilon; g->run.param = param;
     g->run.raw_states = g->layout.params.world > 1;
     std::string err;

@@ -9,8 +9,11 @@
 
 namespace dg {
 
-// Path entry encoding in e_idx (uint32): vertex id in bits 0..29,
+// Path entry encoding in e_idx (uint32): internal vertex id in bits 0..29,
 // bit 31 = first vertex of a path (head), bit 30 = last vertex (tail).
+// Internal ids: the n_proxy highest-degree vertices are renumbered to
+// [0, n_proxy) (shared-memory proxy vertices); every other
+// vertex keeps its id unless it was displaced by a hub.
 constexpr uint32_t kHead = 0x80000000u;
 constexpr uint32_t kTail = 0x40000000u;
 constexpr uint32_t kVMask = 0x3FFFFFFFu;
@@ -37,8 +40,14 @@ struct HostLayout {
     std::vector<uint32_t> e_idx;        // vertex | head | tail
     std::vector<int32_t> e_w;           // weight of the path edge INTO this entry (0 at heads)
     std::vector<int64_t> part_off;      // n_part+1
+    // internal numbering and the CSR in internal ids (device copy for the
+    // ablation, Adsorption weights and out-degrees)
+    int64_t n_proxy = 0;
+    std::vector<int32_t> new_id, orig;  // original -> internal, internal -> original
+    std::vector<int64_t> prow_ptr;
+    std::vector<int32_t> pcol, pw, poutdeg;
     // multi-rank
-    std::vector<int32_t> boundary;      // vertices present on >1 rank (ascending)
+    std::vector<int32_t> boundary;      // internal ids of vertices present on >1 rank (ascending)
     // stats
     int64_t n_layers = 0, n_dep_sccs = 0, giant = 0, paths_before_merge = 0, n_hot = 0;
     double preprocess_ms = 0;
@@ -53,6 +62,9 @@ struct DevLayout {
     int32_t* e_w = nullptr;
     int64_t* part_off = nullptr;
     int32_t* bnd = nullptr;
+    int32_t* new_id = nullptr;  // original -> internal
+    int32_t* orig = nullptr;    // internal -> original
+    int64_t n_proxy = 0;
     // CSR (for the vertex-centric ablation and per-vertex coefficients)
     int64_t* row_ptr = nullptr; int32_t* col = nullptr; int32_t* w = nullptr;
     int32_t* outdeg = nullptr;
@@ -75,7 +87,7 @@ struct RunState {
 
 // Kernel-side entry points (dg_kernels.cu).  All return 0 or DG_E*.
 int dev_select(int device, std::string& err);
-int dev_upload_csr(DevLayout& D, const HostCSR& g, std::string& err);
+int dev_upload_csr(DevLayout& D, const HostCSR& g, const HostLayout& L, std::string& err);
 int dev_upload_layout(DevLayout& D, const HostLayout& L, std::string& err);
 void dev_free_layout(DevLayout& D, bool csr_too);
 int dev_set_vertex_params(DevWork*& W, const DevLayout& D, const double* p_inj, const double* p_cont,

@@ -111,6 +111,8 @@ struct KParams {
     Counters* ctr;
     uint8_t* mark;
     const int32_t* scc_label;
+    const int32_t* orig;
+    int64_t n_proxy;
     float eps;
     unsigned long long eps_fx;
     int max_rounds;
@@ -217,10 +219,13 @@ __device__ void walk_minplus(const KParams& P, int64_t beg, int64_t end, const u
     const int lane = threadIdx.x & 31;
     uint32_t carry = INF;
     bool carry_live = false;
-    for (int64_t base = beg & ~(int64_t)3; base < end; base += 128) {
+    const int64_t first = beg & ~(int64_t)3;
+    uint4 code_nx = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
+    if (first + 4 * lane < end) code_nx = ld_stream_u4(P.e_idx + first + 4 * lane);
+    for (int64_t base = first; base < end; base += 128) {
         const int64_t i0 = base + 4 * lane;
-        uint4 code = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
-        if (i0 < end) code = ld_stream_u4(P.e_idx + i0);
+        const uint4 code = code_nx;  // prefetched in the previous iteration
+        if (i0 + 128 < end) code_nx = ld_stream_u4(P.e_idx + i0 + 128);
         uint32_t vtx[4];
         bool valid[4], act[4], any_act = false;
 #pragma unroll
@@ -355,9 +360,23 @@ constexpr float kFxInv = 2.3283064365386963e-10f;  // 2^-32
 __device__ __forceinline__ unsigned long long fx_from(float x) { return x > 0.f ? __float2ull_rz(x * kFxScale) : 0ull; }
 __device__ __forceinline__ float fx_to(unsigned long long v) { return __ull2float_rn(v) * kFxInv; }
 
+// Shared-memory proxies of the n_proxy highest-degree vertices (internal ids
+// [0, H)): "creates a proxy vertex in the shared memory of
+// each related SMX for each vertex with high in-degree, to accumulate the
+// pushed new states of its local mirrors ... sent to the master when the
+// partition assigned to this SMX has been handled".  Per CTA: the round-start
+// totals and stamps, the CTA's unflushed pushes, the path-edge coefficients.
+struct Proxies {
+    unsigned long long* T;
+    unsigned long long* acc;
+    float* coef;
+    int* stamp;
+    int64_t H;
+};
+
 template <bool ADS>
 __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round, Acc& acc,
-                           unsigned long long pol_stream, unsigned long long pol_keep) {
+                           unsigned long long pol_stream, unsigned long long pol_keep, const Proxies& px) {
     const int lane = threadIdx.x & 31;
     const unsigned long long eps = P.eps_fx;
     float carry = 0.f;
@@ -390,7 +409,15 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round
             T[k] = 0ull;
             cf[k] = 0.f;
             int stamp = -1;
-            if (valid[k]) ld_state_h(&P.vs_a[vtx[k]], T[k], cf[k], stamp, pol_keep);
+            if (valid[k]) {
+                if (vtx[k] < px.H) {
+                    T[k] = px.T[vtx[k]] + *(volatile unsigned long long*)&px.acc[vtx[k]];
+                    cf[k] = px.coef[vtx[k]];
+                    stamp = px.stamp[vtx[k]];
+                } else {
+                    ld_state_h(&P.vs_a[vtx[k]], T[k], cf[k], stamp, pol_keep);
+                }
+            }
             any_act |= stamp == round;
         }
         if (!__any_sync(0xffffffffu, any_act) && carry == 0.f) continue;
@@ -436,7 +463,8 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round
             if (!hd[k]) acc.edges++;
             const unsigned long long p = fx_from(pin[k]);
             if (p) {
-                atomicAdd(&P.vs_a[vtx[k]].T, p);  // no return value used: REDG
+                if (vtx[k] < px.H) atomicAdd(&px.acc[vtx[k]], p);  // proxy: shared-memory atomic
+                else atomicAdd(&P.vs_a[vtx[k]].T, p);               // master: REDG (no return)
                 acc.upd++;
             }
             if (!tl[k] && (pend[k] | p)) st_stream_u64_h(P.s_val + i0 + k, sv[k] + pend[k] + p, pol_stream);
@@ -557,12 +585,30 @@ __global__ void __launch_bounds__(kBlock, DG_PATH_MINB) path_kernel(KParams P) {
     const int lane = threadIdx.x & 31;
     constexpr bool kAccum = ALGO == DG_PAGERANK || ALGO == DG_ADSORPTION;
     const unsigned long long pol_stream = policy_evict_first(), pol_keep = policy_evict_last();
+    extern __shared__ unsigned long long dyn_smem[];
+    Proxies px{nullptr, nullptr, nullptr, nullptr, 0};
+    if (kAccum && P.n_proxy > 0) {
+        px.H = P.n_proxy;
+        px.T = dyn_smem;
+        px.acc = dyn_smem + px.H;
+        px.coef = reinterpret_cast<float*>(dyn_smem + 2 * px.H);
+        px.stamp = reinterpret_cast<int*>(px.coef + px.H);
+        for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) px.coef[i] = P.vs_a[i].coef;
+    }
     Acc acc;
     int r = 0;
     for (; r < P.max_rounds; r++) {
         const int round = P.ctr->round + r;  // ctr->round only changes after the loop
         const int cur = round & 1, nxt = cur ^ 1;
         if (*((volatile unsigned*)&P.ctr->active[cur]) == 0) break;
+        if (kAccum && px.H) {  // round-start snapshot of the proxied masters
+            for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) {
+                px.T[i] = P.vs_a[i].T;
+                px.stamp[i] = P.vs_a[i].stamp;
+                px.acc[i] = 0ull;
+            }
+            __syncthreads();
+        }
         const uint32_t* bcur = P.bits + (int64_t)cur * P.nw;
         uint32_t* bnxt = P.bits + (int64_t)nxt * P.nw;
         while (true) {
@@ -576,10 +622,15 @@ __global__ void __launch_bounds__(kBlock, DG_PATH_MINB) path_kernel(KParams P) {
             else if (ALGO == DG_WCC) walk_minplus<2>(P, beg, end, bcur, bnxt, acc);
             else if (ALGO == 100) walk_minplus<3>(P, beg, end, bcur, bnxt, acc);
             else if (ALGO == 101) walk_scc_bwd(P, beg, end, bcur, bnxt, acc);
-            else if (ALGO == DG_PAGERANK) walk_accum<false>(P, beg, end, round, acc, pol_stream, pol_keep);
-            else if (ALGO == DG_ADSORPTION) walk_accum<true>(P, beg, end, round, acc, pol_stream, pol_keep);
+            else if (ALGO == DG_PAGERANK) walk_accum<false>(P, beg, end, round, acc, pol_stream, pol_keep, px);
+            else if (ALGO == DG_ADSORPTION) walk_accum<true>(P, beg, end, round, acc, pol_stream, pol_keep, px);
         }
         if (kAccum) {
+            if (px.H) {  // send the proxies' accumulated pushes to their masters
+                __syncthreads();
+                for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x)
+                    if (px.acc[i]) atomicAdd(&P.vs_a[i].T, px.acc[i]);
+            }
             grid.sync();  // all pushes of the round landed
             accum_sweep(P, round + 1, acc.sig);
         }
@@ -721,9 +772,10 @@ __global__ void __launch_bounds__(kBlock) vertex_kernel(KParams P) {
 #define GRID_STRIDE(i, n) \
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < (n); i += (int64_t)gridDim.x * blockDim.x)
 
-__global__ void init_u_kernel(uint2* vs, int64_t n, int algo, int64_t source) {
+// WCC labels start as the ORIGINAL vertex id (reading R-CC: smallest original id wins)
+__global__ void init_u_kernel(uint2* vs, const int32_t* orig, int64_t n, int algo, int64_t source) {
     GRID_STRIDE(v, n) {
-        uint32_t val = (algo == DG_WCC) ? (uint32_t)v : (v == source ? 0u : INF);
+        uint32_t val = (algo == DG_WCC) ? (uint32_t)orig[v] : (v == source ? 0u : INF);
         vs[v] = make_uint2(val, 0u);
     }
 }
@@ -788,13 +840,17 @@ __global__ void sum_T_kernel(const float4* vf, const AccState* va, int64_t n, do
     for (int off = 16; off; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
     if ((threadIdx.x & 31) == 0) atomicAdd(out, s);
 }
-__global__ void out_pr_kernel(const float4* vf, const AccState* va, int64_t n, const double* sum, float* out,
-                              int normalize) {
+// outputs are indexed by ORIGINAL vertex id: out[v] = state[new_id[v]]
+__global__ void out_pr_kernel(const float4* vf, const AccState* va, const int32_t* new_id, int64_t n,
+                              const double* sum, float* out, int normalize) {
     const double inv = normalize ? 1.0 / *sum : 1.0;
-    GRID_STRIDE(v, n) out[v] = (float)(final_value(vf, va, v) * inv);
+    GRID_STRIDE(v, n) out[v] = (float)(final_value(vf, va, new_id[v]) * inv);
 }
-__global__ void out_u_kernel(const uint2* vs, int64_t n, uint32_t* out) {
-    GRID_STRIDE(v, n) out[v] = vs[v].x;
+__global__ void out_u_kernel(const uint2* vs, const int32_t* new_id, int64_t n, uint32_t* out) {
+    GRID_STRIDE(v, n) out[v] = vs[new_id[v]].x;
+}
+__global__ void out_i_kernel(const int32_t* x, const int32_t* new_id, int64_t n, int32_t* out) {
+    GRID_STRIDE(v, n) out[v] = x[new_id[v]];
 }
 __global__ void sum_f_kernel(const float* x, int64_t n, double* out) {
     double s = 0;
@@ -808,18 +864,19 @@ __global__ void scale_f_kernel(float* x, int64_t n, const double* sum) {
 }
 
 // ---- SCC helpers
-__global__ void scc_init_kernel(uint2* vs, const int32_t* label, uint8_t* mark, int64_t n) {
+// colours are ORIGINAL vertex ids so an SCC's label is its smallest original id
+__global__ void scc_init_kernel(uint2* vs, const int32_t* label, const int32_t* orig, uint8_t* mark, int64_t n) {
     GRID_STRIDE(v, n) {
-        vs[v] = make_uint2(label[v] < 0 ? (uint32_t)v : INF, 0u);
+        vs[v] = make_uint2(label[v] < 0 ? (uint32_t)orig[v] : INF, 0u);
         mark[v] = 0;
     }
 }
 // roots keep their own id as colour; they seed the backward phase's bitmap
-__global__ void scc_roots_kernel(const uint2* vs, const int32_t* label, uint8_t* mark, int64_t n, uint32_t* b,
-                                 Counters* ctr) {
+__global__ void scc_roots_kernel(const uint2* vs, const int32_t* label, const int32_t* orig, uint8_t* mark,
+                                 int64_t n, uint32_t* b, Counters* ctr) {
     unsigned cnt = 0;
     GRID_STRIDE(v, n) {
-        const bool root = label[v] < 0 && vs[v].x == (uint32_t)v;
+        const bool root = label[v] < 0 && vs[v].x == (uint32_t)orig[v];
         mark[v] = root;
         if (root) cnt += signal_vertex(b, (uint32_t)v);
     }
@@ -899,6 +956,10 @@ int dalloc(T** p, size_t count, int64_t& bytes, std::string& err) {
     return DG_OK;
 }
 template <typename T>
+int dalloc_once(T** p, size_t count, int64_t& bytes, std::string& err) {
+    return *p ? DG_OK : dalloc(p, count, bytes, err);
+}
+template <typename T>
 void dfree(T*& p) {
     if (p) cudaFree((void*)p);
     p = nullptr;
@@ -936,6 +997,7 @@ KParams make_params(const DevLayout& D, DevWork* W) {
     P.vlist0 = W->vlist[0]; P.vlist1 = W->vlist[1];
     P.ctr = W->ctr;
     P.mark = W->scc_mark; P.scc_label = W->scc_label;
+    P.orig = D.orig; P.n_proxy = D.n_proxy;
     return P;
 }
 
@@ -973,15 +1035,16 @@ int write_counters(DevWork* W, const Counters& c, std::string& err) {
     return DG_OK;
 }
 
-int coop_launch(DevWork* W, void* fn, KParams& P, RunState& S, std::string& err) {
+int coop_launch(DevWork* W, void* fn, KParams& P, RunState& S, std::string& err, size_t smem = 0) {
     int dev = 0, sms = 0, per = 0;
     CK(cudaGetDevice(&dev));
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, kBlock, 0));
+    if (smem) CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, kBlock, smem));
     const int grid = sms * std::max(1, per);
     void* args[] = {&P};
     CK(cudaEventRecord(W->kev0));
-    CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kBlock), args, 0, 0));
+    CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kBlock), args, smem, 0));
     CK(cudaGetLastError());
     CK(cudaEventRecord(W->kev1));
     CK(cudaEventSynchronize(W->kev1));
@@ -1009,7 +1072,10 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
         case 101: fn = (void*)path_kernel<101>; break;
         default: err = "bad algo"; return DG_EINVAL;
     }
-    return coop_launch(W, fn, P, S, err);
+    const bool accum = algo_k == DG_PAGERANK || algo_k == DG_ADSORPTION;
+    const size_t smem = accum ? (size_t)D.n_proxy * 24 : 0;
+    if (!accum) P.n_proxy = 0;
+    return coop_launch(W, fn, P, S, err, smem);
 }
 
 int launch_vertex(DevWork* W, const DevLayout& D, int algo, int rounds, RunState& S, std::string& err) {
@@ -1033,7 +1099,7 @@ int init_states(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
             c.active[0] = (unsigned)D.n;
             S.stats.kernel_launches += 2;
         } else {
-            init_u_kernel<<<g, 256>>>(W->vs_u, D.n, algo, S.source);
+            init_u_kernel<<<g, 256>>>(W->vs_u, D.orig, D.n, algo, S.source);
             int32_t s = (int32_t)S.source;
             CK(cudaMemcpy(W->vlist[0], &s, sizeof(int32_t), cudaMemcpyHostToDevice));
             c.active[0] = 1;
@@ -1044,13 +1110,13 @@ int init_states(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
     }
     CK(cudaMemsetAsync(W->bits, 0, sizeof(uint32_t) * 2 * W->nw));
     if (algo == DG_SSSP || algo == DG_BFS) {
-        init_u_kernel<<<g, 256>>>(W->vs_u, D.n, algo, S.source);
+        init_u_kernel<<<g, 256>>>(W->vs_u, D.orig, D.n, algo, S.source);
         bits_set_one_kernel<<<1, 1>>>(W->bits, S.source);
         c.active[0] = 1;
         S.stats.kernel_launches += 2;
     } else {
         if (algo == DG_WCC) {
-            init_u_kernel<<<g, 256>>>(W->vs_u, D.n, algo, 0);
+            init_u_kernel<<<g, 256>>>(W->vs_u, D.orig, D.n, algo, 0);
         } else {
             init_acc_kernel<<<g, 256>>>(W->vs_a, W->sigma, D.outdeg, algo == DG_ADSORPTION ? W->ads_base : nullptr,
                                         D.n, (float)S.param);
@@ -1097,7 +1163,7 @@ int run_scc(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, std
     const int rounds = (int)std::min<int64_t>(max_rounds, 1 << 30);
     for (int64_t it = 0;; it++) {
         // forward colouring: every unassigned vertex starts with its own id, all signalled
-        scc_init_kernel<<<g, 256>>>(W->vs_u, W->scc_label, W->scc_mark, D.n);
+        scc_init_kernel<<<g, 256>>>(W->vs_u, W->scc_label, D.orig, W->scc_mark, D.n);
         CK(cudaMemsetAsync(W->bits, 0, sizeof(uint32_t) * 2 * W->nw));
         bits_all_kernel<<<grid_1d(W->nw), 256>>>(W->bits, W->nw, D.n);
         Counters c0{};
@@ -1111,7 +1177,7 @@ int run_scc(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, std
         CK(cudaMemsetAsync(W->bits, 0, sizeof(uint32_t) * 2 * W->nw));
         Counters c2{};
         if ((rc = write_counters(W, c2, err))) return rc;
-        scc_roots_kernel<<<g, 256>>>(W->vs_u, W->scc_label, W->scc_mark, D.n, W->bits, W->ctr);
+        scc_roots_kernel<<<g, 256>>>(W->vs_u, W->scc_label, D.orig, W->scc_mark, D.n, W->bits, W->ctr);
         S.stats.kernel_launches += 1;
         if ((rc = launch_path(W, D, 101, rounds, S, err))) return rc;
         Counters c3;
@@ -1152,7 +1218,7 @@ int dev_select(int device, std::string& err) {
     return DG_OK;
 }
 
-int dev_upload_csr(DevLayout& D, const HostCSR& g, std::string& err) {
+int dev_upload_csr(DevLayout& D, const HostCSR& g, const HostLayout& L, std::string& err) {
     int dev_count = 0;
     if (cudaGetDeviceCount(&dev_count) != cudaSuccess || dev_count == 0) {
         err = "no CUDA device available (the DiGraph hot path has no CPU fallback)";
@@ -1163,16 +1229,22 @@ int dev_upload_csr(DevLayout& D, const HostCSR& g, std::string& err) {
     D.h2d_bytes = 0;
     g_h2d_counter = &D.h2d_bytes;
     g_pin_list = &D.pinned;
-    if ((rc = dalloc(&D.row_ptr, g.n + 1, D.bytes, err))) return rc;
-    if ((rc = dalloc(&D.col, g.m + kPad, D.bytes, err))) return rc;
-    if ((rc = dalloc(&D.outdeg, g.n + 1, D.bytes, err))) return rc;
-    if ((rc = h2d(D.row_ptr, g.row_ptr.data(), g.n + 1, err))) return rc;
-    if ((rc = h2d(D.col, g.col.data(), g.m, err))) return rc;
-    if ((rc = h2d(D.outdeg, g.outdeg.data(), g.n, err))) return rc;
+    // the CSR in internal vertex ids (HostLayout), plus both id maps
+    if ((rc = dalloc_once(&D.row_ptr, g.n + 1, D.bytes, err))) return rc;
+    if ((rc = dalloc_once(&D.col, g.m + kPad, D.bytes, err))) return rc;
+    if ((rc = dalloc_once(&D.outdeg, g.n + 1, D.bytes, err))) return rc;
+    if ((rc = dalloc_once(&D.new_id, g.n + 1, D.bytes, err))) return rc;
+    if ((rc = dalloc_once(&D.orig, g.n + 1, D.bytes, err))) return rc;
+    if ((rc = h2d(D.row_ptr, L.prow_ptr.data(), g.n + 1, err))) return rc;
+    if ((rc = h2d(D.col, L.pcol.data(), g.m, err))) return rc;
+    if ((rc = h2d(D.outdeg, L.poutdeg.data(), g.n, err))) return rc;
+    if ((rc = h2d(D.new_id, L.new_id.data(), g.n, err))) return rc;
+    if ((rc = h2d(D.orig, L.orig.data(), g.n, err))) return rc;
     if (g.has_w) {
-        if ((rc = dalloc(&D.w, g.m + kPad, D.bytes, err))) return rc;
-        if ((rc = h2d(D.w, g.w.data(), g.m, err))) return rc;
+        if ((rc = dalloc_once(&D.w, g.m + kPad, D.bytes, err))) return rc;
+        if ((rc = h2d(D.w, L.pw.data(), g.m, err))) return rc;
     }
+    D.n_proxy = L.n_proxy;
     return DG_OK;
 }
 
@@ -1183,10 +1255,10 @@ int dev_upload_layout(DevLayout& D, const HostLayout& L, std::string& err) {
     D.M = (int64_t)L.e_idx.size();
     D.n_part = (int64_t)L.part_off.size() - 1;
     D.n_bnd = (int64_t)L.boundary.size();
-    if ((rc = dalloc(&D.e_idx, D.M + kPad, D.bytes, err))) return rc;
-    if ((rc = dalloc(&D.e_w, D.M + kPad, D.bytes, err))) return rc;
-    if ((rc = dalloc(&D.part_off, D.n_part + 1, D.bytes, err))) return rc;
-    if ((rc = dalloc(&D.bnd, D.n_bnd + 1, D.bytes, err))) return rc;
+    if ((rc = dalloc_once(&D.e_idx, D.M + kPad, D.bytes, err))) return rc;
+    if ((rc = dalloc_once(&D.e_w, D.M + kPad, D.bytes, err))) return rc;
+    if ((rc = dalloc_once(&D.part_off, D.n_part + 1, D.bytes, err))) return rc;
+    if ((rc = dalloc_once(&D.bnd, D.n_bnd + 1, D.bytes, err))) return rc;
     CK(cudaMemset(D.e_idx + D.M, 0, sizeof(uint32_t) * kPad));
     CK(cudaMemset(D.e_w + D.M, 0, sizeof(int32_t) * kPad));
     if ((rc = h2d(D.e_idx, L.e_idx.data(), D.M, err))) return rc;
@@ -1207,7 +1279,7 @@ void dev_unpin_all(DevLayout& D) {
 
 void dev_free_layout(DevLayout& D, bool csr_too) {
     dfree(D.e_idx); dfree(D.e_w); dfree(D.part_off); dfree(D.bnd);
-    if (csr_too) { dfree(D.row_ptr); dfree(D.col); dfree(D.w); dfree(D.outdeg); }
+    if (csr_too) { dfree(D.row_ptr); dfree(D.col); dfree(D.w); dfree(D.outdeg); dfree(D.new_id); dfree(D.orig); }
     D.bytes = 0;
     D.M = D.n_part = D.n_bnd = 0;
 }
@@ -1384,11 +1456,12 @@ int dev_get_states(DevWork* W, const DevLayout& D, const RunState& S, void* out,
         const AccState* va = S.mode == DG_MODE_PATH ? W->vs_a : nullptr;
         CK(cudaMemset(W->dsum, 0, sizeof(double)));
         if (S.algo == DG_PAGERANK) sum_T_kernel<<<g, 256>>>(W->vs_f, va, n, W->dsum);
-        out_pr_kernel<<<g, 256>>>(W->vs_f, va, n, W->dsum, (float*)dst, S.algo == DG_PAGERANK && !S.raw_states);
+        out_pr_kernel<<<g, 256>>>(W->vs_f, va, D.new_id, n, W->dsum, (float*)dst,
+                                  S.algo == DG_PAGERANK && !S.raw_states);
     } else if (S.algo == DG_SCC) {
-        CK(cudaMemcpy(dst, W->scc_label, 4 * (size_t)n, cudaMemcpyDeviceToDevice));
+        out_i_kernel<<<g, 256>>>(W->scc_label, D.new_id, n, (int32_t*)dst);
     } else {
-        out_u_kernel<<<g, 256>>>(W->vs_u, n, (uint32_t*)dst);
+        out_u_kernel<<<g, 256>>>(W->vs_u, D.new_id, n, (uint32_t*)dst);
     }
     CK(cudaGetLastError());
     if (tmp) {

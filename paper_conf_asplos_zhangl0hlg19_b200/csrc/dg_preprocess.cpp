@@ -386,7 +386,14 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     std::stable_sort(order.begin(), order.end(), [&](int64_t a, int64_t b) { return pri[a] > pri[b]; });
 
     // ---- partitions over the priority order (greedy, whole paths)
-    const int64_t target = std::max<int32_t>(1, p.part_entries);
+    // part_entries == 0: auto -- about 16K partitions (several per resident
+    // warp of a 148-SM grid), between 128 and 2048 entries each
+    int64_t target = p.part_entries;
+    if (target <= 0) {
+        int64_t tot = 0;
+        for (int64_t i = 0; i < P; i++) tot += nvert[i];
+        target = std::min<int64_t>(2048, std::max<int64_t>(128, tot / 16384));
+    }
     std::vector<int64_t> gpart_first{0};  // global partition -> first index in `order`
     {
         int64_t acc = 0;
@@ -400,8 +407,52 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     const int64_t G = (int64_t)gpart_first.size() - 1;
     const int world = std::max(1, p.world), rank = p.rank;
 
-    // ---- boundary vertices: present in partitions of >1 rank (round-robin owner q % world);
-    // owner of a vertex = lowest rank holding it (rank 0 for vertices on no path)
+    // ---- internal numbering: the H highest-degree vertices (ties by id) get ids
+    // [0, H) so the path kernel can keep them as shared-memory proxies; a
+    // non-hub vertex with id < H takes a freed hub id (both ascending)
+    const int64_t H = std::min<int64_t>(std::max<int32_t>(0, p.n_proxy), n);
+    L.n_proxy = H;
+    L.new_id.resize(n);
+    L.orig.resize(n);
+    {
+        std::vector<int32_t> byd(n);
+        std::iota(byd.begin(), byd.end(), 0);
+        std::partial_sort(byd.begin(), byd.begin() + H, byd.end(), [&](int32_t a, int32_t b) {
+            return deg[a] != deg[b] ? deg[a] > deg[b] : a < b;
+        });
+        std::vector<uint8_t> is_hub(n, 0);
+        std::vector<int32_t> freed, displaced;
+        for (int64_t i = 0; i < H; i++) is_hub[byd[i]] = 1;
+        for (int64_t v = 0; v < n; v++) L.new_id[v] = (int32_t)v;
+        for (int64_t i = 0; i < H; i++) {
+            L.new_id[byd[i]] = (int32_t)i;
+            if (byd[i] >= H) freed.push_back(byd[i]);
+        }
+        for (int64_t v = 0; v < H; v++)
+            if (!is_hub[v]) displaced.push_back((int32_t)v);
+        std::sort(freed.begin(), freed.end());
+        for (size_t j = 0; j < displaced.size(); j++) L.new_id[displaced[j]] = freed[j];
+        for (int64_t v = 0; v < n; v++) L.orig[L.new_id[v]] = (int32_t)v;
+    }
+    // CSR in internal ids
+    L.prow_ptr.assign(n + 1, 0);
+    L.poutdeg.resize(n);
+    for (int64_t u = 0; u < n; u++) {
+        L.poutdeg[u] = g.outdeg[L.orig[u]];
+        L.prow_ptr[u + 1] = L.prow_ptr[u] + L.poutdeg[u];
+    }
+    L.pcol.resize(m);
+    if (g.has_w) L.pw.resize(m);
+    #pragma omp parallel for schedule(dynamic, 4096)
+    for (int64_t u = 0; u < n; u++) {
+        const int64_t src0 = g.row_ptr[L.orig[u]], len = L.poutdeg[u], dst0 = L.prow_ptr[u];
+        for (int64_t k = 0; k < len; k++) {
+            L.pcol[dst0 + k] = L.new_id[g.col[src0 + k]];
+            if (g.has_w) L.pw[dst0 + k] = g.w[src0 + k];
+        }
+    }
+
+    // ---- boundary vertices: present in partitions of >1 rank (round-robin owner q % world)
     if (world > 1) {
         std::vector<uint64_t> present(n, 0);  // ranks whose partitions hold v
         for (int64_t q = 0; q < G; q++) {
@@ -412,7 +463,8 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
             }
         }
         for (int64_t v = 0; v < n; v++)
-            if (__builtin_popcountll(present[v]) > 1) L.boundary.push_back((int32_t)v);
+            if (__builtin_popcountll(present[v]) > 1) L.boundary.push_back(L.new_id[v]);
+        std::sort(L.boundary.begin(), L.boundary.end());
     }
 
     phase("priority+partitions");
@@ -423,7 +475,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
         for (int64_t r = gpart_first[q]; r < gpart_first[q + 1]; r++) {
             int64_t i = order[r];
             for (int64_t k = moff[i]; k < moff[i + 1]; k++) {
-                uint32_t code = (uint32_t)mv[k];
+                uint32_t code = (uint32_t)L.new_id[mv[k]];
                 if (k == moff[i]) code |= kHead;
                 if (k == moff[i + 1] - 1) code |= kTail;
                 L.e_idx.push_back(code);

@@ -72,12 +72,13 @@ class DiGraph:
         return self.load_csr(g.n, g.row_ptr, g.col, g.w)
 
     def build_paths(self, d_max=16, l_merge=64, n_sub=64, order="degree", hot_factor=2.0,
-                    part_entries=2048, rank=0, world=1, merge_rule="relaxed"):
+                    part_entries=0, rank=0, world=1, merge_rule="relaxed", n_proxy=2048):
         p = default_params()
         p.d_max, p.l_merge, p.n_sub = d_max, l_merge, n_sub
         p.order = 0 if order == "degree" else 1
         p.hot_factor, p.part_entries, p.rank, p.world = hot_factor, part_entries, rank, world
         p.merge_rule = {"paper": 0, "relaxed": 1}[merge_rule]
+        p.n_proxy = n_proxy
         check(self._L.dg_build_paths(self._h, ctypes.byref(p)), "dg_build_paths")
         return self
 
