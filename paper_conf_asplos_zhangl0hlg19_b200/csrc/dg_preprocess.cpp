@@ -79,25 +79,26 @@ struct Decomposer {
     }
 };
 
-// Iterative Tarjan over a CSR graph; comp[v] = SCC id in completion order
-// (reverse topological order of the condensation).
-int64_t tarjan(int64_t N, const std::vector<int64_t>& ptr, const std::vector<int64_t>& adj,
-               std::vector<int64_t>& comp) {
-    std::vector<int64_t> index(N, -1), low(N, 0), it(N, 0);
+// Iterative Tarjan over a CSR graph (node ids < 2^31); comp[v] = SCC id in
+// completion order (reverse topological order of the condensation).
+int32_t tarjan(int32_t N, const std::vector<int64_t>& ptr, const std::vector<int32_t>& adj,
+               std::vector<int32_t>& comp) {
+    std::vector<int32_t> index(N, -1), low(N, 0);
+    std::vector<int64_t> it(N, 0);
     std::vector<uint8_t> onst(N, 0);
-    std::vector<int64_t> st, work;
+    std::vector<int32_t> st, work;
     st.reserve(1024); work.reserve(1024);
     comp.assign(N, -1);
-    int64_t counter = 0, ncomp = 0;
-    for (int64_t r = 0; r < N; r++) {
+    int32_t counter = 0, ncomp = 0;
+    for (int32_t r = 0; r < N; r++) {
         if (index[r] != -1) continue;
         index[r] = low[r] = counter++;
         st.push_back(r); onst[r] = 1; it[r] = ptr[r];
         work.push_back(r);
         while (!work.empty()) {
-            int64_t v = work.back();
+            int32_t v = work.back();
             if (it[v] < ptr[v + 1]) {
-                int64_t u = adj[it[v]++];
+                int32_t u = adj[it[v]++];
                 if (index[u] == -1) {
                     index[u] = low[u] = counter++;
                     st.push_back(u); onst[u] = 1; it[u] = ptr[u];
@@ -107,10 +108,10 @@ int64_t tarjan(int64_t N, const std::vector<int64_t>& ptr, const std::vector<int
                 }
             } else {
                 work.pop_back();
-                if (!work.empty()) { int64_t p = work.back(); low[p] = std::min(low[p], low[v]); }
+                if (!work.empty()) { int32_t q = work.back(); low[q] = std::min(low[q], low[v]); }
                 if (low[v] == index[v]) {
                     while (true) {
-                        int64_t x = st.back(); st.pop_back(); onst[x] = 0;
+                        int32_t x = st.back(); st.pop_back(); onst[x] = 0;
                         comp[x] = ncomp;
                         if (x == v) break;
                     }
@@ -208,33 +209,41 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
             pv.insert(pv.end(), s.pv.begin(), s.pv.end());
             pw.insert(pw.end(), s.pw.begin(), s.pw.end());
             for (size_t i = 1; i < s.start.size(); i++) poff.push_back(base + s.start[i]);
-            SubOut().pv.swap(s.pv);
+            std::vector<int32_t>().swap(s.pv);
+            std::vector<int32_t>().swap(s.pw);
+            std::vector<int64_t>().swap(s.start);
         }
     }
     const int64_t P0 = (int64_t)poff.size() - 1;
     L.paths_before_merge = P0;
+    if (P0 >= INT32_MAX || P0 + n >= INT32_MAX) throw std::runtime_error("too many paths for 32-bit path ids");
+    { std::vector<SubOut>().swap(subs); std::vector<std::vector<uint32_t>>().swap(vis); }
 
     phase("concatenate");
     // ---- short-path merging (reading R-MERGE):
     // pair the k-th path ending at x with the k-th path starting at x, cut
     // cycles before their lowest index, cut chains into <= l_merge edges,
     // order merged paths by their first piece.
-    std::vector<int64_t> nxt(P0, -1), prv(P0, -1);
+    std::vector<int32_t> nxt(P0, -1), prv(P0, -1);
     if (p.l_merge > 0 && P0 > 1) {
-        std::vector<int64_t> eptr(n + 1, 0), sptr(n + 1, 0), elist(P0), slist(P0);
+        std::vector<int64_t> eptr(n + 1, 0), sptr(n + 1, 0);
+        std::vector<int32_t> elist(P0), slist(P0);
         for (int64_t i = 0; i < P0; i++) { eptr[pv[poff[i + 1] - 1] + 1]++; sptr[pv[poff[i]] + 1]++; }
         for (int64_t v = 0; v < n; v++) { eptr[v + 1] += eptr[v]; sptr[v + 1] += sptr[v]; }
         {
             std::vector<int64_t> fe(eptr.begin(), eptr.end() - 1), fs(sptr.begin(), sptr.end() - 1);
-            for (int64_t i = 0; i < P0; i++) { elist[fe[pv[poff[i + 1] - 1]]++] = i; slist[fs[pv[poff[i]]]++] = i; }
+            for (int64_t i = 0; i < P0; i++) {
+                elist[fe[pv[poff[i + 1] - 1]]++] = (int32_t)i;
+                slist[fs[pv[poff[i]]]++] = (int32_t)i;
+            }
         }
         #pragma omp parallel for schedule(dynamic, 4096)
         for (int64_t x = 0; x < n; x++) {
             const int64_t na = eptr[x + 1] - eptr[x], nb = sptr[x + 1] - sptr[x];
             if (!na || !nb) continue;
             if (p.merge_rule == 0 && g.indeg[x] > 1 && g.outdeg[x] > 1 && inner[x]) continue;
-            int64_t* A = &elist[eptr[x]];
-            int64_t* B = &slist[sptr[x]];
+            int32_t* A = &elist[eptr[x]];
+            int32_t* B = &slist[sptr[x]];
             for (int64_t k = 0; k < std::min(na, nb); k++) {
                 if (A[k] == B[k]) {
                     if (k + 1 < nb) std::swap(B[k], B[k + 1]);
@@ -247,11 +256,12 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     }
     // chains (start where nothing links in), then cycles cut before their lowest index
     std::vector<uint8_t> seen(P0, 0);
-    std::vector<int64_t> seg_first, seg_len;   // segments: first piece, #pieces
-    std::vector<int64_t> seg_pieces;           // pieces in chain order, segments contiguous per chain
-    auto walk_chain = [&](int64_t s0, std::vector<int64_t>& pieces, std::vector<int64_t>& sf, std::vector<int64_t>& sl) {
-        int64_t cur_len = 0, cur_n = 0;
-        for (int64_t j = s0; j != -1 && !seen[j]; j = nxt[j]) {
+    std::vector<int32_t> seg_first, seg_len;   // segments: first piece, #pieces
+    std::vector<int32_t> seg_pieces;           // pieces in chain order, segments contiguous per chain
+    auto walk_chain = [&](int32_t s0, std::vector<int32_t>& pieces, std::vector<int32_t>& sf, std::vector<int32_t>& sl) {
+        int64_t cur_len = 0;
+        int32_t cur_n = 0;
+        for (int32_t j = s0; j != -1 && !seen[j]; j = nxt[j]) {
             seen[j] = 1;
             const int64_t e = poff[j + 1] - poff[j] - 1;
             if (cur_n && cur_len + e > p.l_merge) { sl.push_back(cur_n); cur_n = 0; cur_len = 0; }
@@ -263,24 +273,25 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     };
     {
         const int nth = omp_get_max_threads();
-        std::vector<std::vector<int64_t>> tp(nth), tf(nth), tl(nth);
+        std::vector<std::vector<int32_t>> tp(nth), tf(nth), tl(nth);
         #pragma omp parallel for schedule(dynamic, 4096)
         for (int64_t i = 0; i < P0; i++)
-            if (prv[i] == -1) { int t = omp_get_thread_num(); walk_chain(i, tp[t], tf[t], tl[t]); }
+            if (prv[i] == -1) { int t = omp_get_thread_num(); walk_chain((int32_t)i, tp[t], tf[t], tl[t]); }
         for (int t = 0; t < nth; t++) {
             seg_pieces.insert(seg_pieces.end(), tp[t].begin(), tp[t].end());
             seg_first.insert(seg_first.end(), tf[t].begin(), tf[t].end());
             seg_len.insert(seg_len.end(), tl[t].begin(), tl[t].end());
         }
         for (int64_t i = 0; i < P0; i++)
-            if (!seen[i]) walk_chain(i, seg_pieces, seg_first, seg_len);
+            if (!seen[i]) walk_chain((int32_t)i, seg_pieces, seg_first, seg_len);
     }
+    { std::vector<int32_t>().swap(nxt); std::vector<int32_t>().swap(prv); std::vector<uint8_t>().swap(seen); }
     const int64_t P = (int64_t)seg_first.size();
     std::vector<int64_t> seg_start(P + 1, 0);   // into seg_pieces
     for (int64_t s2 = 0; s2 < P; s2++) seg_start[s2 + 1] = seg_start[s2] + seg_len[s2];
-    std::vector<int64_t> sorder(P);
+    std::vector<int32_t> sorder(P);
     std::iota(sorder.begin(), sorder.end(), 0);
-    std::sort(sorder.begin(), sorder.end(), [&](int64_t a, int64_t b) { return seg_first[a] < seg_first[b]; });
+    std::sort(sorder.begin(), sorder.end(), [&](int32_t a, int32_t b) { return seg_first[a] < seg_first[b]; });
     // materialise merged paths (merge order) in parallel
     std::vector<int64_t> moff(P + 1, 0);
     for (int64_t r = 0; r < P; r++) {
@@ -322,7 +333,8 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     // vertex node P+x -> path node j for every x left by an edge of j.
     // Reachability between path nodes equals reachability in G'.
     const int64_t N = P + n;
-    std::vector<int64_t> aptr(N + 1, 0), adj;
+    std::vector<int64_t> aptr(N + 1, 0);
+    std::vector<int32_t> adj;
     std::vector<int64_t> layer_of_path(P, 0), scc_label(P, 0);
     int64_t n_layers = 0, n_dep_sccs = 0, giant = 0;
     {
@@ -335,11 +347,11 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
         adj.resize(aptr[N]);
         std::vector<int64_t> fill(aptr.begin(), aptr.end() - 1);
         for (int64_t i = 0; i < P; i++) {
-            for (int64_t k = moff[i] + 1; k < moff[i + 1]; k++) adj[fill[i]++] = P + mv[k];
-            for (int64_t k = moff[i]; k < moff[i + 1] - 1; k++) adj[fill[P + mv[k]]++] = i;
+            for (int64_t k = moff[i] + 1; k < moff[i + 1]; k++) adj[fill[i]++] = (int32_t)(P + mv[k]);
+            for (int64_t k = moff[i]; k < moff[i + 1] - 1; k++) adj[fill[P + mv[k]]++] = (int32_t)i;
         }
-        std::vector<int64_t> comp;
-        int64_t nc = tarjan(N, aptr, adj, comp);
+        std::vector<int32_t> comp;
+        int64_t nc = tarjan((int32_t)N, aptr, adj, comp);
         // group nodes by comp; comps are numbered in reverse topological order
         std::vector<int64_t> cptr(nc + 1, 0), cnodes(N);
         for (int64_t x = 0; x < N; x++) cptr[comp[x] + 1]++;
@@ -372,7 +384,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
         for (int64_t c = 0; c < nc; c++)
             if (npaths[c] > 0) { n_dep_sccs++; giant = std::max(giant, npaths[c]); }
     }
-    { std::vector<int64_t>().swap(adj); std::vector<int64_t>().swap(aptr); }
+    { std::vector<int32_t>().swap(adj); std::vector<int64_t>().swap(aptr); }
 
     phase("dependency DAG");
     // ---- priority Pri(p) = alpha*D(p)*N(p) - L(p)
