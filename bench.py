@@ -287,22 +287,35 @@ def main():
             "kernel_share_of_step": kernel_ms / ms if ms else None}
 
     extras = {}
-    if not args.no_extras and rank == 0 and world == 1:
-        # end-to-end through the public API with host buffers: H2D upload of
-        # the graph layout, the run, D2H of the states
+    if not args.no_extras:
+        # end-to-end through the public API with host buffers, every step: H2D
+        # upload of the graph layout, the run (multi-rank protocol for N > 1),
+        # D2H of the states (gathered over ranks for N > 1)
         e2e_t = []
         for _ in range(max(2, min(args.steps, 3))):
             torch.cuda.synchronize()
+            if world > 1:
+                dist.barrier()
             t = time.perf_counter()
             dg.upload()
-            dg.run(args.algo, mode=args.mode, **run_kw)
-            out = dg.get_states()
+            if world == 1:
+                dg.run(args.algo, mode=args.mode, **run_kw)
+                out = dg.get_states()
+                d2h = int(out.nbytes)
+            else:
+                parallel.run_distributed(dg, args.algo, device=torch.device("cuda", local), **run_kw)
+                out = parallel.gather_states(dg, args.algo, g.n, device=torch.device("cuda", local)).cpu()
+                d2h = out.numel() * out.element_size()
             torch.cuda.synchronize()
-            e2e_t.append(time.perf_counter() - t)
+            dt = torch.tensor([time.perf_counter() - t], dtype=torch.float64, device="cuda")
+            if world > 1:
+                dist.all_reduce(dt, op=dist.ReduceOp.MAX)
+            e2e_t.append(float(dt.item()))
         info2 = dg.layout_info()
         e2e_s = statistics.median(e2e_t)
         extras["e2e"] = {"value": g.m / e2e_s, "unit": "edges/s", "h2d_bytes_per_step": info2["h2d_bytes"],
-                         "d2h_bytes_per_step": int(out.nbytes), "ms_per_step": e2e_s * 1e3}
+                         "d2h_bytes_per_step": d2h, "ms_per_step": e2e_s * 1e3}
+    if not args.no_extras and rank == 0 and world == 1:
         # vertex-centric ablation (north_star: total vertex updates next to it)
         if args.algo in ("pagerank", "sssp", "bfs"):
             other = "vertex" if args.mode == "path" else "path"

@@ -52,6 +52,9 @@ constexpr int kPad = 256;  // zero entries after every per-entry array
 #ifndef DG_PATH_MINB
 #define DG_PATH_MINB 3  // resident CTAs per SM requested for the path kernel
 #endif
+#ifndef DG_PROXY_REFRESH
+#define DG_PROXY_REFRESH 8  // partitions a CTA walks between mid-round proxy flushes (0 = round end only)
+#endif
 
 // device counters of a run
 struct Counters {
@@ -586,6 +589,7 @@ __global__ void __launch_bounds__(kBlock, DG_PATH_MINB) path_kernel(KParams P) {
     constexpr bool kAccum = ALGO == DG_PAGERANK || ALGO == DG_ADSORPTION;
     const unsigned long long pol_stream = policy_evict_first(), pol_keep = policy_evict_last();
     extern __shared__ unsigned long long dyn_smem[];
+    __shared__ int s_done;
     Proxies px{nullptr, nullptr, nullptr, nullptr, 0};
     if (kAccum && P.n_proxy > 0) {
         px.H = P.n_proxy;
@@ -607,6 +611,7 @@ __global__ void __launch_bounds__(kBlock, DG_PATH_MINB) path_kernel(KParams P) {
                 px.stamp[i] = P.vs_a[i].stamp;
                 px.acc[i] = 0ull;
             }
+            if (threadIdx.x == 0) s_done = 0;
             __syncthreads();
         }
         const uint32_t* bcur = P.bits + (int64_t)cur * P.nw;
@@ -616,6 +621,22 @@ __global__ void __launch_bounds__(kBlock, DG_PATH_MINB) path_kernel(KParams P) {
             if (lane == 0) t = atomicAdd(&P.ctr->ticket[cur], 1u);
             t = __shfl_sync(0xffffffffu, t, 0);
             if (t >= (unsigned)P.n_part) break;
+            if (kAccum && px.H && DG_PROXY_REFRESH > 0) {
+                // every DG_PROXY_REFRESH partitions of this CTA, one warp sends the
+                // proxies' pushes to their masters and refreshes the snapshot, so
+                // hub totals propagate between CTAs within the round
+                int c = 0;
+                if (lane == 0) c = atomicAdd(&s_done, 1) + 1;
+                c = __shfl_sync(0xffffffffu, c, 0);
+                if (c % DG_PROXY_REFRESH == 0) {
+                    for (int64_t i = lane; i < px.H; i += 32) {
+                        const unsigned long long a = atomicExch(&px.acc[i], 0ull);
+                        if (a) atomicAdd(&P.vs_a[i].T, a);
+                    }
+                    __syncwarp();
+                    for (int64_t i = lane; i < px.H; i += 32) px.T[i] = *(volatile unsigned long long*)&P.vs_a[i].T;
+                }
+            }
             const int64_t beg = P.part_off[t], end = P.part_off[t + 1];
             if (ALGO == DG_SSSP) walk_minplus<0>(P, beg, end, bcur, bnxt, acc);
             else if (ALGO == DG_BFS) walk_minplus<1>(P, beg, end, bcur, bnxt, acc);
