@@ -172,12 +172,16 @@ __device__ __forceinline__ float4 ld_stream_f4_h(const float* p, unsigned long l
                  : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p), "l"(pol));
     return r;
 }
+// 256-bit (sm_100) vector load/store of a lane's four 64-bit mirrors
 __device__ __forceinline__ void ld_stream_u64x4_h(const unsigned long long* p, unsigned long long (&o)[4],
                                                   unsigned long long pol) {
-    asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;"
-                 : "=l"(o[0]), "=l"(o[1]) : "l"(p), "l"(pol));
-    asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;"
-                 : "=l"(o[2]), "=l"(o[3]) : "l"(p + 2), "l"(pol));
+    asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=l"(o[0]), "=l"(o[1]), "=l"(o[2]), "=l"(o[3]) : "l"(p), "l"(pol));
+}
+__device__ __forceinline__ void st_stream_u64x4_h(unsigned long long* p, const unsigned long long (&v)[4],
+                                                  unsigned long long pol) {
+    asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.u64 [%0], {%1,%2,%3,%4}, %5;"
+                 ::"l"(p), "l"(v[0]), "l"(v[1]), "l"(v[2]), "l"(v[3]), "l"(pol));
 }
 __device__ __forceinline__ void st_stream_u64_h(unsigned long long* p, unsigned long long v, unsigned long long pol) {
     asm volatile("st.global.L1::no_allocate.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(pol));
@@ -459,6 +463,7 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round
             prev = al[k] + be[k] * prev;
         }
         carry = __shfl_sync(0xffffffffu, prev, 31);
+        bool dirty = false;
 #pragma unroll
         for (int k = 0; k < 4; k++) {
             if (!valid[k]) continue;
@@ -470,7 +475,19 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round
                 else atomicAdd(&P.vs_a[vtx[k]].T, p);               // master: REDG (no return)
                 acc.upd++;
             }
-            if (!tl[k] && (pend[k] | p)) st_stream_u64_h(P.s_val + i0 + k, sv[k] + pend[k] + p, pol_stream);
+            if (!tl[k] && (pend[k] | p)) { sv[k] += pend[k] + p; dirty = true; }
+        }
+        // lanes whose four entries all lie in this partition write one 256-bit
+        // store; lanes at the partition's ends write only their own entries
+        // (the neighbouring partition's mirrors belong to another warp)
+        if (dirty) {
+            if (i0 >= beg && i0 + 3 < end) {
+                st_stream_u64x4_h(P.s_val + i0, sv, pol_stream);
+            } else {
+#pragma unroll
+                for (int k = 0; k < 4; k++)
+                    if (valid[k]) st_stream_u64_h(P.s_val + i0 + k, sv[k], pol_stream);
+            }
         }
     }
 }
