@@ -57,6 +57,9 @@ def test_sssp_fullsize_exact_by_properties(lj):
     v = v[v != 0]
     assert np.array_equal(best[v], d[v])
     assert st["converged"]
+    # north_star: fewer vertex updates than the vertex-centric ablation
+    sv = dg.run("sssp", source=0, mode="vertex")
+    assert st["vertex_updates"] <= sv["vertex_updates"], (st, sv)
 
 
 def test_pagerank_fullsize_residual(lj):
