@@ -388,22 +388,27 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round
     const unsigned long long eps = P.eps_fx;
     float carry = 0.f;
     const int64_t first = beg & ~(int64_t)3;
-    // software pipeline: the next window's indices are in flight while this one is walked
+    // software pipeline: the next window's indices and mirrors are in flight
+    // while this one is walked (only the master gathers stay exposed)
     uint4 code_nx = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
-    if (first + 4 * lane < end) code_nx = ld_stream_u4_h(P.e_idx + first + 4 * lane, pol_stream);
+    unsigned long long sv_nx[4] = {0ull, 0ull, 0ull, 0ull};
+    if (first + 4 * lane < end) {
+        code_nx = ld_stream_u4_h(P.e_idx + first + 4 * lane, pol_stream);
+        ld_stream_u64x4_h(P.s_val + first + 4 * lane, sv_nx, pol_stream);
+    }
     for (int64_t base = first; base < end; base += 128) {
         const int64_t i0 = base + 4 * lane;
         const uint4 code = code_nx;
-        if (i0 + 128 < end) code_nx = ld_stream_u4_h(P.e_idx + i0 + 128, pol_stream);
-        // masters (with their signal stamps) and mirrors are fetched together;
-        // a window none of whose vertices was signalled and that receives no
-        // carry is skipped after the fetch (PageRank keeps most windows active)
-        unsigned long long sv[4] = {0ull, 0ull, 0ull, 0ull};
-        float4 c4 = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (i0 < end) {
-            ld_stream_u64x4_h(P.s_val + i0, sv, pol_stream);
-            if (ADS) c4 = ld_stream_f4_h(P.e_coef + i0, pol_stream);
+        unsigned long long sv[4] = {sv_nx[0], sv_nx[1], sv_nx[2], sv_nx[3]};
+        if (i0 + 128 < end) {
+            code_nx = ld_stream_u4_h(P.e_idx + i0 + 128, pol_stream);
+            ld_stream_u64x4_h(P.s_val + i0 + 128, sv_nx, pol_stream);
         }
+        // masters (with their signal stamps) are gathered; a window none of
+        // whose vertices was signalled and that receives no carry is skipped
+        // (PageRank keeps most windows active)
+        float4 c4 = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (ADS && i0 < end) c4 = ld_stream_f4_h(P.e_coef + i0, pol_stream);
         uint32_t vtx[4];
         unsigned long long T[4];
         float cf[4];
@@ -422,7 +427,11 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round
                     cf[k] = px.coef[vtx[k]];
                     stamp = px.stamp[vtx[k]];
                 } else {
+#if defined(DG_EXP) && DG_EXP == 3   // experiment: no master gather
+                    T[k] = 1ull << 40; cf[k] = 0.05f; stamp = round;
+#else
                     ld_state_h(&P.vs_a[vtx[k]], T[k], cf[k], stamp, pol_keep);
+#endif
                 }
             }
             any_act |= stamp == round;
@@ -471,8 +480,15 @@ __device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round
             if (!hd[k]) acc.edges++;
             const unsigned long long p = fx_from(pin[k]);
             if (p) {
+#if defined(DG_EXP) && DG_EXP == 1   // experiment: scattered plain store instead of RED
+                if (vtx[k] < px.H) atomicAdd(&px.acc[vtx[k]], p);
+                else P.sigma[vtx[k]] = p;
+#elif defined(DG_EXP) && DG_EXP == 2  // experiment: no master update at all
+                if (vtx[k] < px.H) atomicAdd(&px.acc[vtx[k]], p);
+#else
                 if (vtx[k] < px.H) atomicAdd(&px.acc[vtx[k]], p);  // proxy: shared-memory atomic
                 else atomicAdd(&P.vs_a[vtx[k]].T, p);               // master: REDG (no return)
+#endif
                 acc.upd++;
             }
             if (!tl[k] && (pend[k] | p)) { sv[k] += pend[k] + p; dirty = true; }
