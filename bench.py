@@ -102,15 +102,19 @@ class ClockSampler:
 # ----------------------------------------------------------------- roofline
 def algorithmic_bytes(algo, st):
     """Useful bytes one launch of the propagation kernel moves (DESIGN.md
-    "Roofline"): path entries (4B index [+4B weight]) + vertex-state reads
-    and the master-state read-modify-writes it performs."""
-    E, U, C = st["entries_processed"], st["vertex_updates"], st["csr_edges"]
+    sec. 0(d)), from the launch's device counters: E = path entries walked,
+    U = master updates.
+      PageRank/Adsorption: per walked entry 4 B e_idx + 4 B path-edge
+        coefficient + 8 B mirror S_val read + 8 B master total T read (24 B);
+        per update 8 B RED on T + 8 B mirror write (16 B).
+      SSSP/BFS: per walked entry 4 B e_idx + 4 B weight + 4 B distance read;
+        per improvement 8 B atomicMin read-modify-write.
+      WCC/SCC: per walked entry 4 B e_idx + 4 B label; 8 B per improvement."""
+    E, U = st["entries_processed"], st["vertex_updates"]
     if algo in ("pagerank", "adsorption"):
-        # entry: 4B e_idx + 8B (g, delta) state read; fire: 8B r RMW + 16B row_ptr pair;
-        # CSR push: 4B col (+4B weight for adsorption) + 8B delta RMW
-        return E * 12 + U * 24 + C * (16 if algo == "adsorption" else 12)
-    if algo == "sssp":
-        return E * 12 + U * 8   # 4B e_idx + 4B weight + 4B dist read; 8B atomicMin RMW per improvement
+        return E * 24 + U * 16
+    if algo in ("sssp", "bfs"):
+        return E * (12 if algo == "sssp" else 8) + U * 8
     return E * 8 + U * 8
 
 

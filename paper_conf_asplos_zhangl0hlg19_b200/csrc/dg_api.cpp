@@ -147,6 +147,7 @@ int dg_upload(dg_graph* g) {
     int rc = dg::dev_upload_csr(g->dev, g->csr, g->layout, err);
     if (!rc) rc = dg::dev_upload_layout(g->dev, g->layout, err);
     if (rc) { dg::dev_free_layout(g->dev, true); return fail(rc, err); }
+    dg::dev_layout_changed(g->work);
     g->uploaded = true;
     g->ran = false;
     return DG_OK;

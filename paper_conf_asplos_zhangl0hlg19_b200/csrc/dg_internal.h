@@ -102,5 +102,6 @@ int dev_normalize(void* buf, int64_t n, std::string& err);
 int dev_get_states(DevWork* W, const DevLayout& D, const RunState& S, void* out, int64_t n, int out_is_device,
                    std::string& err);
 void dev_free_work(DevWork*& W);
+void dev_layout_changed(DevWork* W);  // device layout re-uploaded: drop arrays derived from it
 
 }  // namespace dg

@@ -65,22 +65,16 @@ struct Counters {
     int pad;
 };
 
-// Path-mode PageRank / Adsorption master: exact fixed-point total (2^-32
-// units, reading R-FX) and the PageRank path-edge coefficient d/outdeg.
-struct __align__(16) AccState {
-    unsigned long long T;
-    float coef;
-    int stamp;  // the round this vertex was last signalled for (activity of the path walk)
-};
-
 struct DevWork {
     uint2* vs_u = nullptr;                 // {value, stamp}: SSSP/BFS dist, WCC/SCC label
     float4* vs_f = nullptr;                // vertex-centric ablation: {r, g, delta, stamp}
-    AccState* vs_a = nullptr;              // path-mode PR / Adsorption masters
+    unsigned long long* vs_t = nullptr;    // path-mode PR / Adsorption masters: exact fixed-point totals T
     unsigned long long* sigma = nullptr;   // T at the vertex's last signal
     unsigned long long* s_val = nullptr;   // per-entry mirrors S_val (Fig. 4)
     unsigned long long* bnd_base = nullptr;
     float* e_coef = nullptr;               // Adsorption: coefficient of the path edge out of each entry
+    float* pr_coef = nullptr;              // PageRank: d/outdeg(v_i) of the path edge out of each entry
+    double pr_coef_d = -1.0;               // the damping pr_coef was computed for
     float* ads_base = nullptr;             // Adsorption: p_inj * I
     uint32_t* bits = nullptr;              // 2 x nw signal bitmaps
     int64_t nw = 0;
@@ -104,7 +98,7 @@ struct KParams {
     int64_t n_part, n, nw;
     uint2* vs_u;
     float4* vs_f;
-    AccState* vs_a;
+    unsigned long long* vs_t;
     unsigned long long* sigma;
     unsigned long long* s_val;
     const float* e_coef;
@@ -185,15 +179,6 @@ __device__ __forceinline__ void st_stream_u64x4_h(unsigned long long* p, const u
 }
 __device__ __forceinline__ void st_stream_u64_h(unsigned long long* p, unsigned long long v, unsigned long long pol) {
     asm volatile("st.global.L1::no_allocate.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(pol));
-}
-// 16-byte master-state gather kept in L2 (evict-last): {T, coef, stamp}
-__device__ __forceinline__ void ld_state_h(const void* p, unsigned long long& t, float& coef, int& stamp,
-                                           unsigned long long pol) {
-    unsigned long long a, b;
-    asm volatile("ld.global.L2::cache_hint.v2.u64 {%0,%1}, [%2], %3;" : "=l"(a), "=l"(b) : "l"(p), "l"(pol));
-    t = a;
-    coef = __uint_as_float((unsigned)(b & 0xffffffffull));
-    stamp = (int)(b >> 32);
 }
 __device__ __forceinline__ uint32_t u4get(const uint4& v, int k) {
     return k == 0 ? v.x : k == 1 ? v.y : k == 2 ? v.z : v.w;
@@ -356,12 +341,12 @@ __device__ void walk_minplus(const KParams& P, int64_t beg, int64_t end, const u
 //     a_i = c_i * (pend_i + p_i),   pend_i = T_i - S_val[i] if >= eps else 0,
 // where p_i = a_(i-1) is what its path predecessor pushed in this same walk
 // (used immediately, Observation 1) and c_i the path edge's coefficient
-// (d/outdeg for PageRank).  p_i is added to T(v_i) and S_val[i] += pend_i+p_i.
-// T and S_val are exact 64-bit fixed point (2^-32 units; DESIGN.md reading
-// R-FX): pend is an exact difference and conversions truncate, so no push is
-// inflated by rounding and every cycle contracts -- fp32 totals livelock once
-// eps is ~1 ulp of T.  A vertex whose total grew by >= eps since its last
-// signal is signalled (the per-vertex stop rule at delta < eps).
+// (d/outdeg for PageRank, streamed per entry).  p_i is added to T(v_i) and
+// S_val[i] += pend_i + p_i.  T and S_val are exact 64-bit fixed point (2^-32
+// units; reading R-FX): pend is an exact difference and conversions
+// truncate, so no push is inflated by rounding and every cycle contracts --
+// fp32 totals livelock once eps is ~1 ulp of T.  A window is walked when one
+// of its entries has pend >= eps or a path carries a push into it.
 constexpr float kFxScale = 4294967296.0f;          // 2^32
 constexpr float kFxInv = 2.3283064365386963e-10f;  // 2^-32
 __device__ __forceinline__ unsigned long long fx_from(float x) { return x > 0.f ? __float2ull_rz(x * kFxScale) : 0ull; }
@@ -372,152 +357,222 @@ __device__ __forceinline__ float fx_to(unsigned long long v) { return __ull2floa
 // each related SMX for each vertex with high in-degree, to accumulate the
 // pushed new states of its local mirrors ... sent to the master when the
 // partition assigned to this SMX has been handled".  Per CTA: the round-start
-// totals and stamps, the CTA's unflushed pushes, the path-edge coefficients.
+// totals and the CTA's unflushed pushes.
 struct Proxies {
     unsigned long long* T;
     unsigned long long* acc;
-    float* coef;
-    int* stamp;
     int64_t H;
 };
 
+// cp.async (sm_80+ LDGSTS): 16-byte global -> shared copies that hold no
+// registers while in flight; L2-only (.cg), with an L2 eviction policy.
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, unsigned long long pol) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "l"(pol)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
+
+// A warp's stream of 128-entry windows over the partitions it takes from the
+// round's ticket (priority order): base < 0 marks the end of the stream.
+struct Win {
+    int64_t base, beg, end;
+};
+__device__ __forceinline__ Win win_first_of(const KParams& P, unsigned* ticket) {
+    unsigned t = 0;
+    if ((threadIdx.x & 31) == 0) t = atomicAdd(ticket, 1u);
+    t = __shfl_sync(0xffffffffu, t, 0);
+    if (t >= (unsigned)P.n_part) return Win{-1, 0, 0};
+    const int64_t beg = P.part_off[t], end = P.part_off[t + 1];
+    return Win{beg & ~(int64_t)3, beg, end};
+}
+__device__ __forceinline__ Win win_next(const KParams& P, const Win& w, unsigned* ticket) {
+    if (w.base < 0) return w;
+    if (w.base + 128 < w.end) return Win{w.base + 128, w.beg, w.end};
+    return win_first_of(P, ticket);
+}
+
+// Walk all windows the warp obtains in this round.  Software pipeline over the
+// window stream: while window w is walked, the master totals of window w+1
+// are in flight into shared memory (cp.async, a 2-slot ring per warp), its
+// mirrors and coefficients into registers, and the indices of window w+2.
+// Reading a master one window early is a read slightly before the walk
+// reaches it -- the same asynchronous semantics as any concurrent push.
 template <bool ADS>
-__device__ void walk_accum(const KParams& P, int64_t beg, int64_t end, int round, Acc& acc,
-                           unsigned long long pol_stream, unsigned long long pol_keep, const Proxies& px) {
+__device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigned long long pol_stream,
+                           unsigned long long pol_keep, const Proxies& px, uint4* gbuf, int* s_done) {
     const int lane = threadIdx.x & 31;
     const unsigned long long eps = P.eps_fx;
-    float carry = 0.f;
-    const int64_t first = beg & ~(int64_t)3;
-    // software pipeline: the next window's indices and mirrors are in flight
-    // while this one is walked (only the master gathers stay exposed)
-    uint4 code_nx = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
-    unsigned long long sv_nx[4] = {0ull, 0ull, 0ull, 0ull};
-    if (first + 4 * lane < end) {
-        code_nx = ld_stream_u4_h(P.e_idx + first + 4 * lane, pol_stream);
-        ld_stream_u64x4_h(P.s_val + first + 4 * lane, sv_nx, pol_stream);
-    }
-    for (int64_t base = first; base < end; base += 128) {
-        const int64_t i0 = base + 4 * lane;
-        const uint4 code = code_nx;
-        unsigned long long sv[4] = {sv_nx[0], sv_nx[1], sv_nx[2], sv_nx[3]};
-        if (i0 + 128 < end) {
-            code_nx = ld_stream_u4_h(P.e_idx + i0 + 128, pol_stream);
-            ld_stream_u64x4_h(P.s_val + i0 + 128, sv_nx, pol_stream);
+    const uint4 kFill = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
+    auto load_code = [&](const Win& w) {
+        uint4 c = kFill;
+        if (w.base >= 0 && w.base + 4 * lane < w.end) c = ld_stream_u4_h(P.e_idx + w.base + 4 * lane, pol_stream);
+        return c;
+    };
+    auto load_sv = [&](const Win& w, unsigned long long (&sv)[4], float4& cf) {
+        if (w.base >= 0 && w.base + 4 * lane < w.end) {
+            ld_stream_u64x4_h(P.s_val + w.base + 4 * lane, sv, pol_stream);
+            cf = ld_stream_f4_h(P.e_coef + w.base + 4 * lane, pol_stream);
+        } else {
+            sv[0] = sv[1] = sv[2] = sv[3] = 0ull;
+            cf = make_float4(0.f, 0.f, 0.f, 0.f);
         }
-        // masters (with their signal stamps) are gathered; a window none of
-        // whose vertices was signalled and that receives no carry is skipped
-        // (PageRank keeps most windows active)
-        float4 c4 = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (ADS && i0 < end) c4 = ld_stream_f4_h(P.e_coef + i0, pol_stream);
+    };
+    // masters of a window into ring slot s: entry 4*lane+k -> gbuf[s*128 + k*32 + lane]
+    // (16-byte aligned pair {T[v & ~1], T[v | 1]}); proxies and invalid entries skip
+    auto gather = [&](const Win& w, const uint4& code, int s) {
+        if (w.base >= 0) {
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                const int64_t i = w.base + 4 * lane + k;
+                const uint32_t v = u4get(code, k) & kVMask;
+                if (i >= w.beg && i < w.end && v >= px.H)
+                    cp_async16(&gbuf[s * 128 + k * 32 + lane], P.vs_t + (v & ~1u), pol_keep);
+            }
+        }
+        cp_async_commit();
+    };
+
+    Win wc = win_first_of(P, ticket);
+    if (wc.base < 0) return;
+    Win wn = win_next(P, wc, ticket);
+    uint4 code_c = load_code(wc), code_n = load_code(wn);
+    unsigned long long sv_c[4], sv_n[4];
+    float4 cf_c, cf_n;
+    load_sv(wc, sv_c, cf_c);
+    gather(wc, code_c, 0);
+    int slot = 0;
+    float carry = 0.f;
+    while (wc.base >= 0) {
+        const Win wnn = win_next(P, wn, ticket);
+        const uint4 code_nn = load_code(wnn);
+        gather(wn, code_n, slot ^ 1);
+        load_sv(wn, sv_n, cf_n);
+        const bool part_start = wc.base == (wc.beg & ~(int64_t)3);
+        if (part_start) {
+            carry = 0.f;
+            if (px.H && DG_PROXY_REFRESH > 0) {
+                // every DG_PROXY_REFRESH partitions of this CTA, one warp sends the
+                // proxies' pushes to their masters and refreshes the snapshot, so
+                // hub totals propagate between CTAs within the round
+                int c = 0;
+                if (lane == 0) c = atomicAdd(s_done, 1) + 1;
+                c = __shfl_sync(0xffffffffu, c, 0);
+                if (c % DG_PROXY_REFRESH == 0) {
+                    for (int64_t i = lane; i < px.H; i += 32) {
+                        const unsigned long long a = atomicExch(&px.acc[i], 0ull);
+                        if (a) atomicAdd(&P.vs_t[i], a);
+                    }
+                    __syncwarp();
+                    for (int64_t i = lane; i < px.H; i += 32) px.T[i] = *(volatile unsigned long long*)&P.vs_t[i];
+                }
+            }
+        }
+        cp_async_wait1();  // this window's masters have landed (its own lane's copies)
+        const int64_t i0 = wc.base + 4 * lane;
         uint32_t vtx[4];
-        unsigned long long T[4];
-        float cf[4];
-        bool valid[4], any_act = false;
+        unsigned long long T[4], pend[4];
+        bool valid[4], hd[4], tl[4], any_act = false;
 #pragma unroll
         for (int k = 0; k < 4; k++) {
             const int64_t i = i0 + k;
-            valid[k] = i >= beg && i < end;
-            vtx[k] = u4get(code, k) & kVMask;
+            const uint32_t c = u4get(code_c, k);
+            valid[k] = i >= wc.beg && i < wc.end;
+            vtx[k] = c & kVMask;
+            hd[k] = !valid[k] || (c & kHead);
+            tl[k] = !valid[k] || (c & kTail);
             T[k] = 0ull;
-            cf[k] = 0.f;
-            int stamp = -1;
             if (valid[k]) {
                 if (vtx[k] < px.H) {
                     T[k] = px.T[vtx[k]] + *(volatile unsigned long long*)&px.acc[vtx[k]];
-                    cf[k] = px.coef[vtx[k]];
-                    stamp = px.stamp[vtx[k]];
                 } else {
-#if defined(DG_EXP) && DG_EXP == 3   // experiment: no master gather
-                    T[k] = 1ull << 40; cf[k] = 0.05f; stamp = round;
-#else
-                    ld_state_h(&P.vs_a[vtx[k]], T[k], cf[k], stamp, pol_keep);
-#endif
+                    const uint4 q = gbuf[slot * 128 + k * 32 + lane];
+                    T[k] = (vtx[k] & 1u) ? ((unsigned long long)q.w << 32 | q.z) : ((unsigned long long)q.y << 32 | q.x);
                 }
             }
-            any_act |= stamp == round;
-        }
-        if (!__any_sync(0xffffffffu, any_act) && carry == 0.f) continue;
-        acc.units++;
-        float al[4], be[4];
-        unsigned long long pend[4];
-        bool hd[4], tl[4];
-#pragma unroll
-        for (int k = 0; k < 4; k++) {
-            const uint32_t c = u4get(code, k);
-            hd[k] = !valid[k] || (c & kHead);
-            tl[k] = !valid[k] || (c & kTail);
-            const unsigned long long pd = T[k] > sv[k] ? T[k] - sv[k] : 0ull;
+            const unsigned long long pd = T[k] > sv_c[k] ? T[k] - sv_c[k] : 0ull;
             pend[k] = (!tl[k] && pd >= eps) ? pd : 0ull;
-            const float coef = ADS ? f4get(c4, k) : cf[k];
-            al[k] = tl[k] ? 0.f : coef * fx_to(pend[k]);
-            be[k] = (tl[k] || hd[k]) ? 0.f : coef;
+            any_act |= pend[k] != 0ull;
         }
-        float Al = 0.f, Be = 1.f;
+        if (__any_sync(0xffffffffu, any_act) || carry != 0.f) {
+            acc.units++;
+            float al[4], be[4];
 #pragma unroll
-        for (int k = 0; k < 4; k++) { Al = al[k] + be[k] * Al; Be = be[k] * Be; }
-#pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {
-            float Ap = __shfl_up_sync(0xffffffffu, Al, off);
-            float Bp = __shfl_up_sync(0xffffffffu, Be, off);
-            if (lane >= off) { Al = Al + Be * Ap; Be = Be * Bp; }
-        }
-        float Ae = __shfl_up_sync(0xffffffffu, Al, 1);
-        float Bx = __shfl_up_sync(0xffffffffu, Be, 1);
-        if (lane == 0) { Ae = 0.f; Bx = 1.f; }
-        float prev = Ae + Bx * carry;
-        float pin[4];
-#pragma unroll
-        for (int k = 0; k < 4; k++) {
-            pin[k] = hd[k] ? 0.f : prev;
-            prev = al[k] + be[k] * prev;
-        }
-        carry = __shfl_sync(0xffffffffu, prev, 31);
-        bool dirty = false;
-#pragma unroll
-        for (int k = 0; k < 4; k++) {
-            if (!valid[k]) continue;
-            acc.entries++;
-            if (!hd[k]) acc.edges++;
-            const unsigned long long p = fx_from(pin[k]);
-            if (p) {
-#if defined(DG_EXP) && DG_EXP == 1   // experiment: scattered plain store instead of RED
-                if (vtx[k] < px.H) atomicAdd(&px.acc[vtx[k]], p);
-                else P.sigma[vtx[k]] = p;
-#elif defined(DG_EXP) && DG_EXP == 2  // experiment: no master update at all
-                if (vtx[k] < px.H) atomicAdd(&px.acc[vtx[k]], p);
-#else
-                if (vtx[k] < px.H) atomicAdd(&px.acc[vtx[k]], p);  // proxy: shared-memory atomic
-                else atomicAdd(&P.vs_a[vtx[k]].T, p);               // master: REDG (no return)
-#endif
-                acc.upd++;
+            for (int k = 0; k < 4; k++) {
+                const float coef = f4get(cf_c, k);
+                al[k] = tl[k] ? 0.f : coef * fx_to(pend[k]);
+                be[k] = (tl[k] || hd[k]) ? 0.f : coef;
             }
-            if (!tl[k] && (pend[k] | p)) { sv[k] += pend[k] + p; dirty = true; }
-        }
-        // lanes whose four entries all lie in this partition write one 256-bit
-        // store; lanes at the partition's ends write only their own entries
-        // (the neighbouring partition's mirrors belong to another warp)
-        if (dirty) {
-            if (i0 >= beg && i0 + 3 < end) {
-                st_stream_u64x4_h(P.s_val + i0, sv, pol_stream);
-            } else {
+            float Al = 0.f, Be = 1.f;
 #pragma unroll
-                for (int k = 0; k < 4; k++)
-                    if (valid[k]) st_stream_u64_h(P.s_val + i0 + k, sv[k], pol_stream);
+            for (int k = 0; k < 4; k++) { Al = al[k] + be[k] * Al; Be = be[k] * Be; }
+#pragma unroll
+            for (int off = 1; off < 32; off <<= 1) {  // warp inclusive scan of affine maps
+                float Ap = __shfl_up_sync(0xffffffffu, Al, off);
+                float Bp = __shfl_up_sync(0xffffffffu, Be, off);
+                if (lane >= off) { Al = Al + Be * Ap; Be = Be * Bp; }
             }
+            float Ae = __shfl_up_sync(0xffffffffu, Al, 1);
+            float Bx = __shfl_up_sync(0xffffffffu, Be, 1);
+            if (lane == 0) { Ae = 0.f; Bx = 1.f; }
+            float prev = Ae + Bx * carry;
+            float pin[4];
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                pin[k] = hd[k] ? 0.f : prev;
+                prev = al[k] + be[k] * prev;
+            }
+            carry = __shfl_sync(0xffffffffu, prev, 31);
+            bool dirty = false;
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                if (!valid[k]) continue;
+                acc.entries++;
+                if (!hd[k]) acc.edges++;
+                const unsigned long long p = fx_from(pin[k]);
+                if (p) {
+                    if (vtx[k] < px.H) atomicAdd(&px.acc[vtx[k]], p);  // proxy: shared-memory atomic
+                    else atomicAdd(&P.vs_t[vtx[k]], p);                 // master: REDG (no return)
+                    acc.upd++;
+                }
+                if (!tl[k] && (pend[k] | p)) { sv_c[k] += pend[k] + p; dirty = true; }
+            }
+            // lanes whose four entries all lie in this partition write one 256-bit
+            // store; lanes at the partition's ends write only their own entries
+            // (the neighbouring partition's mirrors belong to another warp)
+            if (dirty) {
+                if (i0 >= wc.beg && i0 + 3 < wc.end) {
+                    st_stream_u64x4_h(P.s_val + i0, sv_c, pol_stream);
+                } else {
+#pragma unroll
+                    for (int k = 0; k < 4; k++)
+                        if (valid[k]) st_stream_u64_h(P.s_val + i0 + k, sv_c[k], pol_stream);
+                }
+            }
+        } else {
+            carry = 0.f;
         }
+        // rotate the pipeline
+        wc = wn; wn = wnn;
+        code_c = code_n; code_n = code_nn;
+#pragma unroll
+        for (int k = 0; k < 4; k++) sv_c[k] = sv_n[k];
+        cf_c = cf_n;
+        slot ^= 1;
     }
+    cp_async_wait0();
 }
 
 // End-of-round vertex sweep of the accumulative algorithms: a vertex whose
-// total grew by >= eps since its last signal is signalled for the next round
-// (the per-vertex stop rule at delta < eps): its stamp is set to that round,
-// which the next walk reads together with the total.
-__device__ void accum_sweep(const KParams& P, int next_round, unsigned& cnt) {
+// total grew by >= eps since its last signal counts as signalled for the next
+// round (the per-vertex stop rule at delta < eps; the device active counter).
+__device__ void accum_sweep(const KParams& P, unsigned& cnt) {
     for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < P.n; v += (int64_t)gridDim.x * blockDim.x) {
-        const unsigned long long T = P.vs_a[v].T;
+        const unsigned long long T = __ldcg(&P.vs_t[v]);
         if (T - P.sigma[v] >= P.eps_fx) {
             P.sigma[v] = T;
-            P.vs_a[v].stamp = next_round;
             cnt++;
         }
     }
@@ -615,22 +670,25 @@ __device__ void walk_scc_bwd(const KParams& P, int64_t beg, int64_t end, const u
 }
 
 // ------------------------------------------------------------------ persistent round driver
+// Dynamic shared memory of the accumulative kernels: per-CTA proxies (16 B per
+// hub) then the per-warp 2 x 128-entry master ring (kWarps x 4 KB).
+constexpr size_t kGbufBytes = (size_t)kWarps * 2 * 128 * sizeof(uint4);
+
 template <int ALGO>
 __global__ void __launch_bounds__(kBlock, DG_PATH_MINB) path_kernel(KParams P) {
     cg::grid_group grid = cg::this_grid();
     const int lane = threadIdx.x & 31;
     constexpr bool kAccum = ALGO == DG_PAGERANK || ALGO == DG_ADSORPTION;
     const unsigned long long pol_stream = policy_evict_first(), pol_keep = policy_evict_last();
-    extern __shared__ unsigned long long dyn_smem[];
+    extern __shared__ __align__(16) unsigned char dyn_smem[];
     __shared__ int s_done;
-    Proxies px{nullptr, nullptr, nullptr, nullptr, 0};
-    if (kAccum && P.n_proxy > 0) {
+    Proxies px{nullptr, nullptr, 0};
+    uint4* gbuf = nullptr;
+    if (kAccum) {
+        gbuf = reinterpret_cast<uint4*>(dyn_smem) + (size_t)(threadIdx.x >> 5) * 256;
         px.H = P.n_proxy;
-        px.T = dyn_smem;
-        px.acc = dyn_smem + px.H;
-        px.coef = reinterpret_cast<float*>(dyn_smem + 2 * px.H);
-        px.stamp = reinterpret_cast<int*>(px.coef + px.H);
-        for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) px.coef[i] = P.vs_a[i].coef;
+        px.T = reinterpret_cast<unsigned long long*>(dyn_smem + kGbufBytes);
+        px.acc = px.T + px.H;
     }
     Acc acc;
     int r = 0;
@@ -638,55 +696,38 @@ __global__ void __launch_bounds__(kBlock, DG_PATH_MINB) path_kernel(KParams P) {
         const int round = P.ctr->round + r;  // ctr->round only changes after the loop
         const int cur = round & 1, nxt = cur ^ 1;
         if (*((volatile unsigned*)&P.ctr->active[cur]) == 0) break;
-        if (kAccum && px.H) {  // round-start snapshot of the proxied masters
-            for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) {
-                px.T[i] = P.vs_a[i].T;
-                px.stamp[i] = P.vs_a[i].stamp;
-                px.acc[i] = 0ull;
-            }
-            if (threadIdx.x == 0) s_done = 0;
-            __syncthreads();
-        }
         const uint32_t* bcur = P.bits + (int64_t)cur * P.nw;
         uint32_t* bnxt = P.bits + (int64_t)nxt * P.nw;
-        while (true) {
-            unsigned t = 0;
-            if (lane == 0) t = atomicAdd(&P.ctr->ticket[cur], 1u);
-            t = __shfl_sync(0xffffffffu, t, 0);
-            if (t >= (unsigned)P.n_part) break;
-            if (kAccum && px.H && DG_PROXY_REFRESH > 0) {
-                // every DG_PROXY_REFRESH partitions of this CTA, one warp sends the
-                // proxies' pushes to their masters and refreshes the snapshot, so
-                // hub totals propagate between CTAs within the round
-                int c = 0;
-                if (lane == 0) c = atomicAdd(&s_done, 1) + 1;
-                c = __shfl_sync(0xffffffffu, c, 0);
-                if (c % DG_PROXY_REFRESH == 0) {
-                    for (int64_t i = lane; i < px.H; i += 32) {
-                        const unsigned long long a = atomicExch(&px.acc[i], 0ull);
-                        if (a) atomicAdd(&P.vs_a[i].T, a);
-                    }
-                    __syncwarp();
-                    for (int64_t i = lane; i < px.H; i += 32) px.T[i] = *(volatile unsigned long long*)&P.vs_a[i].T;
-                }
-            }
-            const int64_t beg = P.part_off[t], end = P.part_off[t + 1];
-            if (ALGO == DG_SSSP) walk_minplus<0>(P, beg, end, bcur, bnxt, acc);
-            else if (ALGO == DG_BFS) walk_minplus<1>(P, beg, end, bcur, bnxt, acc);
-            else if (ALGO == DG_WCC) walk_minplus<2>(P, beg, end, bcur, bnxt, acc);
-            else if (ALGO == 100) walk_minplus<3>(P, beg, end, bcur, bnxt, acc);
-            else if (ALGO == 101) walk_scc_bwd(P, beg, end, bcur, bnxt, acc);
-            else if (ALGO == DG_PAGERANK) walk_accum<false>(P, beg, end, round, acc, pol_stream, pol_keep, px);
-            else if (ALGO == DG_ADSORPTION) walk_accum<true>(P, beg, end, round, acc, pol_stream, pol_keep, px);
-        }
         if (kAccum) {
+            if (px.H) {  // round-start snapshot of the proxied masters
+                for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) {
+                    px.T[i] = __ldcg(&P.vs_t[i]);
+                    px.acc[i] = 0ull;
+                }
+                if (threadIdx.x == 0) s_done = 0;
+                __syncthreads();
+            }
+            walk_accum<ALGO == DG_ADSORPTION>(P, &P.ctr->ticket[cur], acc, pol_stream, pol_keep, px, gbuf, &s_done);
             if (px.H) {  // send the proxies' accumulated pushes to their masters
                 __syncthreads();
                 for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x)
-                    if (px.acc[i]) atomicAdd(&P.vs_a[i].T, px.acc[i]);
+                    if (px.acc[i]) atomicAdd(&P.vs_t[i], px.acc[i]);
             }
             grid.sync();  // all pushes of the round landed
-            accum_sweep(P, round + 1, acc.sig);
+            accum_sweep(P, acc.sig);
+        } else {
+            while (true) {
+                unsigned t = 0;
+                if (lane == 0) t = atomicAdd(&P.ctr->ticket[cur], 1u);
+                t = __shfl_sync(0xffffffffu, t, 0);
+                if (t >= (unsigned)P.n_part) break;
+                const int64_t beg = P.part_off[t], end = P.part_off[t + 1];
+                if (ALGO == DG_SSSP) walk_minplus<0>(P, beg, end, bcur, bnxt, acc);
+                else if (ALGO == DG_BFS) walk_minplus<1>(P, beg, end, bcur, bnxt, acc);
+                else if (ALGO == DG_WCC) walk_minplus<2>(P, beg, end, bcur, bnxt, acc);
+                else if (ALGO == 100) walk_minplus<3>(P, beg, end, bcur, bnxt, acc);
+                else if (ALGO == 101) walk_scc_bwd(P, beg, end, bcur, bnxt, acc);
+            }
         }
         // publish this round's newly signalled vertices (the device active counter)
         unsigned s = acc.sig;
@@ -694,10 +735,12 @@ __global__ void __launch_bounds__(kBlock, DG_PATH_MINB) path_kernel(KParams P) {
         if (lane == 0 && s) atomicAdd(&P.ctr->active[nxt], s);
         acc.sig = 0;
         grid.sync();
-        // retire this round's bitmap for reuse two rounds later
-        uint32_t* bc = P.bits + (int64_t)cur * P.nw;
-        for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.nw; i += (int64_t)gridDim.x * blockDim.x)
-            bc[i] = 0u;
+        if (!kAccum) {  // retire this round's bitmap for reuse two rounds later
+            uint32_t* bc = P.bits + (int64_t)cur * P.nw;
+            for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.nw;
+                 i += (int64_t)gridDim.x * blockDim.x)
+                bc[i] = 0u;
+        }
         if (blockIdx.x == 0 && threadIdx.x == 0) { P.ctr->active[cur] = 0; P.ctr->ticket[cur] = 0; }
         grid.sync();
     }
@@ -842,14 +885,21 @@ __global__ void init_pr_kernel(float4* vs, const int32_t* outdeg, int64_t n, flo
     }
 }
 // path mode: T = 1-d (PageRank) or p_inj*I (Adsorption, base != null), sigma = T
-__global__ void init_acc_kernel(AccState* vs, unsigned long long* sigma, const int32_t* outdeg, const float* base,
-                                int64_t n, float d) {
+__global__ void init_acc_kernel(unsigned long long* vs, unsigned long long* sigma, const float* base, int64_t n,
+                                float d) {
     GRID_STRIDE(v, n) {
         const float t0 = base ? base[v] : 1.f - d;
         const unsigned long long T = (unsigned long long)((double)t0 * 4294967296.0);
-        const float c = (!base && outdeg[v] > 0) ? d / (float)outdeg[v] : 0.f;
-        vs[v] = AccState{T, c, 0};  // stamp 0: active in round 0
+        vs[v] = T;  // S_val = 0: every entry has pend = T >= eps in round 0
         sigma[v] = T;
+    }
+}
+// PageRank: coefficient of the path edge out of entry i = d / outdeg(v_i)
+__global__ void pr_coef_kernel(float* e_coef, const uint32_t* e_idx, const int32_t* outdeg, float d, int64_t M) {
+    GRID_STRIDE(i, M) {
+        const uint32_t c = e_idx[i];
+        const int32_t od = outdeg[c & kVMask];
+        e_coef[i] = (!(c & kTail) && od > 0) ? d / (float)od : 0.f;
     }
 }
 __global__ void fill_iota_kernel(int32_t* a, int64_t n) {
@@ -883,19 +933,19 @@ __global__ void wsum_kernel(float* wsum, const int64_t* row_ptr, const int32_t* 
         wsum[v] = (float)s;
     }
 }
-__device__ __forceinline__ double final_value(const float4* vf, const AccState* va, int64_t v) {
-    if (va) return (double)va[v].T * (1.0 / 4294967296.0);
+__device__ __forceinline__ double final_value(const float4* vf, const unsigned long long* va, int64_t v) {
+    if (va) return (double)va[v] * (1.0 / 4294967296.0);
     float4 x = vf[v];
     return (double)x.x + (double)x.z;  // ablation: r + pending delta
 }
-__global__ void sum_T_kernel(const float4* vf, const AccState* va, int64_t n, double* out) {
+__global__ void sum_T_kernel(const float4* vf, const unsigned long long* va, int64_t n, double* out) {
     double s = 0;
     GRID_STRIDE(v, n) s += final_value(vf, va, v);
     for (int off = 16; off; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
     if ((threadIdx.x & 31) == 0) atomicAdd(out, s);
 }
 // outputs are indexed by ORIGINAL vertex id: out[v] = state[new_id[v]]
-__global__ void out_pr_kernel(const float4* vf, const AccState* va, const int32_t* new_id, int64_t n,
+__global__ void out_pr_kernel(const float4* vf, const unsigned long long* va, const int32_t* new_id, int64_t n,
                               const double* sum, float* out, int normalize) {
     const double inv = normalize ? 1.0 / *sum : 1.0;
     GRID_STRIDE(v, n) out[v] = (float)(final_value(vf, va, new_id[v]) * inv);
@@ -969,14 +1019,14 @@ __global__ void unpack_min_kernel(uint2* vs, const int32_t* bnd, int64_t nb, con
 }
 // SUM algorithms exchange the growth of each boundary total since the last
 // exchange; after the all-reduce every replica holds the same total.
-__global__ void init_base_kernel(const AccState* vs, const int32_t* bnd, int64_t nb, unsigned long long* base) {
-    GRID_STRIDE(k, nb) base[k] = vs[bnd[k]].T;
+__global__ void init_base_kernel(const unsigned long long* vs, const int32_t* bnd, int64_t nb, unsigned long long* base) {
+    GRID_STRIDE(k, nb) base[k] = vs[bnd[k]];
 }
-__global__ void pack_sum_kernel(const AccState* vs, const int32_t* bnd, int64_t nb, const unsigned long long* base,
-                                unsigned long long* buf) {
-    GRID_STRIDE(k, nb) buf[k] = vs[bnd[k]].T - base[k];
+__global__ void pack_sum_kernel(const unsigned long long* vs, const int32_t* bnd, int64_t nb,
+                                const unsigned long long* base, unsigned long long* buf) {
+    GRID_STRIDE(k, nb) buf[k] = vs[bnd[k]] - base[k];
 }
-__global__ void unpack_sum_kernel(AccState* vs, unsigned long long* sigma, const int32_t* bnd, int64_t nb,
+__global__ void unpack_sum_kernel(unsigned long long* vs, unsigned long long* sigma, const int32_t* bnd, int64_t nb,
                                   unsigned long long* base, const unsigned long long* buf, unsigned long long eps,
                                   int round, Counters* ctr, int slot) {
     unsigned cnt = 0;
@@ -984,11 +1034,10 @@ __global__ void unpack_sum_kernel(AccState* vs, unsigned long long* sigma, const
         const int v = bnd[k];
         const unsigned long long t = base[k] + buf[k];
         base[k] = t;
-        vs[v].T = t;
-        if (t - sigma[v] >= eps) {
+        vs[v] = t;
+        if (t - sigma[v] >= eps) {  // the replica's growth counts as a signal of the next local round
             sigma[v] = t;
-            cnt += vs[v].stamp != round;
-            vs[v].stamp = round;
+            cnt++;
         }
     }
     for (int off = 16; off; off >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, off);
@@ -1046,7 +1095,7 @@ KParams make_params(const DevLayout& D, DevWork* W) {
     P.e_idx = D.e_idx; P.e_w = D.e_w; P.part_off = D.part_off;
     P.row_ptr = D.row_ptr; P.col = D.col; P.w = D.w;
     P.n_part = D.n_part; P.n = D.n; P.nw = W->nw;
-    P.vs_u = W->vs_u; P.vs_f = W->vs_f; P.vs_a = W->vs_a; P.sigma = W->sigma; P.s_val = W->s_val;
+    P.vs_u = W->vs_u; P.vs_f = W->vs_f; P.vs_t = W->vs_t; P.sigma = W->sigma; P.s_val = W->s_val;
     P.e_coef = W->e_coef; P.bits = W->bits;
     P.vlist0 = W->vlist[0]; P.vlist1 = W->vlist[1];
     P.ctr = W->ctr;
@@ -1063,7 +1112,7 @@ int ensure_work(DevWork*& W, const DevLayout& D, std::string& err) {
     W->nw = (D.n + 31) / 32 + 1;
     if ((rc = dalloc(&W->vs_u, D.n + 1, bytes, err))) return rc;
     if ((rc = dalloc(&W->vs_f, D.n + 1, bytes, err))) return rc;
-    if ((rc = dalloc(&W->vs_a, D.n + 1, bytes, err))) return rc;
+    if ((rc = dalloc(&W->vs_t, D.n + 2, bytes, err))) return rc;
     if ((rc = dalloc(&W->sigma, D.n + 1, bytes, err))) return rc;
     if ((rc = dalloc(&W->s_val, D.M + kPad, bytes, err))) return rc;
     if ((rc = dalloc(&W->bnd_base, D.n_bnd + 1, bytes, err))) return rc;
@@ -1127,8 +1176,9 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
         default: err = "bad algo"; return DG_EINVAL;
     }
     const bool accum = algo_k == DG_PAGERANK || algo_k == DG_ADSORPTION;
-    const size_t smem = accum ? (size_t)D.n_proxy * 24 : 0;
+    const size_t smem = accum ? kGbufBytes + (size_t)D.n_proxy * 16 : 0;
     if (!accum) P.n_proxy = 0;
+    if (accum) P.e_coef = algo_k == DG_ADSORPTION ? W->e_coef : W->pr_coef;
     return coop_launch(W, fn, P, S, err, smem);
 }
 
@@ -1172,8 +1222,17 @@ int init_states(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
         if (algo == DG_WCC) {
             init_u_kernel<<<g, 256>>>(W->vs_u, D.orig, D.n, algo, 0);
         } else {
-            init_acc_kernel<<<g, 256>>>(W->vs_a, W->sigma, D.outdeg, algo == DG_ADSORPTION ? W->ads_base : nullptr,
-                                        D.n, (float)S.param);
+            init_acc_kernel<<<g, 256>>>(W->vs_t, W->sigma, algo == DG_ADSORPTION ? W->ads_base : nullptr, D.n,
+                                        (float)S.param);
+            if (algo == DG_PAGERANK && W->pr_coef_d != S.param) {  // per-entry d/outdeg, cached per damping
+                int64_t bytes = 0;
+                int rc;
+                if (!W->pr_coef && (rc = dalloc(&W->pr_coef, D.M + kPad, bytes, err))) return rc;
+                CK(cudaMemsetAsync(W->pr_coef, 0, sizeof(float) * (D.M + kPad)));
+                pr_coef_kernel<<<grid_1d(D.M), 256>>>(W->pr_coef, D.e_idx, D.outdeg, (float)S.param, D.M);
+                W->pr_coef_d = S.param;
+                S.stats.kernel_launches++;
+            }
             CK(cudaMemsetAsync(W->s_val, 0, sizeof(unsigned long long) * (D.M + kPad)));
         }
         bits_all_kernel<<<grid_1d(W->nw), 256>>>(W->bits, W->nw, D.n);
@@ -1340,8 +1399,8 @@ void dev_free_layout(DevLayout& D, bool csr_too) {
 
 void dev_free_work(DevWork*& W) {
     if (!W) return;
-    dfree(W->vs_u); dfree(W->vs_f); dfree(W->vs_a); dfree(W->sigma); dfree(W->s_val); dfree(W->bnd_base);
-    dfree(W->e_coef); dfree(W->ads_base); dfree(W->bits); dfree(W->vlist[0]); dfree(W->vlist[1]);
+    dfree(W->vs_u); dfree(W->vs_f); dfree(W->vs_t); dfree(W->sigma); dfree(W->s_val); dfree(W->bnd_base);
+    dfree(W->e_coef); dfree(W->pr_coef); dfree(W->ads_base); dfree(W->bits); dfree(W->vlist[0]); dfree(W->vlist[1]);
     dfree(W->ctr); dfree(W->dsum); dfree(W->scc_label); dfree(W->scc_mark); dfree(W->remaining);
     if (W->ev0) cudaEventDestroy(W->ev0);
     if (W->ev1) cudaEventDestroy(W->ev1);
@@ -1349,6 +1408,10 @@ void dev_free_work(DevWork*& W) {
     if (W->kev1) cudaEventDestroy(W->kev1);
     delete W;
     W = nullptr;
+}
+
+void dev_layout_changed(DevWork* W) {
+    if (W) W->pr_coef_d = -1.0;
 }
 
 int dev_set_vertex_params(DevWork*& W, const DevLayout& D, const double* p_inj, const double* p_cont,
@@ -1421,7 +1484,7 @@ int dev_run_begin(DevWork*& W, const DevLayout& D, RunState& S, std::string& err
     if (S.algo == DG_ADSORPTION && !W->have_params) { err = "Adsorption needs dg_set_vertex_params first"; return DG_EINVAL; }
     if ((rc = init_states(W, D, S, err))) return rc;
     if ((S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION) && D.n_bnd)
-        init_base_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_a, D.bnd, D.n_bnd, W->bnd_base);
+        init_base_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_t, D.bnd, D.n_bnd, W->bnd_base);
     CK(cudaGetLastError());
     CK(cudaEventRecord(W->ev0));
     return DG_OK;
@@ -1439,7 +1502,7 @@ int dev_rounds(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, 
 int dev_boundary_pack(DevWork* W, const DevLayout& D, RunState& S, void* buf, std::string& err) {
     if (!D.n_bnd) return DG_OK;
     if (S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION)
-        pack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_a, D.bnd, D.n_bnd, W->bnd_base, (unsigned long long*)buf);
+        pack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_t, D.bnd, D.n_bnd, W->bnd_base, (unsigned long long*)buf);
     else
         pack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, D.bnd, D.n_bnd, (uint32_t*)buf);
     S.stats.kernel_launches++;
@@ -1457,7 +1520,7 @@ int dev_boundary_unpack(DevWork* W, const DevLayout& D, RunState& S, const void*
     if (D.n_bnd) {
         uint32_t* b = W->bits + (int64_t)slot * W->nw;
         if (S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION)
-            unpack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_a, W->sigma, D.bnd, D.n_bnd, W->bnd_base,
+            unpack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_t, W->sigma, D.bnd, D.n_bnd, W->bnd_base,
                                                          (const unsigned long long*)buf,
                                                          (unsigned long long)(S.eps * 4294967296.0), c.round, W->ctr,
                                                          slot);
@@ -1507,7 +1570,7 @@ int dev_get_states(DevWork* W, const DevLayout& D, const RunState& S, void* out,
     }
     const int g = grid_1d(n);
     if (S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION) {
-        const AccState* va = S.mode == DG_MODE_PATH ? W->vs_a : nullptr;
+        const unsigned long long* va = S.mode == DG_MODE_PATH ? W->vs_t : nullptr;
         CK(cudaMemset(W->dsum, 0, sizeof(double)));
         if (S.algo == DG_PAGERANK) sum_T_kernel<<<g, 256>>>(W->vs_f, va, n, W->dsum);
         out_pr_kernel<<<g, 256>>>(W->vs_f, va, D.new_id, n, W->dsum, (float*)dst,

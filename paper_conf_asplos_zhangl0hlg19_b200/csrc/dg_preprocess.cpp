@@ -15,6 +15,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <numeric>
+#include <parallel/algorithm>
 #include <stdexcept>
 
 #include "dg_internal.h"
@@ -419,9 +420,10 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     const int64_t G = (int64_t)gpart_first.size() - 1;
     const int world = std::max(1, p.world), rank = p.rank;
 
-    // ---- internal numbering: the H highest-degree vertices (ties by id) get ids
-    // [0, H) so the path kernel can keep them as shared-memory proxies; a
-    // non-hub vertex with id < H takes a freed hub id (both ascending)
+    // ---- internal numbering: vertices in degree-descending order (ties by id).
+    // The H highest-degree vertices get ids [0, H) so the path kernel keeps them
+    // as shared-memory proxies; the rest are packed by degree so the vertex
+    // states that most path entries touch share cache sectors and stay in L2.
     const int64_t H = std::min<int64_t>(std::max<int32_t>(0, p.n_proxy), n);
     L.n_proxy = H;
     L.new_id.resize(n);
@@ -429,22 +431,14 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     {
         std::vector<int32_t> byd(n);
         std::iota(byd.begin(), byd.end(), 0);
-        std::partial_sort(byd.begin(), byd.begin() + H, byd.end(), [&](int32_t a, int32_t b) {
+        __gnu_parallel::sort(byd.begin(), byd.end(), [&](int32_t a, int32_t b) {
             return deg[a] != deg[b] ? deg[a] > deg[b] : a < b;
         });
-        std::vector<uint8_t> is_hub(n, 0);
-        std::vector<int32_t> freed, displaced;
-        for (int64_t i = 0; i < H; i++) is_hub[byd[i]] = 1;
-        for (int64_t v = 0; v < n; v++) L.new_id[v] = (int32_t)v;
-        for (int64_t i = 0; i < H; i++) {
+        #pragma omp parallel for schedule(static)
+        for (int64_t i = 0; i < n; i++) {
             L.new_id[byd[i]] = (int32_t)i;
-            if (byd[i] >= H) freed.push_back(byd[i]);
+            L.orig[i] = byd[i];
         }
-        for (int64_t v = 0; v < H; v++)
-            if (!is_hub[v]) displaced.push_back((int32_t)v);
-        std::sort(freed.begin(), freed.end());
-        for (size_t j = 0; j < displaced.size(); j++) L.new_id[displaced[j]] = freed[j];
-        for (int64_t v = 0; v < n; v++) L.orig[L.new_id[v]] = (int32_t)v;
     }
     // CSR in internal ids
     L.prow_ptr.assign(n + 1, 0);
