@@ -26,6 +26,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <string>
@@ -196,140 +197,216 @@ __device__ __forceinline__ bool signal_vertex(uint32_t* b, uint32_t v) {
     return !(atomicOr(&b[v >> 5], m) & m);
 }
 
+// per-thread statistics (32-bit: a thread's share stays far below 2^32;
+// widened to 64 bits for the warp reduction)
 struct Acc {
-    unsigned long long upd = 0, edges = 0, units = 0, entries = 0, pushes = 0;
-    unsigned int sig = 0;
+    unsigned upd = 0, edges = 0, units = 0, entries = 0, pushes = 0;
+    unsigned sig = 0;
 };
 
 // ------------------------------------------------------------------ path walks
+// cp.async (sm_80+ LDGSTS): 16-byte global -> shared copies that hold no
+// registers while in flight; L2-only (.cg), with an L2 eviction policy.
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, unsigned long long pol) {
+    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "l"(pol)
+                 : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
+
+// A warp's stream of 128-entry windows over the partitions it takes from the
+// round's ticket (priority order): base < 0 marks the end of the stream.
+// Entry offsets are 32-bit (dev_upload_layout checks M + padding < 2^32) so
+// the three cursors of the software pipeline stay in 9 registers.
+constexpr uint32_t kNoWin = 0xFFFFFFFFu;
+struct Win {
+    uint32_t base, beg, end;
+};
+__device__ __forceinline__ Win win_first_of(const KParams& P, unsigned* ticket) {
+    unsigned t = 0;
+    if ((threadIdx.x & 31) == 0) t = atomicAdd(ticket, 1u);
+    t = __shfl_sync(0xffffffffu, t, 0);
+    if (t >= (unsigned)P.n_part) return Win{kNoWin, 0, 0};
+    const uint32_t beg = (uint32_t)P.part_off[t], end = (uint32_t)P.part_off[t + 1];
+    return Win{beg & ~3u, beg, end};
+}
+__device__ __forceinline__ Win win_next(const KParams& P, const Win& w, unsigned* ticket) {
+    if (w.base == kNoWin) return w;
+    if (w.base + 128 < w.end) return Win{w.base + 128, w.beg, w.end};
+    return win_first_of(P, ticket);
+}
+
 // Min-plus walk.  MODE 0 SSSP (weights), 1 BFS (unit weights), 2 WCC (weight 0,
 // also backward along every path edge), 3 SCC forward colouring (weight 0,
 // assigned vertices -- scc_label >= 0 -- break their paths).
+// The warp walks its stream of windows with a one-window lookahead: while
+// window w is walked, the signal bits of window w+1 are tested and, if one is
+// set, its master states are already in flight (read slightly early -- the
+// asynchronous semantics of any concurrent update; atomicMin stays the
+// authority), as are the indices of window w+2.
 template <int MODE>
-__device__ void walk_minplus(const KParams& P, int64_t beg, int64_t end, const uint32_t* bcur, uint32_t* bnxt,
-                             Acc& acc) {
+__device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t* bcur, uint32_t* bnxt, Acc& acc) {
     const int lane = threadIdx.x & 31;
-    uint32_t carry = INF;
-    bool carry_live = false;
-    const int64_t first = beg & ~(int64_t)3;
-    uint4 code_nx = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
-    if (first + 4 * lane < end) code_nx = ld_stream_u4(P.e_idx + first + 4 * lane);
-    for (int64_t base = first; base < end; base += 128) {
-        const int64_t i0 = base + 4 * lane;
-        const uint4 code = code_nx;  // prefetched in the previous iteration
-        if (i0 + 128 < end) code_nx = ld_stream_u4(P.e_idx + i0 + 128);
-        uint32_t vtx[4];
-        bool valid[4], act[4], any_act = false;
+    const uint4 kFill = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
+    auto load_code = [&](const Win& w) {
+        uint4 c = kFill;
+        if (w.base != kNoWin && w.base + 4 * lane < w.end) c = ld_stream_u4(P.e_idx + w.base + 4 * lane);
+        return c;
+    };
+    // signal bits of a window; if any is set, issue its master gathers
+    auto probe = [&](const Win& w, const uint4& code, bool (&act)[4], uint32_t (&a)[4]) {
+        bool any = false;
 #pragma unroll
         for (int k = 0; k < 4; k++) {
-            const int64_t i = i0 + k;
-            valid[k] = i >= beg && i < end;
-            vtx[k] = u4get(code, k) & kVMask;
-            act[k] = valid[k] && test_bit(bcur, vtx[k]);
-            any_act |= act[k];
+            const uint32_t i = w.base + 4 * lane + k;
+            const bool valid = w.base != kNoWin && i >= w.beg && i < w.end;
+            act[k] = valid && test_bit(bcur, u4get(code, k) & kVMask);
+            any |= act[k];
         }
+        any = __any_sync(0xffffffffu, any);
+        if (any) {
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                const uint32_t i = w.base + 4 * lane + k;
+                a[k] = (i >= w.beg && i < w.end) ? P.vs_u[u4get(code, k) & kVMask].x : INF;
+            }
+        }
+        return any;
+    };
+
+    Win wc = win_first_of(P, ticket);
+    if (wc.base == kNoWin) return;
+    Win wn = win_next(P, wc, ticket);
+    uint4 code_c = load_code(wc), code_n = load_code(wn);
+    bool act_c[4], act_n[4];
+    uint32_t a_c[4] = {INF, INF, INF, INF}, a_n[4] = {INF, INF, INF, INF};
+    bool any_c = probe(wc, code_c, act_c, a_c);
+    uint32_t carry = INF;
+    bool carry_live = false;
+    while (wc.base != kNoWin) {
+        const Win wnn = win_next(P, wn, ticket);
+        const uint4 code_nn = load_code(wnn);
+        const bool any_n = probe(wn, code_n, act_n, a_n);
+        if (wc.base == (wc.beg & ~3u)) { carry = INF; carry_live = false; }  // partition start
+        const uint32_t i0 = wc.base + 4 * lane;
         // WCC looks one entry ahead: the path edge into the next window is walked backwards too
-        uint32_t nx_code = kHead, nx_lab = INF;
+        uint32_t nx_lab = INF;
         bool nx_act = false;
         if (MODE == 2 && lane == 31) {
-            const int64_t inx = base + 128;
-            if (inx < end) {
-                nx_code = P.e_idx[inx];
+            const uint32_t inx = wc.base + 128;
+            if (inx < wc.end) {
+                const uint32_t nx_code = P.e_idx[inx];
                 if (!(nx_code & kHead)) {
                     nx_act = test_bit(bcur, nx_code & kVMask);
                     nx_lab = P.vs_u[nx_code & kVMask].x;
                 }
             }
-            any_act |= nx_act;
         }
-        if (!__any_sync(0xffffffffu, any_act) && !carry_live) {
-            carry = INF;
-            continue;
-        }
-        acc.units++;
-        int4 wv = make_int4(0, 0, 0, 0);
-        if (MODE == 0 && i0 < end) wv = ld_stream_i4(P.e_w + i0);
-        uint32_t a[4], wgt[4];
-        bool hd[4], tl[4], live[4];
+        const bool nx_any = MODE == 2 ? __any_sync(0xffffffffu, nx_act) : false;
+        const bool walk = any_c || carry_live || nx_any;
+        if (walk) {
+            acc.units++;
+            if (!any_c) {  // walked only for a live carry (or WCC look-ahead): gather now
 #pragma unroll
-        for (int k = 0; k < 4; k++) {
-            const uint32_t c = u4get(code, k);
-            live[k] = valid[k] && (MODE != 3 || P.scc_label[vtx[k]] < 0);
-            hd[k] = !live[k] || (c & kHead);
-            tl[k] = !live[k] || (c & kTail);
-            wgt[k] = MODE == 0 ? (uint32_t)i4get(wv, k) : (MODE == 1 ? 1u : 0u);
-            a[k] = live[k] ? P.vs_u[vtx[k]].x : INF;
-        }
-        // lane aggregate of f_k(x) = hd ? a : min(a, x + w)
-        bool H = false;
-        uint32_t A = INF, W = 0;
-#pragma unroll
-        for (int k = 0; k < 4; k++) {
-            if (hd[k]) { H = true; A = a[k]; W = 0; }
-            else { A = min(a[k], sat_add(A, wgt[k])); W = sat_add(W, wgt[k]); }
-        }
-#pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {  // warp inclusive scan, prefix composed before self
-            bool Hp = __shfl_up_sync(0xffffffffu, H, off);
-            uint32_t Ap = __shfl_up_sync(0xffffffffu, A, off);
-            uint32_t Wp = __shfl_up_sync(0xffffffffu, W, off);
-            if (lane >= off && !H) { A = min(A, sat_add(Ap, W)); W = sat_add(Wp, W); H = Hp; }
-        }
-        bool He = __shfl_up_sync(0xffffffffu, H, 1);
-        uint32_t Ae = __shfl_up_sync(0xffffffffu, A, 1);
-        uint32_t We = __shfl_up_sync(0xffffffffu, W, 1);
-        if (lane == 0) { He = false; Ae = INF; We = 0; }
-        uint32_t cur = He ? Ae : min(Ae, sat_add(carry, We));
-        uint32_t val[4];
-#pragma unroll
-        for (int k = 0; k < 4; k++) {
-            cur = hd[k] ? a[k] : min(a[k], sat_add(cur, wgt[k]));
-            val[k] = cur;
-        }
-        if (MODE == 2) {
-            // backward (suffix) min: x_i = min(a_i, x_(i+1)) until a tail
-            bool T = false;
-            uint32_t B = INF;
-#pragma unroll
-            for (int k = 3; k >= 0; k--) {
-                if (tl[k]) { T = true; B = a[k]; } else B = min(a[k], B);
-            }
-#pragma unroll
-            for (int off = 1; off < 32; off <<= 1) {
-                bool Tn = __shfl_down_sync(0xffffffffu, T, off);
-                uint32_t Bn = __shfl_down_sync(0xffffffffu, B, off);
-                if (lane + off < 32 && !T) { B = min(B, Bn); T = Tn; }
-            }
-            uint32_t bc = __shfl_down_sync(0xffffffffu, B, 1);
-            bool Te = __shfl_down_sync(0xffffffffu, T, 1);
-            if (lane == 31) { bc = nx_lab; Te = false; }
-            (void)Te;
-#pragma unroll
-            for (int k = 3; k >= 0; k--) {
-                bc = tl[k] ? a[k] : min(a[k], bc);
-                val[k] = min(val[k], bc);
-            }
-        }
-        bool changed[4];
-#pragma unroll
-        for (int k = 0; k < 4; k++) {
-            changed[k] = false;
-            if (!live[k]) continue;
-            acc.entries++;
-            if (!(u4get(code, k) & kHead)) acc.edges++;
-            if (val[k] < a[k]) {
-                const uint32_t old = atomicMin(&P.vs_u[vtx[k]].x, val[k]);
-                if (val[k] < old) {
-                    acc.upd++;
-                    changed[k] = true;
-                    acc.sig += signal_vertex(bnxt, vtx[k]);
+                for (int k = 0; k < 4; k++) {
+                    const uint32_t i = i0 + k;
+                    a_c[k] = (i >= wc.beg && i < wc.end) ? P.vs_u[u4get(code_c, k) & kVMask].x : INF;
                 }
             }
+            int4 wv = make_int4(0, 0, 0, 0);
+            if (MODE == 0 && i0 < wc.end) wv = ld_stream_i4(P.e_w + i0);
+            uint32_t vtx[4], a[4], wgt[4];
+            bool hd[4], tl[4], live[4];
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                const uint32_t i = i0 + k;
+                const uint32_t c = u4get(code_c, k);
+                vtx[k] = c & kVMask;
+                live[k] = i >= wc.beg && i < wc.end && (MODE != 3 || P.scc_label[vtx[k]] < 0);
+                hd[k] = !live[k] || (c & kHead);
+                tl[k] = !live[k] || (c & kTail);
+                wgt[k] = MODE == 0 ? (uint32_t)i4get(wv, k) : (MODE == 1 ? 1u : 0u);
+                a[k] = live[k] ? a_c[k] : INF;
+            }
+            // lane aggregate of f_k(x) = hd ? a : min(a, x + w)
+            bool H = false;
+            uint32_t A = INF, W = 0;
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                if (hd[k]) { H = true; A = a[k]; W = 0; }
+                else { A = min(a[k], sat_add(A, wgt[k])); W = sat_add(W, wgt[k]); }
+            }
+#pragma unroll
+            for (int off = 1; off < 32; off <<= 1) {  // warp inclusive scan, prefix composed before self
+                bool Hp = __shfl_up_sync(0xffffffffu, H, off);
+                uint32_t Ap = __shfl_up_sync(0xffffffffu, A, off);
+                uint32_t Wp = __shfl_up_sync(0xffffffffu, W, off);
+                if (lane >= off && !H) { A = min(A, sat_add(Ap, W)); W = sat_add(Wp, W); H = Hp; }
+            }
+            bool He = __shfl_up_sync(0xffffffffu, H, 1);
+            uint32_t Ae = __shfl_up_sync(0xffffffffu, A, 1);
+            uint32_t We = __shfl_up_sync(0xffffffffu, W, 1);
+            if (lane == 0) { He = false; Ae = INF; We = 0; }
+            uint32_t cur = He ? Ae : min(Ae, sat_add(carry, We));
+            uint32_t val[4];
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                cur = hd[k] ? a[k] : min(a[k], sat_add(cur, wgt[k]));
+                val[k] = cur;
+            }
+            if (MODE == 2) {
+                // backward (suffix) min: x_i = min(a_i, x_(i+1)) until a tail
+                bool T = false;
+                uint32_t B = INF;
+#pragma unroll
+                for (int k = 3; k >= 0; k--) {
+                    if (tl[k]) { T = true; B = a[k]; } else B = min(a[k], B);
+                }
+#pragma unroll
+                for (int off = 1; off < 32; off <<= 1) {
+                    bool Tn = __shfl_down_sync(0xffffffffu, T, off);
+                    uint32_t Bn = __shfl_down_sync(0xffffffffu, B, off);
+                    if (lane + off < 32 && !T) { B = min(B, Bn); T = Tn; }
+                }
+                uint32_t bc = __shfl_down_sync(0xffffffffu, B, 1);
+                if (lane == 31) bc = nx_lab;
+#pragma unroll
+                for (int k = 3; k >= 0; k--) {
+                    bc = tl[k] ? a[k] : min(a[k], bc);
+                    val[k] = min(val[k], bc);
+                }
+            }
+            bool changed3 = false;
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                if (!live[k]) continue;
+                acc.entries++;
+                if (!(u4get(code_c, k) & kHead)) acc.edges++;
+                if (val[k] < a[k]) {
+                    const uint32_t old = atomicMin(&P.vs_u[vtx[k]].x, val[k]);
+                    if (val[k] < old) {
+                        acc.upd++;
+                        if (k == 3) changed3 = true;
+                        acc.sig += signal_vertex(bnxt, vtx[k]);
+                    }
+                }
+            }
+            // the carry into the next window is live if the path continues and its
+            // last vertex changed now or was signalled (its out-edge must be relaxed)
+            carry = __shfl_sync(0xffffffffu, cur, 31);
+            carry_live = __shfl_sync(0xffffffffu, !tl[3] && (changed3 || act_c[3]), 31);
+        } else {
+            carry = INF;
+            carry_live = false;
         }
-        // the carry into the next window is live if the path continues and its
-        // last vertex changed now or was signalled (its out-edge must be relaxed)
-        carry = __shfl_sync(0xffffffffu, cur, 31);
-        carry_live = __shfl_sync(0xffffffffu, !tl[3] && (changed[3] || act[3]), 31);
+        // rotate the pipeline
+        wc = wn; wn = wnn;
+        code_c = code_n; code_n = code_nn;
+        any_c = any_n;
+#pragma unroll
+        for (int k = 0; k < 4; k++) { act_c[k] = act_n[k]; a_c[k] = a_n[k]; }
     }
 }
 
@@ -364,36 +441,6 @@ struct Proxies {
     int64_t H;
 };
 
-// cp.async (sm_80+ LDGSTS): 16-byte global -> shared copies that hold no
-// registers while in flight; L2-only (.cg), with an L2 eviction policy.
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, unsigned long long pol) {
-    const unsigned s = (unsigned)__cvta_generic_to_shared(smem);
-    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "l"(pol)
-                 : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
-
-// A warp's stream of 128-entry windows over the partitions it takes from the
-// round's ticket (priority order): base < 0 marks the end of the stream.
-struct Win {
-    int64_t base, beg, end;
-};
-__device__ __forceinline__ Win win_first_of(const KParams& P, unsigned* ticket) {
-    unsigned t = 0;
-    if ((threadIdx.x & 31) == 0) t = atomicAdd(ticket, 1u);
-    t = __shfl_sync(0xffffffffu, t, 0);
-    if (t >= (unsigned)P.n_part) return Win{-1, 0, 0};
-    const int64_t beg = P.part_off[t], end = P.part_off[t + 1];
-    return Win{beg & ~(int64_t)3, beg, end};
-}
-__device__ __forceinline__ Win win_next(const KParams& P, const Win& w, unsigned* ticket) {
-    if (w.base < 0) return w;
-    if (w.base + 128 < w.end) return Win{w.base + 128, w.beg, w.end};
-    return win_first_of(P, ticket);
-}
-
 // Walk all windows the warp obtains in this round.  Software pipeline over the
 // window stream: while window w is walked, the master totals of window w+1
 // are in flight into shared memory (cp.async, a 2-slot ring per warp), its
@@ -408,11 +455,11 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
     const uint4 kFill = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
     auto load_code = [&](const Win& w) {
         uint4 c = kFill;
-        if (w.base >= 0 && w.base + 4 * lane < w.end) c = ld_stream_u4_h(P.e_idx + w.base + 4 * lane, pol_stream);
+        if (w.base != kNoWin && w.base + 4 * lane < w.end) c = ld_stream_u4_h(P.e_idx + w.base + 4 * lane, pol_stream);
         return c;
     };
     auto load_sv = [&](const Win& w, unsigned long long (&sv)[4], float4& cf) {
-        if (w.base >= 0 && w.base + 4 * lane < w.end) {
+        if (w.base != kNoWin && w.base + 4 * lane < w.end) {
             ld_stream_u64x4_h(P.s_val + w.base + 4 * lane, sv, pol_stream);
             cf = ld_stream_f4_h(P.e_coef + w.base + 4 * lane, pol_stream);
         } else {
@@ -423,10 +470,10 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
     // masters of a window into ring slot s: entry 4*lane+k -> gbuf[s*128 + k*32 + lane]
     // (16-byte aligned pair {T[v & ~1], T[v | 1]}); proxies and invalid entries skip
     auto gather = [&](const Win& w, const uint4& code, int s) {
-        if (w.base >= 0) {
+        if (w.base != kNoWin) {
 #pragma unroll
             for (int k = 0; k < 4; k++) {
-                const int64_t i = w.base + 4 * lane + k;
+                const uint32_t i = w.base + 4 * lane + k;
                 const uint32_t v = u4get(code, k) & kVMask;
                 if (i >= w.beg && i < w.end && v >= px.H)
                     cp_async16(&gbuf[s * 128 + k * 32 + lane], P.vs_t + (v & ~1u), pol_keep);
@@ -436,7 +483,7 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
     };
 
     Win wc = win_first_of(P, ticket);
-    if (wc.base < 0) return;
+    if (wc.base == kNoWin) return;
     Win wn = win_next(P, wc, ticket);
     uint4 code_c = load_code(wc), code_n = load_code(wn);
     unsigned long long sv_c[4], sv_n[4];
@@ -445,12 +492,12 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
     gather(wc, code_c, 0);
     int slot = 0;
     float carry = 0.f;
-    while (wc.base >= 0) {
+    while (wc.base != kNoWin) {
         const Win wnn = win_next(P, wn, ticket);
         const uint4 code_nn = load_code(wnn);
         gather(wn, code_n, slot ^ 1);
         load_sv(wn, sv_n, cf_n);
-        const bool part_start = wc.base == (wc.beg & ~(int64_t)3);
+        const bool part_start = wc.base == (wc.beg & ~3u);
         if (part_start) {
             carry = 0.f;
             if (px.H && DG_PROXY_REFRESH > 0) {
@@ -471,13 +518,13 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
             }
         }
         cp_async_wait1();  // this window's masters have landed (its own lane's copies)
-        const int64_t i0 = wc.base + 4 * lane;
+        const uint32_t i0 = wc.base + 4 * lane;
         uint32_t vtx[4];
         unsigned long long T[4], pend[4];
         bool valid[4], hd[4], tl[4], any_act = false;
 #pragma unroll
         for (int k = 0; k < 4; k++) {
-            const int64_t i = i0 + k;
+            const uint32_t i = i0 + k;
             const uint32_t c = u4get(code_c, k);
             valid[k] = i >= wc.beg && i < wc.end;
             vtx[k] = c & kVMask;
@@ -505,26 +552,31 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
                 al[k] = tl[k] ? 0.f : coef * fx_to(pend[k]);
                 be[k] = (tl[k] || hd[k]) ? 0.f : coef;
             }
-            float Al = 0.f, Be = 1.f;
+            // in-order walk = inclusive warp scan of the entries' affine maps
+            // p_(i+1) = al_i + be_i * p_i (heads reset, tails push nothing)
+            auto walk_scan = [&](float (&pin)[4]) {
+                float Al = 0.f, Be = 1.f;
 #pragma unroll
-            for (int k = 0; k < 4; k++) { Al = al[k] + be[k] * Al; Be = be[k] * Be; }
+                for (int k = 0; k < 4; k++) { Al = al[k] + be[k] * Al; Be = be[k] * Be; }
 #pragma unroll
-            for (int off = 1; off < 32; off <<= 1) {  // warp inclusive scan of affine maps
-                float Ap = __shfl_up_sync(0xffffffffu, Al, off);
-                float Bp = __shfl_up_sync(0xffffffffu, Be, off);
-                if (lane >= off) { Al = Al + Be * Ap; Be = Be * Bp; }
-            }
-            float Ae = __shfl_up_sync(0xffffffffu, Al, 1);
-            float Bx = __shfl_up_sync(0xffffffffu, Be, 1);
-            if (lane == 0) { Ae = 0.f; Bx = 1.f; }
-            float prev = Ae + Bx * carry;
+                for (int off = 1; off < 32; off <<= 1) {
+                    float Ap = __shfl_up_sync(0xffffffffu, Al, off);
+                    float Bp = __shfl_up_sync(0xffffffffu, Be, off);
+                    if (lane >= off) { Al = Al + Be * Ap; Be = Be * Bp; }
+                }
+                float Ae = __shfl_up_sync(0xffffffffu, Al, 1);
+                float Bx = __shfl_up_sync(0xffffffffu, Be, 1);
+                if (lane == 0) { Ae = 0.f; Bx = 1.f; }
+                float prev = Ae + Bx * carry;
+#pragma unroll
+                for (int k = 0; k < 4; k++) {
+                    pin[k] = hd[k] ? 0.f : prev;
+                    prev = al[k] + be[k] * prev;
+                }
+                return __shfl_sync(0xffffffffu, prev, 31);
+            };
             float pin[4];
-#pragma unroll
-            for (int k = 0; k < 4; k++) {
-                pin[k] = hd[k] ? 0.f : prev;
-                prev = al[k] + be[k] * prev;
-            }
-            carry = __shfl_sync(0xffffffffu, prev, 31);
+            carry = walk_scan(pin);
             bool dirty = false;
 #pragma unroll
             for (int k = 0; k < 4; k++) {
@@ -674,8 +726,8 @@ __device__ void walk_scc_bwd(const KParams& P, int64_t beg, int64_t end, const u
 // hub) then the per-warp 2 x 128-entry master ring (kWarps x 4 KB).
 constexpr size_t kGbufBytes = (size_t)kWarps * 2 * 128 * sizeof(uint4);
 
-template <int ALGO>
-__global__ void __launch_bounds__(kBlock, DG_PATH_MINB) path_kernel(KParams P) {
+template <int ALGO, int MINB = DG_PATH_MINB>
+__global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
     cg::grid_group grid = cg::this_grid();
     const int lane = threadIdx.x & 31;
     constexpr bool kAccum = ALGO == DG_PAGERANK || ALGO == DG_ADSORPTION;
@@ -716,17 +768,19 @@ __global__ void __launch_bounds__(kBlock, DG_PATH_MINB) path_kernel(KParams P) {
             grid.sync();  // all pushes of the round landed
             accum_sweep(P, acc.sig);
         } else {
-            while (true) {
-                unsigned t = 0;
-                if (lane == 0) t = atomicAdd(&P.ctr->ticket[cur], 1u);
-                t = __shfl_sync(0xffffffffu, t, 0);
-                if (t >= (unsigned)P.n_part) break;
-                const int64_t beg = P.part_off[t], end = P.part_off[t + 1];
-                if (ALGO == DG_SSSP) walk_minplus<0>(P, beg, end, bcur, bnxt, acc);
-                else if (ALGO == DG_BFS) walk_minplus<1>(P, beg, end, bcur, bnxt, acc);
-                else if (ALGO == DG_WCC) walk_minplus<2>(P, beg, end, bcur, bnxt, acc);
-                else if (ALGO == 100) walk_minplus<3>(P, beg, end, bcur, bnxt, acc);
-                else if (ALGO == 101) walk_scc_bwd(P, beg, end, bcur, bnxt, acc);
+            unsigned* ticket = &P.ctr->ticket[cur];
+            if (ALGO == DG_SSSP) walk_minplus<0>(P, ticket, bcur, bnxt, acc);
+            else if (ALGO == DG_BFS) walk_minplus<1>(P, ticket, bcur, bnxt, acc);
+            else if (ALGO == DG_WCC) walk_minplus<2>(P, ticket, bcur, bnxt, acc);
+            else if (ALGO == 100) walk_minplus<3>(P, ticket, bcur, bnxt, acc);
+            else if (ALGO == 101) {
+                while (true) {
+                    unsigned t = 0;
+                    if (lane == 0) t = atomicAdd(ticket, 1u);
+                    t = __shfl_sync(0xffffffffu, t, 0);
+                    if (t >= (unsigned)P.n_part) break;
+                    walk_scc_bwd(P, P.part_off[t], P.part_off[t + 1], bcur, bnxt, acc);
+                }
             }
         }
         // publish this round's newly signalled vertices (the device active counter)
@@ -744,16 +798,17 @@ __global__ void __launch_bounds__(kBlock, DG_PATH_MINB) path_kernel(KParams P) {
         if (blockIdx.x == 0 && threadIdx.x == 0) { P.ctr->active[cur] = 0; P.ctr->ticket[cur] = 0; }
         grid.sync();
     }
+    unsigned long long su = acc.upd, se = acc.edges, sn = acc.entries;
     for (int off = 16; off; off >>= 1) {
-        acc.upd += __shfl_xor_sync(0xffffffffu, acc.upd, off);
-        acc.edges += __shfl_xor_sync(0xffffffffu, acc.edges, off);
-        acc.entries += __shfl_xor_sync(0xffffffffu, acc.entries, off);
+        su += __shfl_xor_sync(0xffffffffu, su, off);
+        se += __shfl_xor_sync(0xffffffffu, se, off);
+        sn += __shfl_xor_sync(0xffffffffu, sn, off);
     }
     if (lane == 0) {  // units are warp-uniform (counted identically by every lane)
-        atomicAdd(&P.ctr->updates, acc.upd);
-        atomicAdd(&P.ctr->edges, acc.edges);
-        atomicAdd(&P.ctr->units, acc.units);
-        atomicAdd(&P.ctr->entries, acc.entries);
+        atomicAdd(&P.ctr->updates, su);
+        atomicAdd(&P.ctr->edges, se);
+        atomicAdd(&P.ctr->units, (unsigned long long)acc.units);
+        atomicAdd(&P.ctr->entries, sn);
     }
     grid.sync();
     if (blockIdx.x == 0 && threadIdx.x == 0) P.ctr->round += r;
@@ -850,16 +905,17 @@ __global__ void __launch_bounds__(kBlock) vertex_kernel(KParams P) {
         if (blockIdx.x == 0 && threadIdx.x == 0) { P.ctr->active[cur] = 0; P.ctr->ticket[cur] = 0; }
         grid.sync();
     }
+    unsigned long long su = acc.upd, sn = acc.units, sp = acc.pushes;
     for (int off = 16; off; off >>= 1) {
-        acc.upd += __shfl_xor_sync(0xffffffffu, acc.upd, off);
-        acc.units += __shfl_xor_sync(0xffffffffu, acc.units, off);
-        acc.pushes += __shfl_xor_sync(0xffffffffu, acc.pushes, off);
+        su += __shfl_xor_sync(0xffffffffu, su, off);
+        sn += __shfl_xor_sync(0xffffffffu, sn, off);
+        sp += __shfl_xor_sync(0xffffffffu, sp, off);
     }
     if (lane == 0) {
-        atomicAdd(&P.ctr->updates, acc.upd);
-        atomicAdd(&P.ctr->edges, acc.pushes);
-        atomicAdd(&P.ctr->units, acc.units);
-        atomicAdd(&P.ctr->pushes, acc.pushes);
+        atomicAdd(&P.ctr->updates, su);
+        atomicAdd(&P.ctr->edges, sp);
+        atomicAdd(&P.ctr->units, sn);
+        atomicAdd(&P.ctr->pushes, sp);
     }
     grid.sync();
     if (blockIdx.x == 0 && threadIdx.x == 0) P.ctr->round += r;
@@ -1158,6 +1214,13 @@ int coop_launch(DevWork* W, void* fn, KParams& P, RunState& S, std::string& err,
     return DG_OK;
 }
 
+// resident CTAs per SM the accumulative kernels are compiled for (2: up to 128
+// registers, no spills; 3: 80 registers); DG_ACC_MINB selects (developer knob)
+int acc_minb() {
+    const char* e = std::getenv("DG_ACC_MINB");
+    return e ? std::atoi(e) : 2;
+}
+
 // Launch the persistent path kernel for at most `rounds` rounds.
 int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState& S, std::string& err) {
     KParams P = make_params(D, W);
@@ -1169,8 +1232,10 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
         case DG_SSSP: fn = (void*)path_kernel<DG_SSSP>; break;
         case DG_BFS: fn = (void*)path_kernel<DG_BFS>; break;
         case DG_WCC: fn = (void*)path_kernel<DG_WCC>; break;
-        case DG_PAGERANK: fn = (void*)path_kernel<DG_PAGERANK>; break;
-        case DG_ADSORPTION: fn = (void*)path_kernel<DG_ADSORPTION>; break;
+        case DG_PAGERANK: fn = acc_minb() == 2 ? (void*)path_kernel<DG_PAGERANK, 2> : (void*)path_kernel<DG_PAGERANK>; break;
+        case DG_ADSORPTION:
+            fn = acc_minb() == 2 ? (void*)path_kernel<DG_ADSORPTION, 2> : (void*)path_kernel<DG_ADSORPTION>;
+            break;
         case 100: fn = (void*)path_kernel<100>; break;
         case 101: fn = (void*)path_kernel<101>; break;
         default: err = "bad algo"; return DG_EINVAL;
@@ -1366,6 +1431,10 @@ int dev_upload_layout(DevLayout& D, const HostLayout& L, std::string& err) {
     g_h2d_counter = &D.h2d_bytes;
     g_pin_list = &D.pinned;
     D.M = (int64_t)L.e_idx.size();
+    if (D.M + kPad + 256 >= (int64_t)0xFFFFFFFFll) {  // the kernels use 32-bit entry offsets
+        err = "layout has >= 2^32 path entries on one rank; use more ranks";
+        return DG_EINVAL;
+    }
     D.n_part = (int64_t)L.part_off.size() - 1;
     D.n_bnd = (int64_t)L.boundary.size();
     if ((rc = dalloc_once(&D.e_idx, D.M + kPad, D.bytes, err))) return rc;
