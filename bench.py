@@ -302,10 +302,14 @@ def main():
                 dist.barrier()
             t = time.perf_counter()
             dg.upload()
+            t_up = time.perf_counter()
             if world == 1:
                 dg.run(args.algo, mode=args.mode, **run_kw)
+                t_run = time.perf_counter()
                 out = dg.get_states()
                 d2h = int(out.nbytes)
+                log(f"[bench] e2e step: upload {1e3 * (t_up - t):.1f} ms, run {1e3 * (t_run - t_up):.1f} ms, "
+                    f"get_states {1e3 * (time.perf_counter() - t_run):.1f} ms")
             else:
                 parallel.run_distributed(dg, args.algo, device=torch.device("cuda", local), **run_kw)
                 out = parallel.gather_states(dg, args.algo, g.n, device=torch.device("cuda", local)).cpu()

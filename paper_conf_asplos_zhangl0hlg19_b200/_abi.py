@@ -11,7 +11,7 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libdigraph.so")
+LIB_PATH = os.environ.get("DG_LIB_PATH") or os.path.join(_HERE, "libdigraph.so")  # env: developer builds only
 
 DG_SSSP, DG_BFS, DG_PAGERANK, DG_WCC, DG_SCC, DG_ADSORPTION = range(6)
 DG_MODE_PATH, DG_MODE_VERTEX = 0, 1

@@ -54,7 +54,7 @@ constexpr int kPad = 256;  // zero entries after every per-entry array
 #define DG_PATH_MINB 3  // resident CTAs per SM requested for the path kernel
 #endif
 #ifndef DG_PROXY_REFRESH
-#define DG_PROXY_REFRESH 8  // partitions a CTA walks between mid-round proxy flushes (0 = round end only)
+#define DG_PROXY_REFRESH 8  // default: partitions a CTA walks between mid-round proxy flushes (0 = round end only)
 #endif
 
 // device counters of a run
@@ -114,6 +114,7 @@ struct KParams {
     float eps;
     unsigned long long eps_fx;
     int max_rounds;
+    int px_refresh;  // partitions a CTA walks between mid-round proxy flushes (0: round end only)
 };
 
 // ------------------------------------------------------------------ helpers
@@ -500,14 +501,14 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
         const bool part_start = wc.base == (wc.beg & ~3u);
         if (part_start) {
             carry = 0.f;
-            if (px.H && DG_PROXY_REFRESH > 0) {
-                // every DG_PROXY_REFRESH partitions of this CTA, one warp sends the
+            if (px.H && P.px_refresh > 0) {
+                // every px_refresh partitions of this CTA, one warp sends the
                 // proxies' pushes to their masters and refreshes the snapshot, so
                 // hub totals propagate between CTAs within the round
                 int c = 0;
                 if (lane == 0) c = atomicAdd(s_done, 1) + 1;
                 c = __shfl_sync(0xffffffffu, c, 0);
-                if (c % DG_PROXY_REFRESH == 0) {
+                if (c % P.px_refresh == 0) {
                     for (int64_t i = lane; i < px.H; i += 32) {
                         const unsigned long long a = atomicExch(&px.acc[i], 0ull);
                         if (a) atomicAdd(&P.vs_t[i], a);
@@ -1244,6 +1245,10 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
     const size_t smem = accum ? kGbufBytes + (size_t)D.n_proxy * 16 : 0;
     if (!accum) P.n_proxy = 0;
     if (accum) P.e_coef = algo_k == DG_ADSORPTION ? W->e_coef : W->pr_coef;
+    {
+        const char* e = std::getenv("DG_PROXY_REFRESH");  // developer knob
+        P.px_refresh = e ? std::atoi(e) : DG_PROXY_REFRESH;
+    }
     return coop_launch(W, fn, P, S, err, smem);
 }
 

@@ -14,6 +14,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <functional>
 #include <numeric>
 #include <parallel/algorithm>
 #include <stdexcept>
@@ -80,18 +81,110 @@ struct Decomposer {
     }
 };
 
-// Iterative Tarjan over a CSR graph (node ids < 2^31); comp[v] = SCC id in
-// completion order (reverse topological order of the condensation).
-int32_t tarjan(int32_t N, const std::vector<int64_t>& ptr, const std::vector<int32_t>& adj,
-               std::vector<int32_t>& comp) {
-    std::vector<int32_t> index(N, -1), low(N, 0);
-    std::vector<int64_t> it(N, 0);
-    std::vector<uint8_t> onst(N, 0);
-    std::vector<int32_t> st, work;
-    st.reserve(1024); work.reserve(1024);
-    comp.assign(N, -1);
-    int32_t counter = 0, ncomp = 0;
-    for (int32_t r = 0; r < N; r++) {
+// ---------------------------------------------------------------------------
+// Dependency graph G' and its DAG sketch (readings
+// R-DEP, R-LAYER), as a bipartite path/vertex graph with implicit adjacency:
+//   path node i    -> vertex node P+x  for every x entered by an edge of i
+//   vertex node P+x -> path node j     for every x left by an edge of j
+// Reachability between path nodes equals reachability in G'.  SCCs are found
+// by the parallel trim / forward-backward / Tarjan scheme: (1) nodes with no
+// remaining predecessor or successor are peeled off in rounds (singleton SCCs;
+// the peel rounds are a topological order of them); (2) the SCC of a pivot is
+// the intersection of its forward and backward reachable sets (the giant SCC
+// of power-law graphs); (3) the rest is split into the pivot's upstream,
+// unrelated and downstream classes, each closed under SCCs, and condensed by
+// sequential Tarjan.  Components are numbered in a topological order and the
+// layers are longest-path depths over it.  SCC sets and layers are unique, so
+// the result equals a plain Tarjan + topological DP (tests/test_host_preprocess.py).
+// ---------------------------------------------------------------------------
+struct DepGraph {
+    int64_t P, n, N;
+    const std::vector<int64_t>& moff;
+    const std::vector<int32_t>& mv;
+    std::vector<int64_t> lptr, eptr;   // vertex x: paths leaving x / entering x
+    std::vector<int32_t> ladj, eadj;
+
+    // Every out-edge (in-edge) of x lies on exactly one path, so x is left
+    // (entered) by exactly outdeg(x) (indeg(x)) path edges: the list sizes are
+    // the graph's degrees.  Lists are filled with atomic cursors; the few
+    // heavy vertices go through per-thread buffers instead (no cursor contention).
+    // List order is irrelevant: SCCs and layers are unique.
+    DepGraph(int64_t P_, int64_t n_, const std::vector<int64_t>& moff_, const std::vector<int32_t>& mv_,
+             const std::vector<int32_t>& outdeg, const std::vector<int32_t>& indeg)
+        : P(P_), n(n_), N(P_ + n_), moff(moff_), mv(mv_) {
+        lptr.assign(n + 1, 0);
+        eptr.assign(n + 1, 0);
+        for (int64_t x = 0; x < n; x++) { lptr[x + 1] = lptr[x] + outdeg[x]; eptr[x + 1] = eptr[x] + indeg[x]; }
+        ladj.resize(lptr[n]);
+        eadj.resize(eptr[n]);
+        constexpr int32_t kHeavy = 2048;
+        std::vector<std::atomic<int64_t>> lc(n), ec(n);
+        #pragma omp parallel for schedule(static)
+        for (int64_t x = 0; x < n; x++) { lc[x].store(lptr[x], std::memory_order_relaxed); ec[x].store(eptr[x], std::memory_order_relaxed); }
+        const int nth = omp_get_max_threads();
+        std::vector<std::vector<std::pair<int32_t, int32_t>>> hl(nth), he(nth);
+        #pragma omp parallel for schedule(dynamic, 4096)
+        for (int64_t i = 0; i < P; i++) {
+            const int t = omp_get_thread_num();
+            for (int64_t k = moff[i]; k < moff[i + 1] - 1; k++) {
+                const int32_t x = mv[k];
+                if (outdeg[x] >= kHeavy) hl[t].push_back({x, (int32_t)i});
+                else ladj[lc[x].fetch_add(1, std::memory_order_relaxed)] = (int32_t)i;
+            }
+            for (int64_t k = moff[i] + 1; k < moff[i + 1]; k++) {
+                const int32_t x = mv[k];
+                if (indeg[x] >= kHeavy) he[t].push_back({x, (int32_t)i});
+                else eadj[ec[x].fetch_add(1, std::memory_order_relaxed)] = (int32_t)i;
+            }
+        }
+        for (int t = 0; t < nth; t++) {
+            for (auto& q : hl[t]) ladj[lc[q.first].fetch_add(1, std::memory_order_relaxed)] = q.second;
+            for (auto& q : he[t]) eadj[ec[q.first].fetch_add(1, std::memory_order_relaxed)] = q.second;
+            std::vector<std::pair<int32_t, int32_t>>().swap(hl[t]);
+            std::vector<std::pair<int32_t, int32_t>>().swap(he[t]);
+        }
+    }
+    template <class F> void for_out(int64_t u, F&& f) const {
+        if (u < P) { for (int64_t k = moff[u] + 1; k < moff[u + 1]; k++) f(P + mv[k]); }
+        else { const int64_t x = u - P; for (int64_t e = lptr[x]; e < lptr[x + 1]; e++) f((int64_t)ladj[e]); }
+    }
+    template <class F> void for_in(int64_t u, F&& f) const {
+        if (u < P) { for (int64_t k = moff[u]; k < moff[u + 1] - 1; k++) f(P + mv[k]); }
+        else { const int64_t x = u - P; for (int64_t e = eptr[x]; e < eptr[x + 1]; e++) f((int64_t)eadj[e]); }
+    }
+    int64_t outdeg(int64_t u) const { return u < P ? moff[u + 1] - moff[u] - 1 : lptr[u - P + 1] - lptr[u - P]; }
+    int64_t indeg(int64_t u) const { return u < P ? moff[u + 1] - moff[u] - 1 : eptr[u - P + 1] - eptr[u - P]; }
+};
+
+// append per-thread vectors in thread order
+template <class T>
+void gather_threads(std::vector<std::vector<T>>& parts, std::vector<T>& out) {
+    out.clear();
+    size_t tot = 0;
+    for (auto& p : parts) tot += p.size();
+    out.reserve(tot);
+    for (auto& p : parts) { out.insert(out.end(), p.begin(), p.end()); p.clear(); }
+}
+
+// Iterative Tarjan restricted to the nodes with cls[u] == c; components are
+// appended to `comps` (members) in completion order = reverse topological order.
+void tarjan_class(const DepGraph& G, const std::vector<int32_t>& nodes, const std::vector<uint8_t>& cls, uint8_t c,
+                  std::vector<int32_t>& local, std::vector<std::vector<int32_t>>& comps) {
+    if (nodes.empty()) return;
+    const int32_t K = (int32_t)nodes.size();
+    for (int32_t q = 0; q < K; q++) local[nodes[q]] = q;  // classes are disjoint: no race
+    // local CSR of the class-internal out-edges
+    std::vector<int64_t> ptr(K + 1, 0);
+    std::vector<int32_t> adj;
+    for (int32_t q = 0; q < K; q++) {
+        G.for_out(nodes[q], [&](int64_t v) { if (cls[v] == c) adj.push_back(local[v]); });
+        ptr[q + 1] = (int64_t)adj.size();
+    }
+    std::vector<int32_t> index(K, -1), low(K, 0), st, work;
+    std::vector<int64_t> it(K, 0);
+    std::vector<uint8_t> onst(K, 0);
+    int32_t counter = 0;
+    for (int32_t r = 0; r < K; r++) {
         if (index[r] != -1) continue;
         index[r] = low[r] = counter++;
         st.push_back(r); onst[r] = 1; it[r] = ptr[r];
@@ -111,17 +204,192 @@ int32_t tarjan(int32_t N, const std::vector<int64_t>& ptr, const std::vector<int
                 work.pop_back();
                 if (!work.empty()) { int32_t q = work.back(); low[q] = std::min(low[q], low[v]); }
                 if (low[v] == index[v]) {
+                    comps.emplace_back();
                     while (true) {
                         int32_t x = st.back(); st.pop_back(); onst[x] = 0;
-                        comp[x] = ncomp;
+                        comps.back().push_back(nodes[x]);
                         if (x == v) break;
                     }
-                    ncomp++;
                 }
             }
         }
     }
-    return ncomp;
+}
+
+struct DagResult {
+    std::vector<int64_t> layer, scc;  // per path
+    int64_t n_layers = 0, n_dep_sccs = 0, giant = 0;
+};
+
+void dependency_dag(const DepGraph& G, DagResult& R, const std::function<void(const char*)>& phase) {
+    const int64_t P = G.P, N = G.N;
+    const int nth = omp_get_max_threads();
+    // ---- (1) trim
+    std::vector<int32_t> indeg(N), outdeg(N), rnd(N, -1);
+    std::vector<uint8_t> side(N, 0);  // 1 peeled as source, 2 peeled as sink
+    std::vector<std::atomic<uint8_t>> claimed(N);
+    std::vector<std::vector<int32_t>> parts(nth);
+    #pragma omp parallel for schedule(static)
+    for (int64_t u = 0; u < N; u++) {
+        indeg[u] = (int32_t)G.indeg(u);
+        outdeg[u] = (int32_t)G.outdeg(u);
+        const bool s = indeg[u] == 0, t = outdeg[u] == 0;
+        claimed[u].store(s || t, std::memory_order_relaxed);
+        if (s || t) { side[u] = s ? 1 : 2; rnd[u] = 0; parts[omp_get_thread_num()].push_back((int32_t)u); }
+    }
+    std::vector<int32_t> frontier, peeled_src, peeled_snk;
+    std::vector<int32_t> src_round_off{0}, snk_round_off{0};
+    gather_threads(parts, frontier);
+    for (int32_t r = 0; !frontier.empty(); r++) {
+        std::sort(frontier.begin(), frontier.end());
+        for (int32_t u : frontier) (side[u] == 1 ? peeled_src : peeled_snk).push_back(u);
+        src_round_off.push_back((int32_t)peeled_src.size());
+        snk_round_off.push_back((int32_t)peeled_snk.size());
+        #pragma omp parallel for schedule(dynamic, 256)
+        for (size_t q = 0; q < frontier.size(); q++) {
+            const int32_t u = frontier[q];
+            auto& out = parts[omp_get_thread_num()];
+            auto claim = [&](int64_t v, uint8_t sd) {
+                uint8_t z = 0;
+                if (claimed[v].compare_exchange_strong(z, 1)) { side[v] = sd; rnd[v] = r + 1; out.push_back((int32_t)v); }
+            };
+            if (side[u] == 1) {
+                G.for_out(u, [&](int64_t v) {
+                    if (__atomic_sub_fetch(&indeg[v], 1, __ATOMIC_RELAXED) == 0) claim(v, 1);
+                });
+            } else {
+                G.for_in(u, [&](int64_t w) {
+                    if (__atomic_sub_fetch(&outdeg[w], 1, __ATOMIC_RELAXED) == 0) claim(w, 2);
+                });
+            }
+        }
+        gather_threads(parts, frontier);
+    }
+    phase("dag: trim");
+    // ---- (2) forward / backward reachability of a pivot among the remaining nodes
+    std::vector<uint8_t> cls(N, 0);  // 0 peeled, 1 upstream (B\F), 2 pivot SCC, 3 unrelated, 4 downstream (F\B)
+    int64_t pivot = -1, best = -1;
+    for (int64_t u = 0; u < P; u++)
+        if (!claimed[u].load(std::memory_order_relaxed)) {
+            const int64_t sc = (G.indeg(u) + 1) * (G.outdeg(u) + 1);
+            if (sc > best) { best = sc; pivot = u; }
+        }
+    std::vector<uint8_t> F(N, 0), B(N, 0);
+    auto bfs = [&](std::vector<uint8_t>& mark, bool fwd) {
+        std::vector<int32_t> fr{(int32_t)pivot};
+        mark[pivot] = 1;
+        while (!fr.empty()) {
+            #pragma omp parallel for schedule(dynamic, 256)
+            for (size_t q = 0; q < fr.size(); q++) {
+                auto& out = parts[omp_get_thread_num()];
+                auto visit = [&](int64_t v) {
+                    if (claimed[v].load(std::memory_order_relaxed) || __atomic_load_n(&mark[v], __ATOMIC_RELAXED)) return;
+                    if (!__atomic_exchange_n(&mark[v], (uint8_t)1, __ATOMIC_RELAXED)) out.push_back((int32_t)v);
+                };
+                if (fwd) G.for_out(fr[q], visit); else G.for_in(fr[q], visit);
+            }
+            gather_threads(parts, fr);
+        }
+    };
+    if (pivot >= 0) { bfs(F, true); bfs(B, false); }
+    phase("dag: fw-bw");
+    std::vector<std::vector<int32_t>> cls_nodes(5);
+    {
+        std::vector<std::vector<std::vector<int32_t>>> tp(nth, std::vector<std::vector<int32_t>>(5));
+        #pragma omp parallel for schedule(static)
+        for (int64_t u = 0; u < N; u++) {
+            if (claimed[u].load(std::memory_order_relaxed)) continue;
+            const uint8_t c = (F[u] && B[u]) ? 2 : B[u] ? 1 : F[u] ? 4 : 3;
+            cls[u] = c;
+            tp[omp_get_thread_num()][c].push_back((int32_t)u);
+        }
+        for (int c = 1; c <= 4; c++) {
+            std::vector<std::vector<int32_t>> pc(nth);
+            for (int t = 0; t < nth; t++) pc[t].swap(tp[t][c]);
+            gather_threads(pc, cls_nodes[c]);
+        }
+    }
+    { std::vector<uint8_t>().swap(F); std::vector<uint8_t>().swap(B); }
+    phase("dag: classes");
+    // ---- (3) Tarjan on the three remaining classes (in parallel)
+    std::vector<std::vector<std::vector<int32_t>>> ccomps(5);
+    {
+        std::vector<int32_t> local(N, -1);
+        #pragma omp parallel for schedule(dynamic, 1)
+        for (int c = 1; c <= 4; c++)
+            if (c != 2) tarjan_class(G, cls_nodes[c], cls, (uint8_t)c, local, ccomps[c]);
+    }
+    phase("dag: tarjan");
+    // ---- component ids in a topological order:
+    // source peel rounds, upstream comps, pivot SCC, unrelated comps,
+    // downstream comps, sink peel rounds in reverse
+    std::vector<int32_t> comp(N, -1);
+    std::vector<int64_t> cstart{0};  // members of comp c (for the non-singleton blocks)
+    int64_t nc = 0;
+    for (int32_t u : peeled_src) comp[u] = (int32_t)nc++;
+    const int64_t c_src_end = nc;
+    std::vector<std::pair<int64_t, const std::vector<int32_t>*>> seq_comps;  // (id, members) of Tarjan comps
+    auto add_tarjan = [&](int c) {
+        auto& cc = ccomps[c];
+        for (size_t q = cc.size(); q-- > 0;) {  // completion order reversed = topological
+            for (int32_t u : cc[q]) comp[u] = (int32_t)nc;
+            seq_comps.push_back({nc, &cc[q]});
+            nc++;
+        }
+    };
+    add_tarjan(1);
+    const int64_t c_giant = cls_nodes[2].empty() ? -1 : nc;
+    if (c_giant >= 0) { for (int32_t u : cls_nodes[2]) comp[u] = (int32_t)c_giant; nc++; }
+    const size_t seq_mid = seq_comps.size();
+    add_tarjan(3);
+    add_tarjan(4);
+    std::vector<int64_t> snk_comp_base(snk_round_off.size(), 0);
+    for (int64_t r = (int64_t)snk_round_off.size() - 2; r >= 0; r--)
+        for (int32_t q = snk_round_off[r]; q < snk_round_off[r + 1]; q++) comp[peeled_snk[q]] = (int32_t)nc++;
+    // ---- per-comp path counts and smallest path index
+    std::vector<int64_t> npaths(nc, 0), minpath(nc, INT64_MAX);
+    for (int64_t i = 0; i < P; i++) {
+        npaths[comp[i]]++;
+        minpath[comp[i]] = std::min(minpath[comp[i]], i);
+    }
+    phase("dag: comp ids");
+    // ---- layers: f[d] = max over condensation edges c->d of f[c] + (c holds a path)
+    std::vector<int64_t> f(nc, 0);
+    auto push = [&](int64_t u) {
+        const int64_t cu = comp[u], val = f[cu] + (npaths[cu] > 0 ? 1 : 0);
+        G.for_out(u, [&](int64_t v) {
+            const int64_t cv = comp[v];
+            if (cv == cu) return;
+            int64_t cur = __atomic_load_n(&f[cv], __ATOMIC_RELAXED);
+            while (val > cur && !__atomic_compare_exchange_n(&f[cv], &cur, val, true, __ATOMIC_RELAXED, __ATOMIC_RELAXED)) {}
+        });
+    };
+    for (size_t r = 0; r + 1 < src_round_off.size(); r++) {
+        #pragma omp parallel for schedule(dynamic, 256)
+        for (int32_t q = src_round_off[r]; q < src_round_off[r + 1]; q++) push(peeled_src[q]);
+    }
+    for (size_t q = 0; q < seq_mid; q++) for (int32_t u : *seq_comps[q].second) push(u);
+    if (c_giant >= 0) {
+        #pragma omp parallel for schedule(dynamic, 256)
+        for (size_t q = 0; q < cls_nodes[2].size(); q++) push(cls_nodes[2][q]);
+    }
+    for (size_t q = seq_mid; q < seq_comps.size(); q++) for (int32_t u : *seq_comps[q].second) push(u);
+    for (int64_t r = (int64_t)snk_round_off.size() - 2; r >= 0; r--) {
+        #pragma omp parallel for schedule(dynamic, 256)
+        for (int32_t q = snk_round_off[r]; q < snk_round_off[r + 1]; q++) push(peeled_snk[q]);
+    }
+    (void)c_src_end;
+    (void)snk_comp_base;
+    phase("dag: layers");
+    R.layer.assign(P, 0);
+    R.scc.assign(P, 0);
+    for (int64_t i = 0; i < P; i++) {
+        R.layer[i] = f[comp[i]];
+        R.scc[i] = minpath[comp[i]];
+        R.n_layers = std::max(R.n_layers, f[comp[i]] + 1);
+    }
+    for (int64_t c = 0; c < nc; c++)
+        if (npaths[c] > 0) { R.n_dep_sccs++; R.giant = std::max(R.giant, npaths[c]); }
 }
 
 }  // namespace
@@ -198,23 +466,30 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     }
 
     phase("algorithm 1");
-    // ---- concatenate (subgraph order)
-    std::vector<int64_t> poff{0};
+    // ---- concatenate (subgraph order), in parallel over subgraphs
+    std::vector<int64_t> poff;
     std::vector<int32_t> pv, pw;
     {
-        int64_t tot = 0;
-        for (auto& s : subs) tot += (int64_t)s.pv.size();
-        pv.reserve(tot); pw.reserve(tot);
-        for (auto& s : subs) {
-            int64_t base = (int64_t)pv.size();
-            pv.insert(pv.end(), s.pv.begin(), s.pv.end());
-            pw.insert(pw.end(), s.pw.begin(), s.pw.end());
-            for (size_t i = 1; i < s.start.size(); i++) poff.push_back(base + s.start[i]);
-            std::vector<int32_t>().swap(s.pv);
-            std::vector<int32_t>().swap(s.pw);
-            std::vector<int64_t>().swap(s.start);
+        std::vector<int64_t> voff(T + 1, 0), qoff(T + 1, 0);
+        for (int k = 0; k < T; k++) {
+            voff[k + 1] = voff[k] + (int64_t)subs[k].pv.size();
+            qoff[k + 1] = qoff[k] + (int64_t)subs[k].start.size() - 1;
+        }
+        pv.resize(voff[T]); pw.resize(voff[T]);
+        poff.resize(qoff[T] + 1);
+        poff[0] = 0;
+        #pragma omp parallel for schedule(dynamic, 1)
+        for (int k = 0; k < T; k++) {
+            SubOut& s2 = subs[k];
+            std::copy(s2.pv.begin(), s2.pv.end(), pv.begin() + voff[k]);
+            std::copy(s2.pw.begin(), s2.pw.end(), pw.begin() + voff[k]);
+            for (size_t i = 1; i < s2.start.size(); i++) poff[qoff[k] + i] = voff[k] + s2.start[i];
+            std::vector<int32_t>().swap(s2.pv);
+            std::vector<int32_t>().swap(s2.pw);
+            std::vector<int64_t>().swap(s2.start);
         }
     }
+    phase("concatenate: copy");
     const int64_t P0 = (int64_t)poff.size() - 1;
     L.paths_before_merge = P0;
     if (P0 >= INT32_MAX || P0 + n >= INT32_MAX) throw std::runtime_error("too many paths for 32-bit path ids");
@@ -227,15 +502,33 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     // order merged paths by their first piece.
     std::vector<int32_t> nxt(P0, -1), prv(P0, -1);
     if (p.l_merge > 0 && P0 > 1) {
+        // paths by end vertex / by start vertex, each bucket in path order
         std::vector<int64_t> eptr(n + 1, 0), sptr(n + 1, 0);
         std::vector<int32_t> elist(P0), slist(P0);
-        for (int64_t i = 0; i < P0; i++) { eptr[pv[poff[i + 1] - 1] + 1]++; sptr[pv[poff[i]] + 1]++; }
-        for (int64_t v = 0; v < n; v++) { eptr[v + 1] += eptr[v]; sptr[v + 1] += sptr[v]; }
         {
-            std::vector<int64_t> fe(eptr.begin(), eptr.end() - 1), fs(sptr.begin(), sptr.end() - 1);
+            std::vector<std::atomic<int64_t>> ce(n), cs(n);
+            #pragma omp parallel for schedule(static)
+            for (int64_t v = 0; v < n; v++) { ce[v].store(0, std::memory_order_relaxed); cs[v].store(0, std::memory_order_relaxed); }
+            #pragma omp parallel for schedule(static)
             for (int64_t i = 0; i < P0; i++) {
-                elist[fe[pv[poff[i + 1] - 1]]++] = (int32_t)i;
-                slist[fs[pv[poff[i]]]++] = (int32_t)i;
+                ce[pv[poff[i + 1] - 1]].fetch_add(1, std::memory_order_relaxed);
+                cs[pv[poff[i]]].fetch_add(1, std::memory_order_relaxed);
+            }
+            for (int64_t v = 0; v < n; v++) {
+                eptr[v + 1] = eptr[v] + ce[v].load(std::memory_order_relaxed);
+                sptr[v + 1] = sptr[v] + cs[v].load(std::memory_order_relaxed);
+            }
+            #pragma omp parallel for schedule(static)
+            for (int64_t v = 0; v < n; v++) { ce[v].store(eptr[v], std::memory_order_relaxed); cs[v].store(sptr[v], std::memory_order_relaxed); }
+            #pragma omp parallel for schedule(static)
+            for (int64_t i = 0; i < P0; i++) {
+                elist[ce[pv[poff[i + 1] - 1]].fetch_add(1, std::memory_order_relaxed)] = (int32_t)i;
+                slist[cs[pv[poff[i]]].fetch_add(1, std::memory_order_relaxed)] = (int32_t)i;
+            }
+            #pragma omp parallel for schedule(dynamic, 4096)
+            for (int64_t v = 0; v < n; v++) {
+                std::sort(elist.begin() + eptr[v], elist.begin() + eptr[v + 1]);
+                std::sort(slist.begin() + sptr[v], slist.begin() + sptr[v + 1]);
             }
         }
         #pragma omp parallel for schedule(dynamic, 4096)
@@ -255,6 +548,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
             }
         }
     }
+    phase("merge: pairing");
     // chains (start where nothing links in), then cycles cut before their lowest index
     std::vector<uint8_t> seen(P0, 0);
     std::vector<int32_t> seg_first, seg_len;   // segments: first piece, #pieces
@@ -287,19 +581,23 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
             if (!seen[i]) walk_chain((int32_t)i, seg_pieces, seg_first, seg_len);
     }
     { std::vector<int32_t>().swap(nxt); std::vector<int32_t>().swap(prv); std::vector<uint8_t>().swap(seen); }
+    phase("merge: chains");
     const int64_t P = (int64_t)seg_first.size();
     std::vector<int64_t> seg_start(P + 1, 0);   // into seg_pieces
     for (int64_t s2 = 0; s2 < P; s2++) seg_start[s2 + 1] = seg_start[s2] + seg_len[s2];
     std::vector<int32_t> sorder(P);
     std::iota(sorder.begin(), sorder.end(), 0);
-    std::sort(sorder.begin(), sorder.end(), [&](int32_t a, int32_t b) { return seg_first[a] < seg_first[b]; });
+    __gnu_parallel::sort(sorder.begin(), sorder.end(), [&](int32_t a, int32_t b) { return seg_first[a] < seg_first[b]; });
+    phase("merge: order");
     // materialise merged paths (merge order) in parallel
     std::vector<int64_t> moff(P + 1, 0);
+    #pragma omp parallel for schedule(static)
     for (int64_t r = 0; r < P; r++) {
         int64_t sgi = sorder[r], len = 1;
         for (int64_t q = seg_start[sgi]; q < seg_start[sgi + 1]; q++) len += poff[seg_pieces[q] + 1] - poff[seg_pieces[q]] - 1;
-        moff[r + 1] = moff[r] + len;
+        moff[r + 1] = len;
     }
+    for (int64_t r = 0; r < P; r++) moff[r + 1] += moff[r];
     std::vector<int32_t> mv(moff[P]), mw(moff[P]);
     #pragma omp parallel for schedule(dynamic, 1024)
     for (int64_t r = 0; r < P; r++) {
@@ -329,63 +627,16 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     }
 
     phase("path stats");
-    // ---- dependency graph G' as a bipartite path/vertex graph (reading R-DEP):
-    // path node i -> vertex node P+x for every x entered by an edge of i;
-    // vertex node P+x -> path node j for every x left by an edge of j.
-    // Reachability between path nodes equals reachability in G'.
-    const int64_t N = P + n;
-    std::vector<int64_t> aptr(N + 1, 0);
-    std::vector<int32_t> adj;
-    std::vector<int64_t> layer_of_path(P, 0), scc_label(P, 0);
-    int64_t n_layers = 0, n_dep_sccs = 0, giant = 0;
+    // ---- dependency graph G' and DAG sketch (reading R-DEP, R-LAYER)
+    DagResult dag;
     {
-        for (int64_t i = 0; i < P; i++) {
-            int64_t len = moff[i + 1] - moff[i];
-            aptr[i + 1] += len - 1;                                   // entered vertices
-            for (int64_t k = moff[i]; k < moff[i + 1] - 1; k++) aptr[P + mv[k] + 1]++;  // left vertices
-        }
-        for (int64_t x = 0; x < N; x++) aptr[x + 1] += aptr[x];
-        adj.resize(aptr[N]);
-        std::vector<int64_t> fill(aptr.begin(), aptr.end() - 1);
-        for (int64_t i = 0; i < P; i++) {
-            for (int64_t k = moff[i] + 1; k < moff[i + 1]; k++) adj[fill[i]++] = (int32_t)(P + mv[k]);
-            for (int64_t k = moff[i]; k < moff[i + 1] - 1; k++) adj[fill[P + mv[k]]++] = (int32_t)i;
-        }
-        std::vector<int32_t> comp;
-        int64_t nc = tarjan((int32_t)N, aptr, adj, comp);
-        // group nodes by comp; comps are numbered in reverse topological order
-        std::vector<int64_t> cptr(nc + 1, 0), cnodes(N);
-        for (int64_t x = 0; x < N; x++) cptr[comp[x] + 1]++;
-        for (int64_t c = 0; c < nc; c++) cptr[c + 1] += cptr[c];
-        {
-            std::vector<int64_t> fill2(cptr.begin(), cptr.end() - 1);
-            for (int64_t x = 0; x < N; x++) cnodes[fill2[comp[x]]++] = x;
-        }
-        std::vector<int64_t> f(nc, 0), minpath(nc, INT64_MAX), npaths(nc, 0);
-        for (int64_t i = 0; i < P; i++) {
-            minpath[comp[i]] = std::min(minpath[comp[i]], i);
-            npaths[comp[i]]++;
-        }
-        // topological order = decreasing comp id (sources first)
-        for (int64_t c = nc - 1; c >= 0; c--) {
-            int64_t add = npaths[c] > 0 ? 1 : 0;
-            for (int64_t q = cptr[c]; q < cptr[c + 1]; q++) {
-                int64_t x = cnodes[q];
-                for (int64_t e = aptr[x]; e < aptr[x + 1]; e++) {
-                    int64_t d = comp[adj[e]];
-                    if (d != c) f[d] = std::max(f[d], f[c] + add);
-                }
-            }
-        }
-        for (int64_t i = 0; i < P; i++) {
-            layer_of_path[i] = f[comp[i]];
-            scc_label[i] = minpath[comp[i]];
-            n_layers = std::max(n_layers, f[comp[i]] + 1);
-        }
-        for (int64_t c = 0; c < nc; c++)
-            if (npaths[c] > 0) { n_dep_sccs++; giant = std::max(giant, npaths[c]); }
+        DepGraph DG(P, n, moff, mv, g.outdeg, g.indeg);
+        phase("dag: bipartite CSR");
+        dependency_dag(DG, dag, phase);
     }
-    { std::vector<int32_t>().swap(adj); std::vector<int64_t>().swap(aptr); }
+    const std::vector<int64_t>& layer_of_path = dag.layer;
+    const std::vector<int64_t>& scc_label = dag.scc;
+    const int64_t n_layers = dag.n_layers, n_dep_sccs = dag.n_dep_sccs, giant = dag.giant;
 
     phase("dependency DAG");
     // ---- priority Pri(p) = alpha*D(p)*N(p) - L(p)
@@ -396,7 +647,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     for (int64_t i = 0; i < P; i++) pri[i] = alpha * dbar[i] * (double)nvert[i] - (double)layer_of_path[i];
     std::vector<int64_t> order(P);
     std::iota(order.begin(), order.end(), 0);
-    std::stable_sort(order.begin(), order.end(), [&](int64_t a, int64_t b) { return pri[a] > pri[b]; });
+    __gnu_parallel::stable_sort(order.begin(), order.end(), [&](int64_t a, int64_t b) { return pri[a] > pri[b]; });
 
     // ---- partitions over the priority order (greedy, whole paths)
     // part_entries == 0: auto -- about 16K partitions (several per resident
@@ -475,26 +726,41 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
 
     phase("priority+partitions");
     // ---- this rank's layout
-    L.part_off.push_back(0);
-    L.path_off.push_back(0);
-    for (int64_t q = rank; q < G; q += world) {
-        for (int64_t r = gpart_first[q]; r < gpart_first[q + 1]; r++) {
-            int64_t i = order[r];
-            for (int64_t k = moff[i]; k < moff[i + 1]; k++) {
+    {
+        // this rank's paths (priority order within its partitions) and offsets
+        std::vector<int64_t> sel;
+        L.part_off.push_back(0);
+        std::vector<int64_t> part_paths{0};
+        for (int64_t q = rank; q < G; q += world) {
+            for (int64_t r = gpart_first[q]; r < gpart_first[q + 1]; r++) sel.push_back(order[r]);
+            part_paths.push_back((int64_t)sel.size());
+        }
+        const int64_t Q = (int64_t)sel.size();
+        L.path_off.assign(Q + 1, 0);
+        for (int64_t r = 0; r < Q; r++) L.path_off[r + 1] = L.path_off[r] + (moff[sel[r] + 1] - moff[sel[r]]);
+        for (size_t q = 1; q < part_paths.size(); q++) L.part_off.push_back(L.path_off[part_paths[q]]);
+        L.e_idx.resize(L.path_off[Q]);
+        L.e_w.resize(L.path_off[Q]);
+        L.layer.resize(Q); L.scc.resize(Q); L.merged_index.resize(Q); L.hot.resize(Q);
+        int64_t nh = 0;
+        #pragma omp parallel for schedule(dynamic, 1024) reduction(+ : nh)
+        for (int64_t r = 0; r < Q; r++) {
+            const int64_t i = sel[r];
+            int64_t o = L.path_off[r];
+            for (int64_t k = moff[i]; k < moff[i + 1]; k++, o++) {
                 uint32_t code = (uint32_t)L.new_id[mv[k]];
                 if (k == moff[i]) code |= kHead;
                 if (k == moff[i + 1] - 1) code |= kTail;
-                L.e_idx.push_back(code);
-                L.e_w.push_back(mw[k]);
+                L.e_idx[o] = code;
+                L.e_w[o] = mw[k];
             }
-            L.path_off.push_back((int64_t)L.e_idx.size());
-            L.layer.push_back((int32_t)layer_of_path[i]);
-            L.scc.push_back(scc_label[i]);
-            L.merged_index.push_back(i);
-            L.hot.push_back(hot[i]);
-            L.n_hot += hot[i];
+            L.layer[r] = (int32_t)layer_of_path[i];
+            L.scc[r] = scc_label[i];
+            L.merged_index[r] = i;
+            L.hot[r] = hot[i];
+            nh += hot[i];
         }
-        L.part_off.push_back((int64_t)L.e_idx.size());
+        L.n_hot = nh;
     }
 
     phase("layout");
