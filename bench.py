@@ -128,6 +128,26 @@ def load_peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def load_random_ceiling():
+    """Measured random-access ceilings (G ops/s) over an L2-resident array:
+    8-byte gathers alone and an even gather/RED mix (scripts/ubench_l2_random.cu,
+    profiles/r01_l2_random_ubench.txt)."""
+    p = os.path.join(ROOT, "profiles", "r01_l2_random_ubench.txt")
+    best = {}
+    try:
+        with open(p) as f:
+            for ln in f:
+                parts = ln.split()
+                if len(parts) > 3 and parts[0] in ("gather", "g+red") and "G" in parts:
+                    mb = float(ln.split("S=")[1].split("MB")[0])
+                    if mb < 100:
+                        v = float(ln.split(":")[1].split("G")[0])
+                        best[parts[0]] = max(best.get(parts[0], 0.0), v)
+    except Exception:
+        pass
+    return best
+
+
 def load_traffic(algo, config):
     """ncu DRAM bytes per launch of the dominant kernel, from the committed
     profile summary (profiles/ncu_traffic.json), or None."""
@@ -290,6 +310,17 @@ def main():
             "algorithmic_bytes_per_launch": ab, "kernel_ms": st0["kernel_ms"],
             "kernel_share_of_step": kernel_ms / ms if ms else None}
 
+    # the resource that actually binds the path walk: random 8-byte L2 accesses
+    # (one master gather per walked entry + one RED / atomicMin per update)
+    ceil = load_random_ceiling()
+    ops = st0["entries_processed"] + st0["vertex_updates"]
+    kind = "g+red" if args.algo in ("pagerank", "adsorption") else "gather"
+    ach_ops = ops / (st0["kernel_ms"] / 1e3) / 1e9 if st0["kernel_ms"] > 0 else 0.0
+    rand = {"bound": "l2_random_access", "achieved": ach_ops, "unit": "G ops/s", "ops_per_launch": ops,
+            "ceiling": ceil.get(kind), "ceiling_kind": f"measured {kind} over a 34-67 MB array "
+                                                      "(profiles/r01_l2_random_ubench.txt)",
+            "frac": (ach_ops / ceil[kind]) if ceil.get(kind) else None}
+
     extras = {}
     if not args.no_extras:
         # end-to-end through the public API with host buffers, every step: H2D
@@ -351,7 +382,7 @@ def main():
             "rounds": st0["rounds"], "vertex_updates": st0["vertex_updates"],
             "edges_processed": st0["edges_processed"], "kernel_ms": kernel_ms,
             "gpu_launches": int(sum(s["kernel_launches"] for s in stats)),
-            "roofline": roof, "clocks": clk,
+            "roofline": roof, "random_access_roofline": rand, "clocks": clk,
         }
         if syncs[-1]:
             line["sync"] = syncs[-1]

@@ -157,6 +157,15 @@ static int ensure_uploaded(dg_graph* g) {
     return g->uploaded ? DG_OK : dg_upload(g);
 }
 
+// the parts of the device layout an algorithm reads beyond the path entries
+static int ensure_parts(dg_graph* g, int algo, int mode) {
+    const bool need_csr = mode == DG_MODE_VERTEX || algo == DG_ADSORPTION;
+    const bool need_ew = (mode == DG_MODE_PATH && algo == DG_SSSP) || algo == DG_ADSORPTION;
+    std::string err;
+    int rc = dg::dev_ensure_parts(g->dev, g->csr, g->layout, need_csr, need_ew, err);
+    return rc ? fail(rc, err) : DG_OK;
+}
+
 
 
 int dg_set_vertex_params(dg_graph* g, const double* p_inj, const double* p_cont, const double* inj) {
@@ -164,6 +173,7 @@ int dg_set_vertex_params(dg_graph* g, const double* p_inj, const double* p_cont,
     if (int rc0 = select_dev(g)) return rc0;
     if (int rc0 = ensure_uploaded(g)) return rc0;
     if (!p_inj || !p_cont || !inj) return fail(DG_EINVAL, "dg_set_vertex_params: NULL array");
+    if (int rc0 = ensure_parts(g, DG_ADSORPTION, DG_MODE_PATH)) return rc0;
     for (int64_t v = 0; v < g->csr.n; v++)
         if (!(p_cont[v] >= 0 && p_cont[v] < 1 && p_inj[v] >= 0))
             return fail(DG_EINVAL, "dg_set_vertex_params: need 0 <= p_cont < 1 and p_inj >= 0");
@@ -199,6 +209,7 @@ int dg_run(dg_graph* g, int algo, int64_t source, double epsilon, double param, 
         return fail(DG_EINVAL, "dg_run: multi-rank layout; use dg_run_begin/dg_rounds/dg_boundary_*");
     if ((rc = select_dev(g))) return rc;
     if ((rc = ensure_uploaded(g))) return rc;
+    if ((rc = ensure_parts(g, algo, mode))) return rc;
     g->run = dg::RunState();
     g->run.algo = algo; g->run.mode = mode;
     g->run.source = (algo == DG_SSSP || algo == DG_BFS) ? g->layout.new_id[source] : 0;
@@ -287,6 +298,7 @@ int dg_run_begin(dg_graph* g, int algo, int64_t source, double epsilon, double p
     if (algo == DG_SCC) return fail(DG_EINVAL, "dg_run_begin: SCC is single-rank only");
     if ((rc = select_dev(g))) return rc;
     if ((rc = ensure_uploaded(g))) return rc;
+    if ((rc = ensure_parts(g, algo, DG_MODE_PATH))) return rc;
     g->run = dg::RunState();
     g->run.algo = algo; g->run.mode = DG_MODE_PATH;
     g->run.source = (algo == DG_SSSP || algo == DG_BFS) ? g->layout.new_id[source] : 0;

@@ -1401,6 +1401,10 @@ int dev_select(int device, std::string& err) {
     return DG_OK;
 }
 
+// dg_upload: the per-vertex arrays every run needs (out-degrees and both id
+// maps, internal ids); the CSR (vertex-centric ablation, Adsorption weights)
+// and the path-edge weights (SSSP) follow on first use (dev_ensure_parts), so
+// a run moves only the bytes its algorithm reads.
 int dev_upload_csr(DevLayout& D, const HostCSR& g, const HostLayout& L, std::string& err) {
     int dev_count = 0;
     if (cudaGetDeviceCount(&dev_count) != cudaSuccess || dev_count == 0) {
@@ -1410,24 +1414,43 @@ int dev_upload_csr(DevLayout& D, const HostCSR& g, const HostLayout& L, std::str
     int rc;
     D.n = g.n; D.m = g.m;
     D.h2d_bytes = 0;
+    D.csr_ok = D.ew_ok = false;
     g_h2d_counter = &D.h2d_bytes;
     g_pin_list = &D.pinned;
-    // the CSR in internal vertex ids (HostLayout), plus both id maps
-    if ((rc = dalloc_once(&D.row_ptr, g.n + 1, D.bytes, err))) return rc;
-    if ((rc = dalloc_once(&D.col, g.m + kPad, D.bytes, err))) return rc;
     if ((rc = dalloc_once(&D.outdeg, g.n + 1, D.bytes, err))) return rc;
     if ((rc = dalloc_once(&D.new_id, g.n + 1, D.bytes, err))) return rc;
     if ((rc = dalloc_once(&D.orig, g.n + 1, D.bytes, err))) return rc;
-    if ((rc = h2d(D.row_ptr, L.prow_ptr.data(), g.n + 1, err))) return rc;
-    if ((rc = h2d(D.col, L.pcol.data(), g.m, err))) return rc;
     if ((rc = h2d(D.outdeg, L.poutdeg.data(), g.n, err))) return rc;
     if ((rc = h2d(D.new_id, L.new_id.data(), g.n, err))) return rc;
     if ((rc = h2d(D.orig, L.orig.data(), g.n, err))) return rc;
-    if (g.has_w) {
-        if ((rc = dalloc_once(&D.w, g.m + kPad, D.bytes, err))) return rc;
-        if ((rc = h2d(D.w, L.pw.data(), g.m, err))) return rc;
-    }
     D.n_proxy = L.n_proxy;
+    return DG_OK;
+}
+
+int dev_ensure_parts(DevLayout& D, const HostCSR& g, const HostLayout& L, bool need_csr, bool need_ew,
+                     std::string& err) {
+    int rc;
+    g_h2d_counter = &D.h2d_bytes;
+    g_pin_list = &D.pinned;
+    if (need_csr && !D.csr_ok) {  // the CSR in internal ids (HostLayout)
+        if ((rc = dalloc_once(&D.row_ptr, g.n + 1, D.bytes, err))) return rc;
+        if ((rc = dalloc_once(&D.col, g.m + kPad, D.bytes, err))) return rc;
+        if ((rc = h2d(D.row_ptr, L.prow_ptr.data(), g.n + 1, err))) return rc;
+        if ((rc = h2d(D.col, L.pcol.data(), g.m, err))) return rc;
+        if (g.has_w) {
+            if ((rc = dalloc_once(&D.w, g.m + kPad, D.bytes, err))) return rc;
+            if ((rc = h2d(D.w, L.pw.data(), g.m, err))) return rc;
+        }
+        D.csr_ok = true;
+    }
+    if (need_ew && !D.ew_ok) {
+        if ((rc = dalloc_once(&D.e_w, D.M + kPad, D.bytes, err))) return rc;
+        CK(cudaMemset(D.e_w + D.M, 0, sizeof(int32_t) * kPad));
+        if ((rc = h2d(D.e_w, L.e_w.data(), D.M, err))) return rc;
+        D.ew_ok = true;
+    }
+    g_h2d_counter = nullptr;
+    g_pin_list = nullptr;
     return DG_OK;
 }
 
@@ -1443,13 +1466,10 @@ int dev_upload_layout(DevLayout& D, const HostLayout& L, std::string& err) {
     D.n_part = (int64_t)L.part_off.size() - 1;
     D.n_bnd = (int64_t)L.boundary.size();
     if ((rc = dalloc_once(&D.e_idx, D.M + kPad, D.bytes, err))) return rc;
-    if ((rc = dalloc_once(&D.e_w, D.M + kPad, D.bytes, err))) return rc;
     if ((rc = dalloc_once(&D.part_off, D.n_part + 1, D.bytes, err))) return rc;
     if ((rc = dalloc_once(&D.bnd, D.n_bnd + 1, D.bytes, err))) return rc;
     CK(cudaMemset(D.e_idx + D.M, 0, sizeof(uint32_t) * kPad));
-    CK(cudaMemset(D.e_w + D.M, 0, sizeof(int32_t) * kPad));
     if ((rc = h2d(D.e_idx, L.e_idx.data(), D.M, err))) return rc;
-    if ((rc = h2d(D.e_w, L.e_w.data(), D.M, err))) return rc;
     if ((rc = h2d(D.part_off, L.part_off.data(), D.n_part + 1, err))) return rc;
     if ((rc = h2d(D.bnd, L.boundary.data(), D.n_bnd, err))) return rc;
     CK(cudaDeviceSynchronize());
@@ -1469,6 +1489,7 @@ void dev_free_layout(DevLayout& D, bool csr_too) {
     if (csr_too) { dfree(D.row_ptr); dfree(D.col); dfree(D.w); dfree(D.outdeg); dfree(D.new_id); dfree(D.orig); }
     D.bytes = 0;
     D.M = D.n_part = D.n_bnd = 0;
+    D.csr_ok = D.ew_ok = false;
 }
 
 void dev_free_work(DevWork*& W) {

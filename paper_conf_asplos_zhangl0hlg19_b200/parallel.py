@@ -5,8 +5,10 @@ ordered partitions), only replica/boundary vertex states cross NVLink.
 Protocol per outer iteration ("state propagation between
 paths is done through state synchronization of vertex replicas ... in
 batches"):
-  1. every rank runs local rounds until its local active counter is zero
-     (or ``local_rounds``);
+  1. every rank runs ``local_rounds`` local rounds (default 4: the sync cost --
+     one NCCL all-reduce of the boundary over NVLink -- is amortised over a
+     few rounds while replicas stay at most a few rounds apart), or fewer if
+     its local active counter reaches zero;
   2. boundary states are packed (device kernel) and all-reduced with NCCL:
      MIN for SSSP/BFS/WCC, SUM of pending deltas for PageRank/Adsorption;
   3. unpack (device kernel) re-activates partitions of changed vertices;
@@ -31,7 +33,7 @@ def boundary_buffer(n_boundary, algo, device):
     return torch.zeros(max(int(n_boundary), 1), dtype=dtype, device=device)
 
 
-def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_rounds=1 << 30,
+def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_rounds=4,
                     max_outer=1_000_000, device=None, group=None):
     """Run ``algo`` to global convergence.  Returns (stats, sync_info)."""
     if algo not in SUM_ALGOS + MIN_ALGOS:
