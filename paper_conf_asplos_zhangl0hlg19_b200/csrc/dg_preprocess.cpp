@@ -24,6 +24,79 @@
 namespace dg {
 namespace {
 
+// Vector whose resize() leaves PODs uninitialised (the big temporaries are
+// overwritten in parallel right after; value-initialising them is a
+// single-threaded memset of tens of GB at Twitter scale).
+template <class T>
+struct NoInit : std::allocator<T> {
+    template <class U> struct rebind { using other = NoInit<U>; };
+    NoInit() = default;
+    template <class U> NoInit(const NoInit<U>&) noexcept {}
+    template <class U> void construct(U* p) noexcept { ::new ((void*)p) U; }
+    template <class U, class... A> void construct(U* p, A&&... a) { ::new ((void*)p) U(std::forward<A>(a)...); }
+};
+template <class T> using rvec = std::vector<T, NoInit<T>>;
+
+// Parallel stable group-by (radix partition + per-bucket counting sort):
+// items [0, n_items) each emit (key, value) pairs through
+// emit(item, sink); the result is a CSR over keys [0, n_keys) whose lists
+// hold the values in item order (then emission order) -- deterministic and
+// independent of the thread count.  Cache-friendly: pass 1 counts pairs per
+// (thread, bucket of 2^16 keys), pass 2 scatters them into bucket-major
+// runs, pass 3 sorts each bucket by key with a bucket-local cursor array.
+template <class Emit>
+void group_by(int64_t n_items, int64_t n_keys, Emit&& emit, std::vector<int64_t>& ptr, rvec<int32_t>& vals) {
+    constexpr int kShift = 16;
+    const int64_t B = std::max<int64_t>(1, (n_keys + (1 << kShift) - 1) >> kShift);
+    const int T = omp_get_max_threads();
+    std::vector<int64_t> cnt((size_t)T * B, 0);
+    auto chunk = [&](int t, int64_t& lo, int64_t& hi) {
+        lo = n_items * t / T;
+        hi = n_items * (t + 1) / T;
+    };
+    #pragma omp parallel num_threads(T)
+    {
+        const int t = omp_get_thread_num();
+        int64_t lo, hi;
+        chunk(t, lo, hi);
+        int64_t* c = &cnt[(size_t)t * B];
+        for (int64_t i = lo; i < hi; i++) emit(i, [&](int32_t key, int32_t) { c[key >> kShift]++; });
+    }
+    std::vector<int64_t> off((size_t)T * B), bstart(B + 1, 0);
+    {
+        int64_t acc = 0;
+        for (int64_t b = 0; b < B; b++) {
+            bstart[b] = acc;
+            for (int t = 0; t < T; t++) { off[(size_t)t * B + b] = acc; acc += cnt[(size_t)t * B + b]; }
+        }
+        bstart[B] = acc;
+    }
+    const int64_t total = bstart[B];
+    rvec<int32_t> tk(total), tv(total);
+    #pragma omp parallel num_threads(T)
+    {
+        const int t = omp_get_thread_num();
+        int64_t lo, hi;
+        chunk(t, lo, hi);
+        int64_t* o = &off[(size_t)t * B];
+        for (int64_t i = lo; i < hi; i++)
+            emit(i, [&](int32_t key, int32_t v) { const int64_t q = o[key >> kShift]++; tk[q] = key; tv[q] = v; });
+    }
+    ptr.assign(n_keys + 1, 0);
+    vals.resize(total);
+    #pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t b = 0; b < B; b++) {
+        const int64_t k0 = b << kShift, k1 = std::min<int64_t>(n_keys, (b + 1) << kShift);
+        std::vector<int64_t> cur(k1 - k0 + 1, 0);
+        for (int64_t q = bstart[b]; q < bstart[b + 1]; q++) cur[tk[q] - k0 + 1]++;
+        for (int64_t k = 0; k < k1 - k0; k++) cur[k + 1] += cur[k];
+        for (int64_t k = k0; k < k1; k++) ptr[k] = bstart[b] + cur[k - k0];
+        for (int64_t q = bstart[b]; q < bstart[b + 1]; q++) vals[bstart[b] + cur[tk[q] - k0]++] = tv[q];
+    }
+    ptr[n_keys] = total;
+}
+
+
 struct SubOut {
     std::vector<int32_t> pv;     // path vertices, concatenated
     std::vector<int32_t> pw;     // weight of the edge into each path vertex (0 at heads)
@@ -100,49 +173,18 @@ struct Decomposer {
 struct DepGraph {
     int64_t P, n, N;
     const std::vector<int64_t>& moff;
-    const std::vector<int32_t>& mv;
+    const rvec<int32_t>& mv;
     std::vector<int64_t> lptr, eptr;   // vertex x: paths leaving x / entering x
-    std::vector<int32_t> ladj, eadj;
+    rvec<int32_t> ladj, eadj;
 
-    // Every out-edge (in-edge) of x lies on exactly one path, so x is left
-    // (entered) by exactly outdeg(x) (indeg(x)) path edges: the list sizes are
-    // the graph's degrees.  Lists are filled with atomic cursors; the few
-    // heavy vertices go through per-thread buffers instead (no cursor contention).
-    // List order is irrelevant: SCCs and layers are unique.
-    DepGraph(int64_t P_, int64_t n_, const std::vector<int64_t>& moff_, const std::vector<int32_t>& mv_,
-             const std::vector<int32_t>& outdeg, const std::vector<int32_t>& indeg)
+    DepGraph(int64_t P_, int64_t n_, const std::vector<int64_t>& moff_, const rvec<int32_t>& mv_)
         : P(P_), n(n_), N(P_ + n_), moff(moff_), mv(mv_) {
-        lptr.assign(n + 1, 0);
-        eptr.assign(n + 1, 0);
-        for (int64_t x = 0; x < n; x++) { lptr[x + 1] = lptr[x] + outdeg[x]; eptr[x + 1] = eptr[x] + indeg[x]; }
-        ladj.resize(lptr[n]);
-        eadj.resize(eptr[n]);
-        constexpr int32_t kHeavy = 2048;
-        std::vector<std::atomic<int64_t>> lc(n), ec(n);
-        #pragma omp parallel for schedule(static)
-        for (int64_t x = 0; x < n; x++) { lc[x].store(lptr[x], std::memory_order_relaxed); ec[x].store(eptr[x], std::memory_order_relaxed); }
-        const int nth = omp_get_max_threads();
-        std::vector<std::vector<std::pair<int32_t, int32_t>>> hl(nth), he(nth);
-        #pragma omp parallel for schedule(dynamic, 4096)
-        for (int64_t i = 0; i < P; i++) {
-            const int t = omp_get_thread_num();
-            for (int64_t k = moff[i]; k < moff[i + 1] - 1; k++) {
-                const int32_t x = mv[k];
-                if (outdeg[x] >= kHeavy) hl[t].push_back({x, (int32_t)i});
-                else ladj[lc[x].fetch_add(1, std::memory_order_relaxed)] = (int32_t)i;
-            }
-            for (int64_t k = moff[i] + 1; k < moff[i + 1]; k++) {
-                const int32_t x = mv[k];
-                if (indeg[x] >= kHeavy) he[t].push_back({x, (int32_t)i});
-                else eadj[ec[x].fetch_add(1, std::memory_order_relaxed)] = (int32_t)i;
-            }
-        }
-        for (int t = 0; t < nth; t++) {
-            for (auto& q : hl[t]) ladj[lc[q.first].fetch_add(1, std::memory_order_relaxed)] = q.second;
-            for (auto& q : he[t]) eadj[ec[q.first].fetch_add(1, std::memory_order_relaxed)] = q.second;
-            std::vector<std::pair<int32_t, int32_t>>().swap(hl[t]);
-            std::vector<std::pair<int32_t, int32_t>>().swap(he[t]);
-        }
+        group_by(P, n, [&](int64_t i, auto&& sink) {
+            for (int64_t k = moff[i]; k < moff[i + 1] - 1; k++) sink(mv[k], (int32_t)i);
+        }, lptr, ladj);
+        group_by(P, n, [&](int64_t i, auto&& sink) {
+            for (int64_t k = moff[i] + 1; k < moff[i + 1]; k++) sink(mv[k], (int32_t)i);
+        }, eptr, eadj);
     }
     template <class F> void for_out(int64_t u, F&& f) const {
         if (u < P) { for (int64_t k = moff[u] + 1; k < moff[u + 1]; k++) f(P + mv[k]); }
@@ -418,7 +460,8 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     for (int64_t v = 0; v < n; v++) {
         int64_t b = g.row_ptr[v], e = g.row_ptr[v + 1];
         if (e - b < 2) continue;
-        std::vector<std::pair<int32_t, int32_t>> tmp(e - b);
+        static thread_local std::vector<std::pair<int32_t, int32_t>> tmp;
+        tmp.resize(e - b);
         for (int64_t i = b; i < e; i++) tmp[i - b] = {scol[i], sw[i]};
         if (p.order == 0)
             std::stable_sort(tmp.begin(), tmp.end(), [&](const auto& x, const auto& y) {
@@ -467,8 +510,8 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
 
     phase("algorithm 1");
     // ---- concatenate (subgraph order), in parallel over subgraphs
-    std::vector<int64_t> poff;
-    std::vector<int32_t> pv, pw;
+    rvec<int64_t> poff;
+    rvec<int32_t> pv, pw;
     {
         std::vector<int64_t> voff(T + 1, 0), qoff(T + 1, 0);
         for (int k = 0; k < T; k++) {
@@ -503,34 +546,10 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     std::vector<int32_t> nxt(P0, -1), prv(P0, -1);
     if (p.l_merge > 0 && P0 > 1) {
         // paths by end vertex / by start vertex, each bucket in path order
-        std::vector<int64_t> eptr(n + 1, 0), sptr(n + 1, 0);
-        std::vector<int32_t> elist(P0), slist(P0);
-        {
-            std::vector<std::atomic<int64_t>> ce(n), cs(n);
-            #pragma omp parallel for schedule(static)
-            for (int64_t v = 0; v < n; v++) { ce[v].store(0, std::memory_order_relaxed); cs[v].store(0, std::memory_order_relaxed); }
-            #pragma omp parallel for schedule(static)
-            for (int64_t i = 0; i < P0; i++) {
-                ce[pv[poff[i + 1] - 1]].fetch_add(1, std::memory_order_relaxed);
-                cs[pv[poff[i]]].fetch_add(1, std::memory_order_relaxed);
-            }
-            for (int64_t v = 0; v < n; v++) {
-                eptr[v + 1] = eptr[v] + ce[v].load(std::memory_order_relaxed);
-                sptr[v + 1] = sptr[v] + cs[v].load(std::memory_order_relaxed);
-            }
-            #pragma omp parallel for schedule(static)
-            for (int64_t v = 0; v < n; v++) { ce[v].store(eptr[v], std::memory_order_relaxed); cs[v].store(sptr[v], std::memory_order_relaxed); }
-            #pragma omp parallel for schedule(static)
-            for (int64_t i = 0; i < P0; i++) {
-                elist[ce[pv[poff[i + 1] - 1]].fetch_add(1, std::memory_order_relaxed)] = (int32_t)i;
-                slist[cs[pv[poff[i]]].fetch_add(1, std::memory_order_relaxed)] = (int32_t)i;
-            }
-            #pragma omp parallel for schedule(dynamic, 4096)
-            for (int64_t v = 0; v < n; v++) {
-                std::sort(elist.begin() + eptr[v], elist.begin() + eptr[v + 1]);
-                std::sort(slist.begin() + sptr[v], slist.begin() + sptr[v + 1]);
-            }
-        }
+        std::vector<int64_t> eptr, sptr;
+        rvec<int32_t> elist, slist;
+        group_by(P0, n, [&](int64_t i, auto&& sink) { sink(pv[poff[i + 1] - 1], (int32_t)i); }, eptr, elist);
+        group_by(P0, n, [&](int64_t i, auto&& sink) { sink(pv[poff[i]], (int32_t)i); }, sptr, slist);
         #pragma omp parallel for schedule(dynamic, 4096)
         for (int64_t x = 0; x < n; x++) {
             const int64_t na = eptr[x + 1] - eptr[x], nb = sptr[x + 1] - sptr[x];
@@ -569,9 +588,52 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     {
         const int nth = omp_get_max_threads();
         std::vector<std::vector<int32_t>> tp(nth), tf(nth), tl(nth);
-        #pragma omp parallel for schedule(dynamic, 4096)
-        for (int64_t i = 0; i < P0; i++)
-            if (prv[i] == -1) { int t = omp_get_thread_num(); walk_chain((int32_t)i, tp[t], tf[t], tl[t]); }
+        // chains from their heads are disjoint; each thread walks 16 of them
+        // round-robin so 16 independent pointer-chasing misses are in flight
+        // (segment order is irrelevant: segments are sorted by first piece below)
+        #pragma omp parallel
+        {
+            const int t = omp_get_thread_num(), T = omp_get_num_threads();
+            constexpr int K = 16;
+            struct Cur { int32_t j = -1; int64_t len = 0; int32_t cnt = 0; std::vector<int32_t> pieces, sf, sl; };
+            std::vector<Cur> cs(K);
+            int64_t i = P0 * t / T;
+            const int64_t iend = P0 * (t + 1) / T;
+            int active = 0;
+            auto start = [&](Cur& c) {
+                while (i < iend && prv[i] != -1) i++;
+                if (i >= iend) return false;
+                c.j = (int32_t)i++; c.len = 0; c.cnt = 0;
+                return true;
+            };
+            for (auto& c : cs) if (start(c)) active++;
+            while (active) {
+                for (auto& c : cs) {
+                    if (c.j < 0) continue;
+                    const int32_t j = c.j;
+                    seen[j] = 1;
+                    const int64_t e = poff[j + 1] - poff[j] - 1;
+                    if (c.cnt && c.len + e > p.l_merge) { c.sl.push_back(c.cnt); c.cnt = 0; c.len = 0; }
+                    if (!c.cnt) c.sf.push_back(j);
+                    c.pieces.push_back(j);
+                    c.cnt++; c.len += e;
+                    const int32_t nj = nxt[j];
+                    if (nj != -1) {
+                        __builtin_prefetch(&nxt[nj]);
+                        __builtin_prefetch(&poff[nj]);
+                        c.j = nj;
+                    } else {
+                        c.sl.push_back(c.cnt);
+                        tp[t].insert(tp[t].end(), c.pieces.begin(), c.pieces.end());
+                        tf[t].insert(tf[t].end(), c.sf.begin(), c.sf.end());
+                        tl[t].insert(tl[t].end(), c.sl.begin(), c.sl.end());
+                        c.pieces.clear(); c.sf.clear(); c.sl.clear();
+                        c.j = -1;
+                        if (!start(c)) active--;
+                    }
+                }
+            }
+        }
         for (int t = 0; t < nth; t++) {
             seg_pieces.insert(seg_pieces.end(), tp[t].begin(), tp[t].end());
             seg_first.insert(seg_first.end(), tf[t].begin(), tf[t].end());
@@ -598,7 +660,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
         moff[r + 1] = len;
     }
     for (int64_t r = 0; r < P; r++) moff[r + 1] += moff[r];
-    std::vector<int32_t> mv(moff[P]), mw(moff[P]);
+    rvec<int32_t> mv(moff[P]), mw(moff[P]);
     #pragma omp parallel for schedule(dynamic, 1024)
     for (int64_t r = 0; r < P; r++) {
         int64_t sgi = sorder[r], o = moff[r];
@@ -609,7 +671,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
             first = false;
         }
     }
-    { std::vector<int32_t>().swap(pv); std::vector<int32_t>().swap(pw); }
+    { rvec<int32_t>().swap(pv); rvec<int32_t>().swap(pw); }
 
     phase("merge");
     // ---- path statistics (reading R-HOT)
@@ -630,7 +692,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
     // ---- dependency graph G' and DAG sketch (reading R-DEP, R-LAYER)
     DagResult dag;
     {
-        DepGraph DG(P, n, moff, mv, g.outdeg, g.indeg);
+        DepGraph DG(P, n, moff, mv);
         phase("dag: bipartite CSR");
         dependency_dag(DG, dag, phase);
     }
