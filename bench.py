@@ -83,6 +83,17 @@ class ClockSampler:
             self.proc.kill()
         sm, mx, reasons = [], [], set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        how = "sampled every 100 ms during the timed region"
+        if not any(len(ln.split(",")) >= 7 for ln in self.lines):
+            # the timed region was shorter than one sampling period: one query
+            # right after it (clocks and throttle reasons of the same warm state)
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=10)
+                self.lines = out.stdout.strip().splitlines()
+                how = "timed region < 100 ms: one query right after it"
+            except Exception:
+                pass
         for ln in self.lines:
             parts = [p.strip() for p in ln.split(",")]
             if len(parts) < 7:
@@ -96,7 +107,7 @@ class ClockSampler:
                 if v.lower().startswith("active"):
                     reasons.add(nm)
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+                "reasons": sorted(reasons), "samples": len(sm), "how": how}
 
 
 # ----------------------------------------------------------------- roofline

@@ -85,6 +85,7 @@ struct DevWork {
     int32_t* scc_label = nullptr;
     uint8_t* scc_mark = nullptr;
     int32_t* remaining = nullptr;
+    uint32_t* out_stage = nullptr;         // dg_get_states staging buffer (n words)
     cudaEvent_t ev0 = nullptr, ev1 = nullptr, kev0 = nullptr, kev1 = nullptr;
     bool have_params = false;
 };
@@ -256,14 +257,24 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
         if (w.base != kNoWin && w.base + 4 * lane < w.end) c = ld_stream_u4(P.e_idx + w.base + 4 * lane);
         return c;
     };
-    // signal bits of a window; if any is set, issue its master gathers
-    auto probe = [&](const Win& w, const uint4& code, bool (&act)[4], uint32_t (&a)[4]) {
-        bool any = false;
+    // signal-bitmap words of a window's entries (issued two windows ahead)
+    auto probe_words = [&](const Win& w, const uint4& code, uint4& words) {
+        words = make_uint4(0u, 0u, 0u, 0u);
+        if (w.base == kNoWin) return;
 #pragma unroll
         for (int k = 0; k < 4; k++) {
             const uint32_t i = w.base + 4 * lane + k;
-            const bool valid = w.base != kNoWin && i >= w.beg && i < w.end;
-            act[k] = valid && test_bit(bcur, u4get(code, k) & kVMask);
+            const uint32_t wd = (i >= w.beg && i < w.end) ? bcur[(u4get(code, k) & kVMask) >> 5] : 0u;
+            if (k == 0) words.x = wd; else if (k == 1) words.y = wd; else if (k == 2) words.z = wd; else words.w = wd;
+        }
+    };
+    // the window's signal bits; if one is set, issue its master gathers (one window ahead)
+    auto probe_finish = [&](const Win& w, const uint4& code, const uint4& words, bool (&act)[4], uint32_t (&a)[4]) {
+        bool any = false;
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            const uint32_t v = u4get(code, k) & kVMask;
+            act[k] = (u4get(words, k) >> (v & 31)) & 1u;
             any |= act[k];
         }
         any = __any_sync(0xffffffffu, any);
@@ -277,19 +288,26 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
         return any;
     };
 
+    // pipeline: indices three windows ahead, bitmap words two ahead, masters one ahead
     Win wc = win_first_of(P, ticket);
     if (wc.base == kNoWin) return;
     Win wn = win_next(P, wc, ticket);
-    uint4 code_c = load_code(wc), code_n = load_code(wn);
+    Win wn2 = win_next(P, wn, ticket);
+    uint4 code_c = load_code(wc), code_n = load_code(wn), code_n2 = load_code(wn2);
+    uint4 words_c, words_n;
+    probe_words(wc, code_c, words_c);
+    probe_words(wn, code_n, words_n);
     bool act_c[4], act_n[4];
     uint32_t a_c[4] = {INF, INF, INF, INF}, a_n[4] = {INF, INF, INF, INF};
-    bool any_c = probe(wc, code_c, act_c, a_c);
+    bool any_c = probe_finish(wc, code_c, words_c, act_c, a_c);
     uint32_t carry = INF;
     bool carry_live = false;
     while (wc.base != kNoWin) {
-        const Win wnn = win_next(P, wn, ticket);
-        const uint4 code_nn = load_code(wnn);
-        const bool any_n = probe(wn, code_n, act_n, a_n);
+        const Win wn3 = win_next(P, wn2, ticket);
+        const uint4 code_n3 = load_code(wn3);
+        uint4 words_n2;
+        probe_words(wn2, code_n2, words_n2);
+        const bool any_n = probe_finish(wn, code_n, words_n, act_n, a_n);
         if (wc.base == (wc.beg & ~3u)) { carry = INF; carry_live = false; }  // partition start
         const uint32_t i0 = wc.base + 4 * lane;
         // WCC looks one entry ahead: the path edge into the next window is walked backwards too
@@ -403,8 +421,9 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
             carry_live = false;
         }
         // rotate the pipeline
-        wc = wn; wn = wnn;
-        code_c = code_n; code_n = code_nn;
+        wc = wn; wn = wn2; wn2 = wn3;
+        code_c = code_n; code_n = code_n2; code_n2 = code_n3;
+        words_n = words_n2;
         any_c = any_n;
 #pragma unroll
         for (int k = 0; k < 4; k++) { act_c[k] = act_n[k]; a_c[k] = a_n[k]; }
@@ -436,11 +455,30 @@ __device__ __forceinline__ float fx_to(unsigned long long v) { return __ull2floa
 // pushed new states of its local mirrors ... sent to the master when the
 // partition assigned to this SMX has been handled".  Per CTA: the round-start
 // totals and the CTA's unflushed pushes.
+// The pushes accumulate in two 32-bit words per hub (lo, hi) because shared
+// memory has native 32-bit atomic adds only (a 64-bit add is a CAS loop): lo
+// takes the push, its carry goes to hi.  A concurrent reader can see a carry
+// not yet applied (an under-estimate: pend only shrinks, safe) and a flush can
+// leave a pending carry for the next flush (the total is conserved).
 struct Proxies {
     unsigned long long* T;
-    unsigned long long* acc;
+    unsigned* acc;  // 2 words per hub
     int64_t H;
 };
+__device__ __forceinline__ void px_add(unsigned* a, unsigned long long p) {
+    const unsigned lo = (unsigned)p, hi = (unsigned)(p >> 32);
+    const unsigned old = atomicAdd(&a[0], lo);
+    const unsigned c = hi + (old + lo < old ? 1u : 0u);
+    if (c) atomicAdd(&a[1], c);
+}
+__device__ __forceinline__ unsigned long long px_read(const unsigned* a) {
+    const unsigned lo = *(const volatile unsigned*)&a[0], hi = *(const volatile unsigned*)&a[1];
+    return ((unsigned long long)hi << 32) + lo;
+}
+__device__ __forceinline__ unsigned long long px_take(unsigned* a) {
+    const unsigned lo = atomicExch(&a[0], 0u), hi = atomicExch(&a[1], 0u);
+    return ((unsigned long long)hi << 32) + lo;
+}
 
 // Walk all windows the warp obtains in this round.  Software pipeline over the
 // window stream: while window w is walked, the master totals of window w+1
@@ -510,7 +548,7 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
                 c = __shfl_sync(0xffffffffu, c, 0);
                 if (c % P.px_refresh == 0) {
                     for (int64_t i = lane; i < px.H; i += 32) {
-                        const unsigned long long a = atomicExch(&px.acc[i], 0ull);
+                        const unsigned long long a = px_take(&px.acc[2 * i]);
                         if (a) atomicAdd(&P.vs_t[i], a);
                     }
                     __syncwarp();
@@ -534,7 +572,7 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
             T[k] = 0ull;
             if (valid[k]) {
                 if (vtx[k] < px.H) {
-                    T[k] = px.T[vtx[k]] + *(volatile unsigned long long*)&px.acc[vtx[k]];
+                    T[k] = px.T[vtx[k]] + px_read(&px.acc[2 * vtx[k]]);
                 } else {
                     const uint4 q = gbuf[slot * 128 + k * 32 + lane];
                     T[k] = (vtx[k] & 1u) ? ((unsigned long long)q.w << 32 | q.z) : ((unsigned long long)q.y << 32 | q.x);
@@ -586,7 +624,7 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
                 if (!hd[k]) acc.edges++;
                 const unsigned long long p = fx_from(pin[k]);
                 if (p) {
-                    if (vtx[k] < px.H) atomicAdd(&px.acc[vtx[k]], p);  // proxy: shared-memory atomic
+                    if (vtx[k] < px.H) px_add(&px.acc[2 * vtx[k]], p);  // proxy: shared-memory atomics
                     else atomicAdd(&P.vs_t[vtx[k]], p);                 // master: REDG (no return)
                     acc.upd++;
                 }
@@ -741,7 +779,7 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
         gbuf = reinterpret_cast<uint4*>(dyn_smem) + (size_t)(threadIdx.x >> 5) * 256;
         px.H = P.n_proxy;
         px.T = reinterpret_cast<unsigned long long*>(dyn_smem + kGbufBytes);
-        px.acc = px.T + px.H;
+        px.acc = reinterpret_cast<unsigned*>(px.T + px.H);
     }
     Acc acc;
     int r = 0;
@@ -755,7 +793,7 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             if (px.H) {  // round-start snapshot of the proxied masters
                 for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) {
                     px.T[i] = __ldcg(&P.vs_t[i]);
-                    px.acc[i] = 0ull;
+                    px.acc[2 * i] = px.acc[2 * i + 1] = 0u;
                 }
                 if (threadIdx.x == 0) s_done = 0;
                 __syncthreads();
@@ -764,7 +802,7 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             if (px.H) {  // send the proxies' accumulated pushes to their masters
                 __syncthreads();
                 for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x)
-                    if (px.acc[i]) atomicAdd(&P.vs_t[i], px.acc[i]);
+                    if (const unsigned long long a = px_read(&px.acc[2 * i])) atomicAdd(&P.vs_t[i], a);
             }
             grid.sync();  // all pushes of the round landed
             accum_sweep(P, acc.sig);
@@ -1496,7 +1534,7 @@ void dev_free_work(DevWork*& W) {
     if (!W) return;
     dfree(W->vs_u); dfree(W->vs_f); dfree(W->vs_t); dfree(W->sigma); dfree(W->s_val); dfree(W->bnd_base);
     dfree(W->e_coef); dfree(W->pr_coef); dfree(W->ads_base); dfree(W->bits); dfree(W->vlist[0]); dfree(W->vlist[1]);
-    dfree(W->ctr); dfree(W->dsum); dfree(W->scc_label); dfree(W->scc_mark); dfree(W->remaining);
+    dfree(W->ctr); dfree(W->dsum); dfree(W->scc_label); dfree(W->scc_mark); dfree(W->remaining); dfree(W->out_stage);
     if (W->ev0) cudaEventDestroy(W->ev0);
     if (W->ev1) cudaEventDestroy(W->ev1);
     if (W->kev0) cudaEventDestroy(W->kev0);
@@ -1659,8 +1697,11 @@ int dev_get_states(DevWork* W, const DevLayout& D, const RunState& S, void* out,
     if (!W) { err = "no run state"; return DG_EINVAL; }
     void* dst = out;
     void* tmp = nullptr;
-    if (!out_is_device) {
-        CK(cudaMalloc(&tmp, 4 * (size_t)std::max<int64_t>(n, 1)));
+    if (!out_is_device) {  // device staging buffer kept in the work set (no cudaMalloc per call)
+        int64_t bytes = 0;
+        int rc;
+        if (!W->out_stage && (rc = dalloc(&W->out_stage, (size_t)std::max<int64_t>(n, 1), bytes, err))) return rc;
+        tmp = W->out_stage;
         dst = tmp;
     }
     const int g = grid_1d(n);
@@ -1678,7 +1719,6 @@ int dev_get_states(DevWork* W, const DevLayout& D, const RunState& S, void* out,
     CK(cudaGetLastError());
     if (tmp) {
         cudaError_t e = cudaMemcpy(out, tmp, 4 * (size_t)n, cudaMemcpyDeviceToHost);
-        cudaFree(tmp);
         if (e != cudaSuccess) { err = cudaGetErrorString(e); return DG_ENOCUDA; }
     } else {
         CK(cudaDeviceSynchronize());
