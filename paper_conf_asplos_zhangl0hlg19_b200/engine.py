@@ -65,6 +65,7 @@ class DiGraph:
         self.n, self.m = int(n), int(self._row_ptr[-1])
         check(self._L.dg_load_csr(self._h, self.n, self.m, _p(self._row_ptr), _p(self._col), _p(self._w)),
               "dg_load_csr")
+        self._row_ptr = self._col = self._w = None  # dg_load_csr copied them
         return self
 
     def load_graph(self, g):
