@@ -31,6 +31,10 @@ CONFIGS = {
     "friendster": dict(kind="rmat", scale=26, n=65_608_366, m=1_806_067_135),
     # configs[4]: long-chain-heavy digraph (100M vertices, 2B edges)
     "chains": dict(kind="chains", n=100_000_000, m=2_000_000_000, chain_len=4096),
+    # configs[4] at 1/4 scale for one host (same chain length and cross-edge mix)
+    "chains_q": dict(kind="chains", n=25_000_000, m=500_000_000, chain_len=4096),
+    # configs[4] at 1/40 scale (CPU-side checks)
+    "chains_s": dict(kind="chains", n=2_500_000, m=50_000_000, chain_len=4096),
 }
 
 

@@ -116,6 +116,7 @@ struct KParams {
     unsigned long long eps_fx;
     int max_rounds;
     int px_refresh;  // partitions a CTA walks between mid-round proxy flushes (0: round end only)
+    int part_order;  // 0: priority order; 1: reversed; k > 1: t -> t*k mod n_part (k coprime to n_part)
 };
 
 // ------------------------------------------------------------------ helpers
@@ -231,6 +232,8 @@ __device__ __forceinline__ Win win_first_of(const KParams& P, unsigned* ticket) 
     if ((threadIdx.x & 31) == 0) t = atomicAdd(ticket, 1u);
     t = __shfl_sync(0xffffffffu, t, 0);
     if (t >= (unsigned)P.n_part) return Win{kNoWin, 0, 0};
+    if (P.part_order == 1) t = (unsigned)P.n_part - 1 - t;  // developer knob: dispatch-order experiments
+    else if (P.part_order > 1) t = (unsigned)(((unsigned long long)t * P.part_order) % (unsigned long long)P.n_part);
     const uint32_t beg = (uint32_t)P.part_off[t], end = (uint32_t)P.part_off[t + 1];
     return Win{beg & ~3u, beg, end};
 }
@@ -1286,6 +1289,12 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
     {
         const char* e = std::getenv("DG_PROXY_REFRESH");  // developer knob
         P.px_refresh = e ? std::atoi(e) : DG_PROXY_REFRESH;
+        const char* o = std::getenv("DG_PART_ORDER");
+        P.part_order = o ? std::atoi(o) : 0;
+        if (P.part_order > 1) {  // keep the map a permutation
+            auto gcd = [](long long a, long long b) { while (b) { long long t2 = a % b; a = b; b = t2; } return a; };
+            while (gcd(P.part_order, D.n_part) != 1) P.part_order++;
+        }
     }
     return coop_launch(W, fn, P, S, err, smem);
 }
