@@ -1,0 +1,95 @@
+"""-m gpu: the asynchronous path walk must not depend on WHEN a partition is
+walked (sec. 3.1: paths are handled concurrently and asynchronously;
+any interleaving of the pushes reaches the same fixed point).  The dispatch
+order of the partitions is permuted through the kernel's developer knob
+(DG_PART_ORDER: 1 = reversed, k > 1 = t -> t*k mod #partitions) and the
+results are compared with the oracle: bit-exact for the min-plus algorithms,
+within the PageRank tolerance for the accumulative one.
+
+Also checks the bytes the public API moves: dg_upload copies only what every
+run needs, SSSP adds the path-edge weights and the vertex-centric ablation
+the CSR, each once.
+"""
+import os
+
+import numpy as np
+import pytest
+
+import inputs
+from oracle import algorithms as OA
+from paper_conf_asplos_zhangl0hlg19_b200 import DiGraph
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(autouse=True)
+def _cuda(cuda_required):
+    pass
+
+
+@pytest.fixture(scope="module")
+def graph():
+    return inputs.rmat(13, 8192, 90000, seed=21)
+
+
+@pytest.fixture(params=["1", "7919", "65537"])
+def order(request):
+    old = os.environ.get("DG_PART_ORDER")
+    os.environ["DG_PART_ORDER"] = request.param
+    yield request.param
+    if old is None:
+        os.environ.pop("DG_PART_ORDER", None)
+    else:
+        os.environ["DG_PART_ORDER"] = old
+
+
+def test_sssp_bfs_wcc_exact_under_any_dispatch_order(graph, order):
+    g = graph
+    dg = DiGraph()
+    dg.load_graph(g)
+    dg.build_paths(part_entries=128)
+    src, dst, w = g.edges()
+    dg.run("sssp", source=0)
+    assert np.array_equal(dg.get_states().astype(np.int64), OA.sssp_bellman_ford(g.n, src, dst, w, 0)[0])
+    dg.run("bfs", source=0)
+    assert np.array_equal(dg.get_states().astype(np.int64), OA.bfs_levels(g.n, src, dst, 0))
+    dg.run("wcc")
+    assert np.array_equal(dg.get_states().astype(np.int64), OA.wcc_label_propagation(g.n, src, dst)[0])
+    dg.run("scc")
+    assert np.array_equal(dg.get_states().astype(np.int64), OA.scc_tarjan(g.n, src, dst))
+
+
+def test_pagerank_within_tolerance_under_any_dispatch_order(graph, order):
+    g = graph
+    dg = DiGraph()
+    dg.load_graph(g)
+    dg.build_paths(part_entries=128)
+    dg.run("pagerank", epsilon=1e-7)
+    got = dg.get_states().astype(np.float64)
+    src, dst, _ = g.edges()
+    exp, _ = OA.pagerank_power(g.n, src, dst, d=0.85, tol=1e-12)
+    assert np.abs(got - exp).sum() <= 1e-4
+    assert (np.abs(got - exp) / exp).max() <= 1e-3
+
+
+def test_upload_moves_only_what_the_algorithm_reads(graph):
+    g = graph
+    dg = DiGraph()
+    dg.load_graph(g)
+    dg.build_paths()
+    dg.upload()
+    info = dg.layout_info()
+    base = info["h2d_bytes"]
+    M, n = info["n_entries"], g.n
+    # e_idx + part_off + per-vertex maps (out-degree, both id maps); no weights, no CSR
+    assert base == 4 * M + 8 * (info["n_partitions"] + 1) + 12 * n
+    dg.run("pagerank")
+    assert dg.layout_info()["h2d_bytes"] == base
+    dg.run("sssp", source=0)
+    assert dg.layout_info()["h2d_bytes"] == base + 4 * M           # path-edge weights, once
+    dg.run("sssp", source=0)
+    assert dg.layout_info()["h2d_bytes"] == base + 4 * M
+    dg.run("sssp", source=0, mode="vertex")                        # the ablation reads the CSR
+    assert dg.layout_info()["h2d_bytes"] == base + 4 * M + 8 * (n + 1) + 8 * g.m
+    dg.upload()                                                    # a new upload starts over
+    assert dg.layout_info()["h2d_bytes"] == base
