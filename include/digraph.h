@@ -160,7 +160,13 @@ int dg_set_vertex_params(dg_graph *g, const double *p_inj, const double *p_cont,
  *   epsilon  PageRank/Adsorption per-vertex stop threshold on the delta
  *            (north_star: 1e-7 with unnormalised ranks (1-d) + d*sum);
  *            ignored by the exact algorithms
- *   param    PageRank damping d (0 < d < 1); ignored otherwise
+ *   param    PageRank: damping d (0 < d < 1).
+ *            SSSP/BFS: bucket width Delta of the rounds (DESIGN.md reading
+ *            R-DELTA): a round commits only distances <= (smallest distance
+ *            signalled by the previous round) + Delta.  0 = library default
+ *            (SSSP: 2 * max edge weight; BFS: unbounded), < 0 = unbounded,
+ *            > 0 = that width.  Results are exact for every value; it trades
+ *            redundant updates against rounds.  Ignored by the others.
  *   mode     DG_MODE_PATH or DG_MODE_VERTEX (ablation)
  *   max_rounds  safety cap (<= 0: 1,000,000)
  *   stats    may be NULL

@@ -89,6 +89,9 @@ int dg_load_csr(dg_graph* g, int64_t n, int64_t m, const int64_t* row_ptr, const
         c.col.assign(col, col + m);
         c.has_w = weight != nullptr;
         if (weight) c.w.assign(weight, weight + m);
+        c.max_w = 1;
+        if (weight)
+            for (int64_t e = 0; e < m; e++) c.max_w = std::max(c.max_w, weight[e]);
         c.indeg.assign(n, 0); c.outdeg.assign(n, 0);
         for (int64_t v = 0; v < n; v++) {
             if (row_ptr[v + 1] < row_ptr[v]) return fail(DG_EINVAL, "dg_load_csr: row_ptr decreasing");
@@ -187,6 +190,14 @@ int dg_set_vertex_params(dg_graph* g, const double* p_inj, const double* p_cont,
     return rc ? fail(rc, err) : DG_OK;
 }
 
+// SSSP/BFS bucket width from dg_run's param (include/digraph.h, reading R-DELTA)
+static int64_t run_delta(const dg_graph* g, int algo, double param) {
+    if (algo != DG_SSSP && algo != DG_BFS) return 0;
+    if (param > 0) return (int64_t)param;
+    if (param < 0) return 0;
+    return algo == DG_SSSP ? 2 * (int64_t)g->csr.max_w : 0;
+}
+
 static int check_run_args(dg_graph* g, int algo, int64_t source, double epsilon, double param, int mode) {
     if (!g || !g->layout.built) return fail(DG_EINVAL, "dg_run: no layout built");
     if (algo < DG_SSSP || algo > DG_ADSORPTION) return fail(DG_EINVAL, "dg_run: unknown algorithm");
@@ -214,6 +225,7 @@ int dg_run(dg_graph* g, int algo, int64_t source, double epsilon, double param, 
     g->run.algo = algo; g->run.mode = mode;
     g->run.source = (algo == DG_SSSP || algo == DG_BFS) ? g->layout.new_id[source] : 0;
     g->run.eps = epsilon; g->run.param = param;
+    g->run.delta = run_delta(g, algo, param);
     std::string err;
     rc = dg::dev_run(g->work, g->dev, g->run, max_rounds <= 0 ? 1000000 : max_rounds, err);
     if (stats) *stats = g->run.stats;
@@ -303,6 +315,7 @@ int dg_run_begin(dg_graph* g, int algo, int64_t source, double epsilon, double p
     g->run.algo = algo; g->run.mode = DG_MODE_PATH;
     g->run.source = (algo == DG_SSSP || algo == DG_BFS) ? g->layout.new_id[source] : 0;
     g->run.eps = epsilon; g->run.param = param;
+    g->run.delta = run_delta(g, algo, param);
     g->run.raw_states = g->layout.params.world > 1;
     std::string err;
     rc = dg::dev_run_begin(g->work, g->dev, g->run, err);

@@ -23,6 +23,7 @@ struct HostCSR {
     std::vector<int64_t> row_ptr;
     std::vector<int32_t> col, w;
     bool has_w = false;
+    int32_t max_w = 1;  // largest edge weight (1 without weights)
     std::vector<int32_t> indeg, outdeg;
 };
 
@@ -81,6 +82,7 @@ struct RunState {
     int algo = -1, mode = 0;
     int64_t source = 0;
     double eps = 0, param = 0;
+    int64_t delta = 0;  // SSSP/BFS bucket width (reading R-DELTA), 0 = unbounded
     int64_t round = 0;
     bool raw_states = false;  // multi-rank: per-rank additive contributions, not normalised
     dg_run_stats stats{};

@@ -62,6 +62,7 @@ struct Counters {
     unsigned long long updates, edges, units, entries, pushes;
     unsigned int active[2];  // path mode: vertices signalled into bitmap[k]; vertex mode: frontier sizes
     unsigned int ticket[2];
+    unsigned int minval[2];  // SSSP/BFS: smallest distance signalled into bitmap[k] (bucket base of its round)
     int round;  // global round number of the next round
     int pad;
 };
@@ -117,6 +118,8 @@ struct KParams {
     int max_rounds;
     int px_refresh;  // partitions a CTA walks between mid-round proxy flushes (0: round end only)
     int part_order;  // 0: priority order; 1: reversed; k > 1: t -> t*k mod n_part (k coprime to n_part)
+    uint64_t hot_master_bytes;  // evict-last prefix of the accumulative masters
+    uint32_t delta;  // SSSP/BFS bucket width (reading R-DELTA); 0 = unbounded
 };
 
 // ------------------------------------------------------------------ helpers
@@ -157,6 +160,18 @@ __device__ __forceinline__ unsigned long long policy_evict_last() {
     unsigned long long p;
     asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
     return p;
+}
+// Masters: evict-last for the hot prefix of the degree-ordered state array
+// (the vertices most entries touch), unchanged priority for the cold tail --
+// when the states exceed L2 (Twitter scale) the hot prefix stays resident.
+__device__ __forceinline__ unsigned long long policy_masters(const void* base, uint32_t hot_bytes, uint32_t total) {
+    unsigned long long p;
+    asm volatile("createpolicy.range.global.L2::evict_last.L2::evict_unchanged.b64 %0, [%1], %2, %3;"
+                 : "=l"(p) : "l"(base), "r"(hot_bytes), "r"(total));
+    return p;
+}
+__device__ __forceinline__ void red_add_u64_h(unsigned long long* p, unsigned long long v, unsigned long long pol) {
+    asm volatile("red.global.add.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(pol) : "memory");
 }
 __device__ __forceinline__ uint4 ld_stream_u4_h(const uint32_t* p, unsigned long long pol) {
     uint4 r;
@@ -205,6 +220,7 @@ __device__ __forceinline__ bool signal_vertex(uint32_t* b, uint32_t v) {
 struct Acc {
     unsigned upd = 0, edges = 0, units = 0, entries = 0, pushes = 0;
     unsigned sig = 0;
+    uint32_t vmin = 0x7FFFFFFFu;  // SSSP/BFS: smallest distance committed this round
 };
 
 // ------------------------------------------------------------------ path walks
@@ -252,7 +268,8 @@ __device__ __forceinline__ Win win_next(const KParams& P, const Win& w, unsigned
 // asynchronous semantics of any concurrent update; atomicMin stays the
 // authority), as are the indices of window w+2.
 template <int MODE>
-__device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t* bcur, uint32_t* bnxt, Acc& acc) {
+__device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t* bcur, uint32_t* bnxt,
+                             uint32_t theta, Acc& acc) {
     const int lane = threadIdx.x & 31;
     const uint4 kFill = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
     auto load_code = [&](const Win& w) {
@@ -303,7 +320,7 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
     bool act_c[4], act_n[4];
     uint32_t a_c[4] = {INF, INF, INF, INF}, a_n[4] = {INF, INF, INF, INF};
     bool any_c = probe_finish(wc, code_c, words_c, act_c, a_c);
-    uint32_t carry = INF;
+    uint32_t carry = INF, carry_vtx = 0;
     bool carry_live = false;
     while (wc.base != kNoWin) {
         const Win wn3 = win_next(P, wn2, ticket);
@@ -401,23 +418,34 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
                 }
             }
             bool changed3 = false;
+            // path predecessor of entry 0 (previous lane's last entry, or the carry's vertex)
+            uint32_t pred0 = __shfl_up_sync(0xffffffffu, vtx[3], 1);
+            if (lane == 0) pred0 = carry_vtx;
 #pragma unroll
             for (int k = 0; k < 4; k++) {
                 if (!live[k]) continue;
                 acc.entries++;
                 if (!(u4get(code_c, k) & kHead)) acc.edges++;
                 if (val[k] < a[k]) {
+                    if (val[k] > theta) {
+                        // beyond this round's bucket: not committed; the path
+                        // predecessor stays active so the edge is relaxed again
+                        acc.sig += signal_vertex(bnxt, k ? vtx[k - 1] : pred0);
+                        continue;
+                    }
                     const uint32_t old = atomicMin(&P.vs_u[vtx[k]].x, val[k]);
                     if (val[k] < old) {
                         acc.upd++;
                         if (k == 3) changed3 = true;
                         acc.sig += signal_vertex(bnxt, vtx[k]);
+                        acc.vmin = min(acc.vmin, val[k]);
                     }
                 }
             }
             // the carry into the next window is live if the path continues and its
             // last vertex changed now or was signalled (its out-edge must be relaxed)
             carry = __shfl_sync(0xffffffffu, cur, 31);
+            carry_vtx = __shfl_sync(0xffffffffu, vtx[3], 31);
             carry_live = __shfl_sync(0xffffffffu, !tl[3] && (changed3 || act_c[3]), 31);
         } else {
             carry = INF;
@@ -628,7 +656,7 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
                 const unsigned long long p = fx_from(pin[k]);
                 if (p) {
                     if (vtx[k] < px.H) px_add(&px.acc[2 * vtx[k]], p);  // proxy: shared-memory atomics
-                    else atomicAdd(&P.vs_t[vtx[k]], p);                 // master: REDG (no return)
+                    else red_add_u64_h(&P.vs_t[vtx[k]], p, pol_keep);   // master: REDG (no return)
                     acc.upd++;
                 }
                 if (!tl[k] && (pend[k] | p)) { sv_c[k] += pend[k] + p; dirty = true; }
@@ -773,7 +801,14 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
     cg::grid_group grid = cg::this_grid();
     const int lane = threadIdx.x & 31;
     constexpr bool kAccum = ALGO == DG_PAGERANK || ALGO == DG_ADSORPTION;
-    const unsigned long long pol_stream = policy_evict_first(), pol_keep = policy_evict_last();
+    const unsigned long long pol_stream = policy_evict_first();
+    unsigned long long pol_keep = policy_evict_last();
+    if (kAccum) {  // masters: hot prefix evict-last (at most kHotMasterBytes), the rest unchanged
+        const uint64_t tot = (uint64_t)(P.n + 2) * 8;
+        const uint32_t total = (uint32_t)(tot < 0xFFFFFF00ull ? tot : 0xFFFFFF00ull);
+        const uint32_t hot = (uint32_t)(P.hot_master_bytes < total ? P.hot_master_bytes : total);
+        pol_keep = policy_masters(P.vs_t, hot, total);
+    }
     extern __shared__ __align__(16) unsigned char dyn_smem[];
     __shared__ int s_done;
     Proxies px{nullptr, nullptr, 0};
@@ -811,10 +846,13 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             accum_sweep(P, acc.sig);
         } else {
             unsigned* ticket = &P.ctr->ticket[cur];
-            if (ALGO == DG_SSSP) walk_minplus<0>(P, ticket, bcur, bnxt, acc);
-            else if (ALGO == DG_BFS) walk_minplus<1>(P, ticket, bcur, bnxt, acc);
-            else if (ALGO == DG_WCC) walk_minplus<2>(P, ticket, bcur, bnxt, acc);
-            else if (ALGO == 100) walk_minplus<3>(P, ticket, bcur, bnxt, acc);
+            // bucket bound of this round (reading R-DELTA): only distances <= theta are committed
+            const uint32_t theta = ((ALGO == DG_SSSP || ALGO == DG_BFS) && P.delta)
+                                       ? sat_add(*(volatile unsigned*)&P.ctr->minval[cur], P.delta) : INF;
+            if (ALGO == DG_SSSP) walk_minplus<0>(P, ticket, bcur, bnxt, theta, acc);
+            else if (ALGO == DG_BFS) walk_minplus<1>(P, ticket, bcur, bnxt, theta, acc);
+            else if (ALGO == DG_WCC) walk_minplus<2>(P, ticket, bcur, bnxt, INF, acc);
+            else if (ALGO == 100) walk_minplus<3>(P, ticket, bcur, bnxt, INF, acc);
             else if (ALGO == 101) {
                 while (true) {
                     unsigned t = 0;
@@ -830,6 +868,12 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
         for (int off = 16; off; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
         if (lane == 0 && s) atomicAdd(&P.ctr->active[nxt], s);
         acc.sig = 0;
+        if ((ALGO == DG_SSSP || ALGO == DG_BFS) && P.delta) {
+            uint32_t mv = acc.vmin;
+            for (int off = 16; off; off >>= 1) mv = min(mv, __shfl_xor_sync(0xffffffffu, mv, off));
+            if (lane == 0 && mv != INF) atomicMin(&P.ctr->minval[nxt], mv);
+            acc.vmin = INF;
+        }
         grid.sync();
         if (!kAccum) {  // retire this round's bitmap for reuse two rounds later
             uint32_t* bc = P.bits + (int64_t)cur * P.nw;
@@ -837,7 +881,15 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
                  i += (int64_t)gridDim.x * blockDim.x)
                 bc[i] = 0u;
         }
-        if (blockIdx.x == 0 && threadIdx.x == 0) { P.ctr->active[cur] = 0; P.ctr->ticket[cur] = 0; }
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            // a round whose pending relaxations were all beyond the bucket keeps the
+            // bucket base; otherwise the next bucket starts at the smallest new distance
+            if ((ALGO == DG_SSSP || ALGO == DG_BFS) && P.ctr->minval[nxt] == INF)
+                P.ctr->minval[nxt] = P.ctr->minval[cur] == INF ? INF : P.ctr->minval[cur] + P.delta;
+            P.ctr->active[cur] = 0;
+            P.ctr->ticket[cur] = 0;
+            P.ctr->minval[cur] = INF;
+        }
         grid.sync();
     }
     unsigned long long su = acc.upd, se = acc.edges, sn = acc.entries;
@@ -1289,6 +1341,10 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
     {
         const char* e = std::getenv("DG_PROXY_REFRESH");  // developer knob
         P.px_refresh = e ? std::atoi(e) : DG_PROXY_REFRESH;
+        const char* dl = std::getenv("DG_DELTA");  // bucket width knob; default: reading R-DELTA
+        P.delta = dl ? (uint32_t)std::atoi(dl) : (uint32_t)S.delta;
+        const char* hm = std::getenv("DG_HOT_MASTER_MB");  // developer knob (default 64 MB)
+        P.hot_master_bytes = (uint64_t)(hm ? std::atof(hm) : 64.0) * (1ull << 20);
         const char* o = std::getenv("DG_PART_ORDER");
         P.part_order = o ? std::atoi(o) : 0;
         if (P.part_order > 1) {  // keep the map a permutation
@@ -1330,9 +1386,11 @@ int init_states(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
         return write_counters(W, c, err);
     }
     CK(cudaMemsetAsync(W->bits, 0, sizeof(uint32_t) * 2 * W->nw));
+    c.minval[0] = c.minval[1] = INF;
     if (algo == DG_SSSP || algo == DG_BFS) {
         init_u_kernel<<<g, 256>>>(W->vs_u, D.orig, D.n, algo, S.source);
         bits_set_one_kernel<<<1, 1>>>(W->bits, S.source);
+        c.minval[0] = 0;  // round 0's bucket starts at the source's distance
         c.active[0] = 1;
         S.stats.kernel_launches += 2;
     } else {

@@ -92,10 +92,18 @@ class DiGraph:
         check(self._L.dg_set_vertex_params(self._h, *[_p(x) for x in a]), "dg_set_vertex_params")
 
     # -- dg_run / dg_get_states ----------------------------------------------
+    @staticmethod
+    def _param(algo, damping, delta):
+        """dg_run's `param`: PageRank damping; SSSP/BFS bucket width (None: library
+        default, 0: unbounded, k > 0: k; include/digraph.h, DESIGN.md R-DELTA)."""
+        if algo in ("sssp", "bfs"):
+            return 0.0 if delta is None else (-1.0 if delta == 0 else float(delta))
+        return float(damping)
+
     def run(self, algo, source=0, epsilon=1e-7, damping=0.85, mode="path", max_rounds=0,
-            allow_noconv=False):
+            allow_noconv=False, delta=None):
         st = _abi.dg_run_stats()
-        rc = self._L.dg_run(self._h, ALGOS[algo], int(source), float(epsilon), float(damping),
+        rc = self._L.dg_run(self._h, ALGOS[algo], int(source), float(epsilon), self._param(algo, damping, delta),
                             MODES[mode], int(max_rounds), ctypes.byref(st))
         if rc != 0 and not (allow_noconv and rc == -4):
             check(rc, "dg_run")
@@ -142,9 +150,9 @@ class DiGraph:
         check(self._L.dg_boundary_vertices(self._h, _p(out)), "dg_boundary_vertices")
         return out[: nb.value]
 
-    def run_begin(self, algo, source=0, epsilon=1e-7, damping=0.85):
-        check(self._L.dg_run_begin(self._h, ALGOS[algo], int(source), float(epsilon), float(damping)),
-              "dg_run_begin")
+    def run_begin(self, algo, source=0, epsilon=1e-7, damping=0.85, delta=None):
+        check(self._L.dg_run_begin(self._h, ALGOS[algo], int(source), float(epsilon),
+                                   self._param(algo, damping, delta)), "dg_run_begin")
         self.algo = algo
 
     def rounds(self, max_rounds):

@@ -93,3 +93,46 @@ def test_upload_moves_only_what_the_algorithm_reads(graph):
     assert dg.layout_info()["h2d_bytes"] == base + 4 * M + 8 * (n + 1) + 8 * g.m
     dg.upload()                                                    # a new upload starts over
     assert dg.layout_info()["h2d_bytes"] == base
+
+
+@pytest.mark.parametrize("delta", [None, 0, 1, 37, 255, 100000])
+def test_sssp_exact_for_every_bucket_width(graph, delta):
+    # reading R-DELTA: the bucket width trades redundant updates for rounds;
+    # the distances are exact for every width (None = library default 2*w_max,
+    # 0 = unbounded)
+    g = graph
+    dg = DiGraph()
+    dg.load_graph(g)
+    dg.build_paths()
+    src, dst, w = g.edges()
+    exp = OA.sssp_bellman_ford(g.n, src, dst, w, 5)[0]
+    st = dg.run("sssp", source=5, delta=delta)
+    assert np.array_equal(dg.get_states().astype(np.int64), exp)
+    assert st["converged"]
+
+
+def test_bfs_unit_buckets_are_level_synchronous(graph):
+    # with Delta = 1 a BFS round commits exactly one level: every reachable
+    # vertex but the source is updated once, like the level-synchronous ablation
+    g = graph
+    dg = DiGraph()
+    dg.load_graph(g)
+    dg.build_paths()
+    src, dst, _ = g.edges()
+    exp = OA.bfs_levels(g.n, src, dst, 0)
+    st = dg.run("bfs", source=0, delta=1)
+    assert np.array_equal(dg.get_states().astype(np.int64), exp)
+    reached = int((exp < OA.UNREACHED).sum())
+    assert st["vertex_updates"] == reached - 1
+    sv = dg.run("bfs", source=0, mode="vertex")
+    assert sv["vertex_updates"] == st["vertex_updates"]
+
+
+def test_default_bucket_width_cuts_sssp_updates(graph):
+    g = graph
+    dg = DiGraph()
+    dg.load_graph(g)
+    dg.build_paths()
+    st_def = dg.run("sssp", source=0)
+    st_unb = dg.run("sssp", source=0, delta=0)
+    assert st_def["vertex_updates"] <= st_unb["vertex_updates"]
