@@ -68,7 +68,8 @@ struct Counters {
 };
 
 struct DevWork {
-    uint2* vs_u = nullptr;                 // {value, stamp}: SSSP/BFS dist, WCC/SCC label
+    uint32_t* vs_u = nullptr;              // SSSP/BFS dist, WCC/SCC label (4 B: twice the masters per L2 sector)
+    uint32_t* vstamp = nullptr;            // vertex-centric ablation: round a vertex was last queued
     float4* vs_f = nullptr;                // vertex-centric ablation: {r, g, delta, stamp}
     unsigned long long* vs_t = nullptr;    // path-mode PR / Adsorption masters: exact fixed-point totals T
     unsigned long long* sigma = nullptr;   // T at the vertex's last signal
@@ -99,7 +100,8 @@ struct KParams {
     const int32_t* col;
     const int32_t* w;
     int64_t n_part, n, nw;
-    uint2* vs_u;
+    uint32_t* vs_u;
+    uint32_t* vstamp;
     float4* vs_f;
     unsigned long long* vs_t;
     unsigned long long* sigma;
@@ -302,7 +304,7 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
 #pragma unroll
             for (int k = 0; k < 4; k++) {
                 const uint32_t i = w.base + 4 * lane + k;
-                a[k] = (i >= w.beg && i < w.end) ? P.vs_u[u4get(code, k) & kVMask].x : INF;
+                a[k] = (i >= w.beg && i < w.end) ? P.vs_u[u4get(code, k) & kVMask] : INF;
             }
         }
         return any;
@@ -339,7 +341,7 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
                 const uint32_t nx_code = P.e_idx[inx];
                 if (!(nx_code & kHead)) {
                     nx_act = test_bit(bcur, nx_code & kVMask);
-                    nx_lab = P.vs_u[nx_code & kVMask].x;
+                    nx_lab = P.vs_u[nx_code & kVMask];
                 }
             }
         }
@@ -351,7 +353,7 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
 #pragma unroll
                 for (int k = 0; k < 4; k++) {
                     const uint32_t i = i0 + k;
-                    a_c[k] = (i >= wc.beg && i < wc.end) ? P.vs_u[u4get(code_c, k) & kVMask].x : INF;
+                    a_c[k] = (i >= wc.beg && i < wc.end) ? P.vs_u[u4get(code_c, k) & kVMask] : INF;
                 }
             }
             int4 wv = make_int4(0, 0, 0, 0);
@@ -433,7 +435,7 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
                         acc.sig += signal_vertex(bnxt, k ? vtx[k - 1] : pred0);
                         continue;
                     }
-                    const uint32_t old = atomicMin(&P.vs_u[vtx[k]].x, val[k]);
+                    const uint32_t old = atomicMin(&P.vs_u[vtx[k]], val[k]);
                     if (val[k] < old) {
                         acc.upd++;
                         if (k == 3) changed3 = true;
@@ -739,7 +741,7 @@ __device__ void walk_scc_bwd(const KParams& P, int64_t beg, int64_t end, const u
             const uint32_t c = u4get(code, k);
             live[k] = valid[k] && P.scc_label[vtx[k]] < 0;
             tl[k] = !live[k] || (c & kTail);
-            col[k] = live[k] ? P.vs_u[vtx[k]].x : INF;
+            col[k] = live[k] ? P.vs_u[vtx[k]] : INF;
             mk[k] = live[k] && P.mark[vtx[k]];
         }
         // element k on the successor's mark x:  m_k = mk_k | (x & eq_k),
@@ -949,7 +951,7 @@ __global__ void __launch_bounds__(kBlock) vertex_kernel(KParams P) {
                     s_push[wid][lane] = d * s->y;
                     if (!(d > 0.f)) deg = 0;
                 } else {
-                    s_dist[wid][lane] = P.vs_u[v].x;
+                    s_dist[wid][lane] = P.vs_u[v];
                 }
             }
             s_v[wid][lane] = v;
@@ -980,13 +982,13 @@ __global__ void __launch_bounds__(kBlock) vertex_kernel(KParams P) {
                     push = old < P.eps && old + a >= P.eps;
                 } else {
                     uint32_t cand = sat_add(s_dist[wid][lo], ALGO == DG_BFS ? 1u : (uint32_t)P.w[e]);
-                    if (cand < P.vs_u[x].x) {
-                        uint32_t old = atomicMin(&P.vs_u[x].x, cand);
+                    if (cand < P.vs_u[x]) {
+                        uint32_t old = atomicMin(&P.vs_u[x], cand);
                         if (cand < old) { acc.upd++; push = true; }
                     }
                 }
                 if (push) {
-                    unsigned* stp = ALGO == DG_PAGERANK ? reinterpret_cast<unsigned*>(&P.vs_f[x].w) : &P.vs_u[x].y;
+                    unsigned* stp = ALGO == DG_PAGERANK ? reinterpret_cast<unsigned*>(&P.vs_f[x].w) : &P.vstamp[x];
                     if (atomicExch(stp, (unsigned)(round + 1)) != (unsigned)(round + 1)) {
                         unsigned slot = atomicAdd(&P.ctr->active[nxt], 1u);
                         out[slot] = x;
@@ -1020,10 +1022,11 @@ __global__ void __launch_bounds__(kBlock) vertex_kernel(KParams P) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < (n); i += (int64_t)gridDim.x * blockDim.x)
 
 // WCC labels start as the ORIGINAL vertex id (reading R-CC: smallest original id wins)
-__global__ void init_u_kernel(uint2* vs, const int32_t* orig, int64_t n, int algo, int64_t source) {
+__global__ void init_u_kernel(uint32_t* vs, uint32_t* stamp, const int32_t* orig, int64_t n, int algo,
+                              int64_t source) {
     GRID_STRIDE(v, n) {
-        uint32_t val = (algo == DG_WCC) ? (uint32_t)orig[v] : (v == source ? 0u : INF);
-        vs[v] = make_uint2(val, 0u);
+        vs[v] = (algo == DG_WCC) ? (uint32_t)orig[v] : (v == source ? 0u : INF);
+        stamp[v] = 0u;
     }
 }
 // vertex-centric ablation: {r, g, delta, stamp} = {0, d/outdeg, 1-d, 0}
@@ -1100,8 +1103,8 @@ __global__ void out_pr_kernel(const float4* vf, const unsigned long long* va, co
     const double inv = normalize ? 1.0 / *sum : 1.0;
     GRID_STRIDE(v, n) out[v] = (float)(final_value(vf, va, new_id[v]) * inv);
 }
-__global__ void out_u_kernel(const uint2* vs, const int32_t* new_id, int64_t n, uint32_t* out) {
-    GRID_STRIDE(v, n) out[v] = vs[new_id[v]].x;
+__global__ void out_u_kernel(const uint32_t* vs, const int32_t* new_id, int64_t n, uint32_t* out) {
+    GRID_STRIDE(v, n) out[v] = vs[new_id[v]];
 }
 __global__ void out_i_kernel(const int32_t* x, const int32_t* new_id, int64_t n, int32_t* out) {
     GRID_STRIDE(v, n) out[v] = x[new_id[v]];
@@ -1119,29 +1122,29 @@ __global__ void scale_f_kernel(float* x, int64_t n, const double* sum) {
 
 // ---- SCC helpers
 // colours are ORIGINAL vertex ids so an SCC's label is its smallest original id
-__global__ void scc_init_kernel(uint2* vs, const int32_t* label, const int32_t* orig, uint8_t* mark, int64_t n) {
+__global__ void scc_init_kernel(uint32_t* vs, const int32_t* label, const int32_t* orig, uint8_t* mark, int64_t n) {
     GRID_STRIDE(v, n) {
-        vs[v] = make_uint2(label[v] < 0 ? (uint32_t)orig[v] : INF, 0u);
+        vs[v] = label[v] < 0 ? (uint32_t)orig[v] : INF;
         mark[v] = 0;
     }
 }
 // roots keep their own id as colour; they seed the backward phase's bitmap
-__global__ void scc_roots_kernel(const uint2* vs, const int32_t* label, const int32_t* orig, uint8_t* mark,
+__global__ void scc_roots_kernel(const uint32_t* vs, const int32_t* label, const int32_t* orig, uint8_t* mark,
                                  int64_t n, uint32_t* b, Counters* ctr) {
     unsigned cnt = 0;
     GRID_STRIDE(v, n) {
-        const bool root = label[v] < 0 && vs[v].x == (uint32_t)orig[v];
+        const bool root = label[v] < 0 && vs[v] == (uint32_t)orig[v];
         mark[v] = root;
         if (root) cnt += signal_vertex(b, (uint32_t)v);
     }
     for (int off = 16; off; off >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, off);
     if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(&ctr->active[0], cnt);
 }
-__global__ void scc_assign_kernel(const uint2* vs, int32_t* label, const uint8_t* mark, int64_t n, int32_t* remaining) {
+__global__ void scc_assign_kernel(const uint32_t* vs, int32_t* label, const uint8_t* mark, int64_t n, int32_t* remaining) {
     int cnt = 0;
     GRID_STRIDE(v, n) {
         if (label[v] < 0) {
-            if (mark[v]) label[v] = (int32_t)vs[v].x;
+            if (mark[v]) label[v] = (int32_t)vs[v];
             else cnt++;
         }
     }
@@ -1151,16 +1154,16 @@ __global__ void scc_assign_kernel(const uint2* vs, int32_t* label, const uint8_t
 
 // ---- multi-GPU boundary exchange ("each mirror always
 // sends its new state to its master"; line 96: synchronisation in batches)
-__global__ void pack_min_kernel(const uint2* vs, const int32_t* bnd, int64_t nb, uint32_t* buf) {
-    GRID_STRIDE(k, nb) buf[k] = vs[bnd[k]].x;
+__global__ void pack_min_kernel(const uint32_t* vs, const int32_t* bnd, int64_t nb, uint32_t* buf) {
+    GRID_STRIDE(k, nb) buf[k] = vs[bnd[k]];
 }
-__global__ void unpack_min_kernel(uint2* vs, const int32_t* bnd, int64_t nb, const uint32_t* buf, uint32_t* b,
+__global__ void unpack_min_kernel(uint32_t* vs, const int32_t* bnd, int64_t nb, const uint32_t* buf, uint32_t* b,
                                   Counters* ctr, int slot) {
     unsigned cnt = 0;
     GRID_STRIDE(k, nb) {
         const int v = bnd[k];
-        if (buf[k] < vs[v].x) {
-            vs[v].x = buf[k];
+        if (buf[k] < vs[v]) {
+            vs[v] = buf[k];
             cnt += signal_vertex(b, (uint32_t)v);
         }
     }
@@ -1245,7 +1248,7 @@ KParams make_params(const DevLayout& D, DevWork* W) {
     P.e_idx = D.e_idx; P.e_w = D.e_w; P.part_off = D.part_off;
     P.row_ptr = D.row_ptr; P.col = D.col; P.w = D.w;
     P.n_part = D.n_part; P.n = D.n; P.nw = W->nw;
-    P.vs_u = W->vs_u; P.vs_f = W->vs_f; P.vs_t = W->vs_t; P.sigma = W->sigma; P.s_val = W->s_val;
+    P.vs_u = W->vs_u; P.vstamp = W->vstamp; P.vs_f = W->vs_f; P.vs_t = W->vs_t; P.sigma = W->sigma; P.s_val = W->s_val;
     P.e_coef = W->e_coef; P.bits = W->bits;
     P.vlist0 = W->vlist[0]; P.vlist1 = W->vlist[1];
     P.ctr = W->ctr;
@@ -1261,6 +1264,7 @@ int ensure_work(DevWork*& W, const DevLayout& D, std::string& err) {
     int rc;
     W->nw = (D.n + 31) / 32 + 1;
     if ((rc = dalloc(&W->vs_u, D.n + 1, bytes, err))) return rc;
+    if ((rc = dalloc(&W->vstamp, D.n + 1, bytes, err))) return rc;
     if ((rc = dalloc(&W->vs_f, D.n + 1, bytes, err))) return rc;
     if ((rc = dalloc(&W->vs_t, D.n + 2, bytes, err))) return rc;
     if ((rc = dalloc(&W->sigma, D.n + 1, bytes, err))) return rc;
@@ -1376,7 +1380,7 @@ int init_states(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
             c.active[0] = (unsigned)D.n;
             S.stats.kernel_launches += 2;
         } else {
-            init_u_kernel<<<g, 256>>>(W->vs_u, D.orig, D.n, algo, S.source);
+            init_u_kernel<<<g, 256>>>(W->vs_u, W->vstamp, D.orig, D.n, algo, S.source);
             int32_t s = (int32_t)S.source;
             CK(cudaMemcpy(W->vlist[0], &s, sizeof(int32_t), cudaMemcpyHostToDevice));
             c.active[0] = 1;
@@ -1388,14 +1392,14 @@ int init_states(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
     CK(cudaMemsetAsync(W->bits, 0, sizeof(uint32_t) * 2 * W->nw));
     c.minval[0] = c.minval[1] = INF;
     if (algo == DG_SSSP || algo == DG_BFS) {
-        init_u_kernel<<<g, 256>>>(W->vs_u, D.orig, D.n, algo, S.source);
+        init_u_kernel<<<g, 256>>>(W->vs_u, W->vstamp, D.orig, D.n, algo, S.source);
         bits_set_one_kernel<<<1, 1>>>(W->bits, S.source);
         c.minval[0] = 0;  // round 0's bucket starts at the source's distance
         c.active[0] = 1;
         S.stats.kernel_launches += 2;
     } else {
         if (algo == DG_WCC) {
-            init_u_kernel<<<g, 256>>>(W->vs_u, D.orig, D.n, algo, 0);
+            init_u_kernel<<<g, 256>>>(W->vs_u, W->vstamp, D.orig, D.n, algo, 0);
         } else {
             init_acc_kernel<<<g, 256>>>(W->vs_t, W->sigma, algo == DG_ADSORPTION ? W->ads_base : nullptr, D.n,
                                         (float)S.param);
@@ -1599,7 +1603,7 @@ void dev_free_layout(DevLayout& D, bool csr_too) {
 
 void dev_free_work(DevWork*& W) {
     if (!W) return;
-    dfree(W->vs_u); dfree(W->vs_f); dfree(W->vs_t); dfree(W->sigma); dfree(W->s_val); dfree(W->bnd_base);
+    dfree(W->vs_u); dfree(W->vstamp); dfree(W->vs_f); dfree(W->vs_t); dfree(W->sigma); dfree(W->s_val); dfree(W->bnd_base);
     dfree(W->e_coef); dfree(W->pr_coef); dfree(W->ads_base); dfree(W->bits); dfree(W->vlist[0]); dfree(W->vlist[1]);
     dfree(W->ctr); dfree(W->dsum); dfree(W->scc_label); dfree(W->scc_mark); dfree(W->remaining); dfree(W->out_stage);
     if (W->ev0) cudaEventDestroy(W->ev0);
