@@ -23,6 +23,7 @@
 // the run ends when a round signals no vertex (device-side active counter,
 // north_star (4)).
 #include <cooperative_groups.h>
+#include <cub/device/device_scan.cuh>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -63,6 +64,9 @@ struct Counters {
     unsigned int active[2];  // path mode: vertices signalled into bitmap[k]; vertex mode: frontier sizes
     unsigned int ticket[2];
     unsigned int minval[2];  // SSSP/BFS: smallest distance signalled into bitmap[k] (bucket base of its round)
+    unsigned int qn[2];      // SSSP/BFS sparse rounds: length of the round's compacted frontier list
+    unsigned int osum[2];    // ... and the occurrences (out-edges) of its vertices
+    unsigned int qcur[2];    // append cursor of the list
     int round;  // global round number of the next round
     int pad;
 };
@@ -88,6 +92,10 @@ struct DevWork {
     uint8_t* scc_mark = nullptr;
     int32_t* remaining = nullptr;
     uint32_t* out_stage = nullptr;         // dg_get_states staging buffer (n words)
+    uint32_t* occ_off = nullptr;           // vertex -> its non-tail path entries (sparse rounds), n+1
+    uint32_t* occ = nullptr;               // entry indices grouped by vertex
+    uint2* occ_items = nullptr;            // frontier items (v, chunk of <= kOccChunk occurrences)
+    bool occ_ok = false;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr, kev0 = nullptr, kev1 = nullptr;
     bool have_params = false;
 };
@@ -122,6 +130,12 @@ struct KParams {
     int part_order;  // 0: priority order; 1: reversed; k > 1: t -> t*k mod n_part (k coprime to n_part)
     uint64_t hot_master_bytes;  // evict-last prefix of the accumulative masters
     uint32_t delta;  // SSSP/BFS bucket width (reading R-DELTA); 0 = unbounded
+    const uint32_t* occ_off;  // SSSP/BFS sparse rounds: occurrence index (null: dense rounds only)
+    const uint32_t* occ;
+    uint2* occ_items;         // the round's frontier items (v, chunk)
+    uint32_t sparse_max;      // rounds with at most this many signalled vertices are candidates (n/4)
+    uint32_t sparse_occ;      // ... and are walked sparse if their out-edges are at most this many
+    int sparse_walk;          // path edges a sparse walk follows at most
 };
 
 // ------------------------------------------------------------------ helpers
@@ -460,6 +474,157 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
         any_c = any_n;
 #pragma unroll
         for (int k = 0; k < 4; k++) { act_c[k] = act_n[k]; a_c[k] = a_n[k]; }
+    }
+}
+
+// Sparse min-plus rounds (SSSP/BFS).  When few
+// vertices are signalled, probing every window's signal bits costs more than
+// the work: the round instead starts the path walks at the signalled vertices.
+// Every out-edge of v lies on exactly one path, right after one of v's
+// non-tail entries (the occurrence index), so walking forward from each
+// occurrence relaxes exactly v's out-edges -- and, as in the dense walk, a
+// vertex lowered on the way passes its new distance on along its path in the
+// same round (the vertices of a path are handled in
+// order and a new state is used immediately).  A walk stops at the path's
+// tail, at a vertex it does not improve (that vertex's own distance was, or
+// will be, propagated from its own signal), or at a relaxation beyond the
+// round's bucket (reading R-DELTA: the predecessor stays signalled).
+//
+// Walks are capped at P.sparse_walk path edges: every vertex a walk lowers is
+// signalled, so the walk's continuation is picked up in the next round; the
+// cap bounds a round's latency (merged paths reach ~1000 edges).
+//
+// Frontier list: the round's signal bitmap compacted with warp-aggregated
+// appends (one pass over n/32 words) into items (v, chunk) of at most
+// kOccChunk occurrences, so a hub's out-edges spread over many warps.
+constexpr uint32_t kOccChunk = 32;
+// Pass 1 (count): out-edges and items of the signalled vertices.
+__device__ void count_bits(const KParams& P, const uint32_t* bcur, unsigned* qn, unsigned* osum) {
+    const int64_t T = (int64_t)gridDim.x * blockDim.x;
+    unsigned c = 0, o = 0;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < P.nw; i += T) {
+        for (uint32_t x = bcur[i]; x; x &= x - 1) {
+            const uint32_t v = (uint32_t)(i * 32 + __ffs(x) - 1);
+            const uint32_t d = P.occ_off[v + 1] - P.occ_off[v];
+            c += (d + kOccChunk - 1) / kOccChunk;
+            o += d;
+        }
+    }
+    for (int off = 16; off; off >>= 1) {
+        c += __shfl_xor_sync(0xffffffffu, c, off);
+        o += __shfl_xor_sync(0xffffffffu, o, off);
+    }
+    if ((threadIdx.x & 31) == 0 && o) {
+        atomicAdd(qn, c);
+        atomicAdd(osum, o);
+    }
+}
+// Pass 2 (write): the items, appended warp by warp (order is irrelevant).
+__device__ void compact_bits(const KParams& P, const uint32_t* bcur, uint2* list, unsigned* cursor) {
+    const int lane = threadIdx.x & 31;
+    const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+    const int64_t gw = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    for (int64_t b = gw * 32; b < P.nw; b += warps * 32) {
+        const int64_t i = b + lane;
+        uint32_t w = i < P.nw ? bcur[i] : 0u;
+        unsigned c = 0;
+        for (uint32_t x = w; x; x &= x - 1) {
+            const uint32_t v = (uint32_t)(i * 32 + __ffs(x) - 1);
+            c += (P.occ_off[v + 1] - P.occ_off[v] + kOccChunk - 1) / kOccChunk;
+        }
+        unsigned inc = c;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const unsigned y = __shfl_up_sync(0xffffffffu, inc, off);
+            if (lane >= off) inc += y;
+        }
+        const unsigned tot = __shfl_sync(0xffffffffu, inc, 31);
+        if (tot == 0) continue;
+        unsigned base = 0;
+        if (lane == 31) base = atomicAdd(cursor, tot);
+        base = __shfl_sync(0xffffffffu, base, 31) + inc - c;
+        while (w) {
+            const uint32_t v = (uint32_t)(i * 32 + __ffs(w) - 1);
+            w &= w - 1;
+            const uint32_t nch = (P.occ_off[v + 1] - P.occ_off[v] + kOccChunk - 1) / kOccChunk;
+            for (uint32_t k = 0; k < nch; k++) list[base++] = make_uint2(v, k);
+        }
+    }
+}
+
+template <int MODE>
+__device__ void walk_sparse(const KParams& P, const uint2* list, unsigned qn, unsigned* ticket, uint32_t* bnxt,
+                            uint32_t theta, Acc& acc) {
+    __shared__ uint32_t s_off[kWarps][33];
+    __shared__ uint32_t s_beg[kWarps][32], s_x[kWarps][32], s_v[kWarps][32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    while (true) {
+        unsigned t = 0;
+        if (lane == 0) t = atomicAdd(ticket, 32u);
+        t = __shfl_sync(0xffffffffu, t, 0);
+        if (t >= qn) break;
+        uint32_t cnt = 0, beg = 0, x = INF, v = 0;
+        if (t + lane < qn) {
+            const uint2 it = list[t + lane];
+            v = it.x;
+            beg = P.occ_off[v] + it.y * kOccChunk;
+            cnt = min(P.occ_off[v + 1] - beg, kOccChunk);
+            x = P.vs_u[v];
+            acc.units++;
+        }
+        uint32_t inc = cnt;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, off);
+            if (lane >= off) inc += y;
+        }
+        s_off[wid][lane + 1] = inc;
+        if (lane == 0) s_off[wid][0] = 0;
+        s_beg[wid][lane] = beg;
+        s_x[wid][lane] = x;
+        s_v[wid][lane] = v;
+        __syncwarp();
+        const uint32_t total = s_off[wid][32];
+        for (uint32_t j = lane; j < total; j += 32) {
+            int lo = 0, hi = 31;  // owner: largest o with s_off[o] <= j
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (s_off[wid][mid] <= j) lo = mid; else hi = mid - 1;
+            }
+            uint32_t cur = s_x[wid][lo], pred = s_v[wid][lo];
+            uint32_t e = P.occ[s_beg[wid][lo] + (j - s_off[wid][lo])] + 1;  // the path edge out of the occurrence
+            // the next entry of the path is loaded one step ahead
+            uint32_t code = __ldg(P.e_idx + e);
+            uint32_t w = MODE == 0 ? (uint32_t)__ldg(P.e_w + e) : 1u;
+            for (int step = 0; step < P.sparse_walk; step++) {
+                const uint32_t u = code & kVMask;
+                const uint32_t cand = sat_add(cur, w);
+                const bool last = code & kTail;
+                acc.entries++;
+                acc.edges++;
+                if (cand > theta) {  // beyond the bucket: not committed, the predecessor stays signalled
+                    acc.sig += signal_vertex(bnxt, pred);
+                    break;
+                }
+                if (!last) {  // prefetch the path's next entry
+                    code = __ldg(P.e_idx + e + 1);
+                    if (MODE == 0) w = (uint32_t)__ldg(P.e_w + e + 1);
+                }
+                // read before the atomic: in-edges of hubs would otherwise
+                // serialise on one address
+                if (cand >= __ldcg(&P.vs_u[u])) break;
+                const uint32_t old = atomicMin(&P.vs_u[u], cand);
+                if (cand >= old) break;
+                acc.upd++;
+                acc.sig += signal_vertex(bnxt, u);
+                acc.vmin = min(acc.vmin, cand);
+                if (last) break;
+                cur = cand;
+                pred = u;
+                e++;
+            }
+        }
+        __syncwarp();
     }
 }
 
@@ -851,7 +1016,25 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             // bucket bound of this round (reading R-DELTA): only distances <= theta are committed
             const uint32_t theta = ((ALGO == DG_SSSP || ALGO == DG_BFS) && P.delta)
                                        ? sat_add(*(volatile unsigned*)&P.ctr->minval[cur], P.delta) : INF;
-            if (ALGO == DG_SSSP) walk_minplus<0>(P, ticket, bcur, bnxt, theta, acc);
+            // sparse round: when few vertices are
+            // signalled, compact them; walk from them if their out-edges are
+            // at most 1/sparse_div of the path entries, else walk the windows
+            bool sparse = false;
+            if ((ALGO == DG_SSSP || ALGO == DG_BFS) && P.occ_off &&
+                *((volatile unsigned*)&P.ctr->active[cur]) <= P.sparse_max) {
+                count_bits(P, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
+                grid.sync();
+                sparse = *((volatile unsigned*)&P.ctr->osum[cur]) <= P.sparse_occ;
+                if (sparse) {
+                    compact_bits(P, bcur, P.occ_items, &P.ctr->qcur[cur]);
+                    grid.sync();
+                }
+            }
+            if (sparse) {
+                const unsigned qn = *((volatile unsigned*)&P.ctr->qn[cur]);
+                if (ALGO == DG_SSSP) walk_sparse<0>(P, P.occ_items, qn, ticket, bnxt, theta, acc);
+                else walk_sparse<1>(P, P.occ_items, qn, ticket, bnxt, theta, acc);
+            } else if (ALGO == DG_SSSP) walk_minplus<0>(P, ticket, bcur, bnxt, theta, acc);
             else if (ALGO == DG_BFS) walk_minplus<1>(P, ticket, bcur, bnxt, theta, acc);
             else if (ALGO == DG_WCC) walk_minplus<2>(P, ticket, bcur, bnxt, INF, acc);
             else if (ALGO == 100) walk_minplus<3>(P, ticket, bcur, bnxt, INF, acc);
@@ -891,6 +1074,9 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             P.ctr->active[cur] = 0;
             P.ctr->ticket[cur] = 0;
             P.ctr->minval[cur] = INF;
+            P.ctr->qn[cur] = 0;
+            P.ctr->osum[cur] = 0;
+            P.ctr->qcur[cur] = 0;
         }
         grid.sync();
     }
@@ -1120,6 +1306,20 @@ __global__ void scale_f_kernel(float* x, int64_t n, const double* sum) {
     GRID_STRIDE(v, n) x[v] = (float)((double)x[v] * inv);
 }
 
+// ---- occurrence index (sparse min-plus rounds): vertex -> its non-tail entries
+__global__ void occ_count_kernel(const uint32_t* e_idx, int64_t M, uint32_t* cnt) {
+    GRID_STRIDE(i, M) {
+        const uint32_t c = e_idx[i];
+        if (!(c & kTail)) atomicAdd(&cnt[(c & kVMask) + 1], 1u);
+    }
+}
+__global__ void occ_fill_kernel(const uint32_t* e_idx, int64_t M, uint32_t* cursor, uint32_t* occ) {
+    GRID_STRIDE(i, M) {
+        const uint32_t c = e_idx[i];
+        if (!(c & kTail)) occ[atomicAdd(&cursor[c & kVMask], 1u)] = (uint32_t)i;
+    }
+}
+
 // ---- SCC helpers
 // colours are ORIGINAL vertex ids so an SCC's label is its smallest original id
 __global__ void scc_init_kernel(uint32_t* vs, const int32_t* label, const int32_t* orig, uint8_t* mark, int64_t n) {
@@ -1319,6 +1519,56 @@ int acc_minb() {
     return e ? std::atoi(e) : 2;
 }
 
+// Sparse min-plus rounds: a round with at most
+// n/4 signalled vertices whose out-edges are at most M / DG_SPARSE_DIV walks
+// from them; 0 disables.
+int64_t sparse_div() {
+    const char* e = std::getenv("DG_SPARSE_DIV");  // developer knob
+    return e ? std::atoll(e) : 16;
+}
+// Below this many path entries a dense round costs less than a sparse round's
+// two extra grid barriers and its dependent walk steps (measured: 1.1 M
+// entries lose, 56 M and 73 M win).
+int64_t sparse_min_entries() {
+    const char* e = std::getenv("DG_SPARSE_MIN_M");  // developer knob
+    return e ? std::atoll(e) : (int64_t)1 << 23;
+}
+
+// Occurrence index: counting sort of the non-tail entries by vertex (built on
+// the device on the first SSSP/BFS run after an upload).
+int ensure_occ(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
+    if (W->occ_ok) return DG_OK;
+    int64_t bytes = 0;
+    int rc;
+    uint32_t *cur = nullptr;
+    void* tmp = nullptr;
+    size_t tmp_bytes = 0;
+    if ((rc = dalloc(&W->occ_off, D.n + 1, bytes, err))) return rc;
+    if ((rc = dalloc(&cur, D.n + 1, bytes, err))) return rc;
+    CK(cudaMemsetAsync(W->occ_off, 0, sizeof(uint32_t) * (D.n + 1)));
+    occ_count_kernel<<<grid_1d(D.M), 256>>>(D.e_idx, D.M, W->occ_off);
+    CK(cub::DeviceScan::InclusiveSum(nullptr, tmp_bytes, W->occ_off, W->occ_off, (int)(D.n + 1)));
+    CK(cudaMalloc(&tmp, tmp_bytes ? tmp_bytes : 1));
+    CK(cub::DeviceScan::InclusiveSum(tmp, tmp_bytes, W->occ_off, W->occ_off, (int)(D.n + 1)));
+    uint32_t total = 0;
+    CK(cudaMemcpy(&total, W->occ_off + D.n, sizeof(uint32_t), cudaMemcpyDeviceToHost));
+    if ((rc = dalloc(&W->occ, (size_t)total + 1, bytes, err)) ||
+        (rc = dalloc(&W->occ_items, (size_t)(D.n + total / kOccChunk + 1), bytes, err))) {
+        cudaFree(cur);
+        cudaFree(tmp);
+        return rc;
+    }
+    CK(cudaMemcpyAsync(cur, W->occ_off, sizeof(uint32_t) * D.n, cudaMemcpyDeviceToDevice));
+    occ_fill_kernel<<<grid_1d(D.M), 256>>>(D.e_idx, D.M, cur, W->occ);
+    CK(cudaGetLastError());
+    CK(cudaDeviceSynchronize());
+    cudaFree(cur);
+    cudaFree(tmp);
+    S.stats.kernel_launches += 3;
+    W->occ_ok = true;
+    return DG_OK;
+}
+
 // Launch the persistent path kernel for at most `rounds` rounds.
 int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState& S, std::string& err) {
     KParams P = make_params(D, W);
@@ -1347,6 +1597,18 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
         P.px_refresh = e ? std::atoi(e) : DG_PROXY_REFRESH;
         const char* dl = std::getenv("DG_DELTA");  // bucket width knob; default: reading R-DELTA
         P.delta = dl ? (uint32_t)std::atoi(dl) : (uint32_t)S.delta;
+        const int64_t sd = sparse_div();
+        if ((algo_k == DG_SSSP || algo_k == DG_BFS) && sd > 0 && D.M >= sparse_min_entries()) {
+            int rc;
+            if ((rc = ensure_occ(W, D, S, err))) return rc;
+            P.occ_off = W->occ_off;
+            P.occ = W->occ;
+            P.occ_items = W->occ_items;
+            P.sparse_max = (uint32_t)std::min<int64_t>(D.n / 4, 0xFFFFFFFFll);
+            P.sparse_occ = (uint32_t)std::min<int64_t>(D.M / sd, 0xFFFFFFFFll);
+            const char* sw = std::getenv("DG_SPARSE_WALK");  // developer knob
+            P.sparse_walk = sw ? std::max(1, std::atoi(sw)) : 4;
+        }
         const char* hm = std::getenv("DG_HOT_MASTER_MB");  // developer knob (default 64 MB)
         P.hot_master_bytes = (uint64_t)(hm ? std::atof(hm) : 64.0) * (1ull << 20);
         const char* o = std::getenv("DG_PART_ORDER");
@@ -1606,6 +1868,7 @@ void dev_free_work(DevWork*& W) {
     dfree(W->vs_u); dfree(W->vstamp); dfree(W->vs_f); dfree(W->vs_t); dfree(W->sigma); dfree(W->s_val); dfree(W->bnd_base);
     dfree(W->e_coef); dfree(W->pr_coef); dfree(W->ads_base); dfree(W->bits); dfree(W->vlist[0]); dfree(W->vlist[1]);
     dfree(W->ctr); dfree(W->dsum); dfree(W->scc_label); dfree(W->scc_mark); dfree(W->remaining); dfree(W->out_stage);
+    dfree(W->occ_off); dfree(W->occ); dfree(W->occ_items);
     if (W->ev0) cudaEventDestroy(W->ev0);
     if (W->ev1) cudaEventDestroy(W->ev1);
     if (W->kev0) cudaEventDestroy(W->kev0);
@@ -1615,7 +1878,10 @@ void dev_free_work(DevWork*& W) {
 }
 
 void dev_layout_changed(DevWork* W) {
-    if (W) W->pr_coef_d = -1.0;
+    if (!W) return;
+    W->pr_coef_d = -1.0;
+    dfree(W->occ_off); dfree(W->occ); dfree(W->occ_items);
+    W->occ_ok = false;
 }
 
 int dev_set_vertex_params(DevWork*& W, const DevLayout& D, const double* p_inj, const double* p_cont,

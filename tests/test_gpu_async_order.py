@@ -136,3 +136,43 @@ def test_default_bucket_width_cuts_sssp_updates(graph):
     st_def = dg.run("sssp", source=0)
     st_unb = dg.run("sssp", source=0, delta=0)
     assert st_def["vertex_updates"] <= st_unb["vertex_updates"]
+
+
+@pytest.fixture(params=["0", "1", "16"])
+def sparse_div(request):
+    # DG_SPARSE_DIV: 0 = dense rounds only; k > 0 = a round with at most n/4
+    # signalled vertices whose out-edges are at most M/k walks from them (1:
+    # every such round, 16: the library default)
+    # (DG_SPARSE_MIN_M = 0: also on these small graphs)
+    old = {k: os.environ.get(k) for k in ("DG_SPARSE_DIV", "DG_SPARSE_MIN_M")}
+    os.environ["DG_SPARSE_DIV"] = request.param
+    os.environ["DG_SPARSE_MIN_M"] = "0"
+    yield request.param
+    for k, v in old.items():
+        if v is None:
+            del os.environ[k]
+        else:
+            os.environ[k] = v
+
+
+@pytest.mark.parametrize("gname", ["rmat", "chains", "uniform_dup"])
+@pytest.mark.parametrize("delta", [None, 1, 0])
+def test_min_plus_exact_in_sparse_and_dense_rounds(graph, sparse_div, gname, delta):
+    # walking from the signalled vertices through the
+    # occurrence index relaxes the same edges as the window walk, so SSSP and
+    # BFS stay bit-exact whichever kind of round runs, for every bucket width
+    g = {"rmat": graph,
+         "chains": inputs.chains(20000, 26000, chain_len=700, seed=13),
+         "uniform_dup": inputs.uniform(3000, 9000, seed=12, dedupe=False, drop_self=False)}[gname]
+    dg = DiGraph()
+    dg.load_graph(g)
+    dg.build_paths()
+    src, dst, w = g.edges()
+    st = dg.run("sssp", source=0, delta=delta)
+    assert np.array_equal(dg.get_states().astype(np.int64), OA.sssp_bellman_ford(g.n, src, dst, w, 0)[0])
+    assert st["converged"]
+    st = dg.run("bfs", source=0, delta=delta)
+    exp = OA.bfs_levels(g.n, src, dst, 0)
+    assert np.array_equal(dg.get_states().astype(np.int64), exp)
+    if delta == 1:  # level-synchronous in either kind of round
+        assert st["vertex_updates"] == int((exp < OA.UNREACHED).sum()) - 1
