@@ -95,6 +95,13 @@ struct DevWork {
     uint32_t* occ_off = nullptr;           // vertex -> its non-tail path entries (sparse rounds), n+1
     uint32_t* occ = nullptr;               // entry indices grouped by vertex
     uint2* occ_items = nullptr;            // frontier items (v, chunk of <= kOccChunk occurrences)
+    uint32_t* iocc_off = nullptr;          // vertex -> its non-head path entries (SCC backward), n+1
+    uint32_t* iocc = nullptr;
+    bool iocc_ok = false;
+    int64_t occ_cap = 0, iocc_cap = 0;     // allocated lengths of occ / iocc
+    uint32_t* occ_cur = nullptr;           // index build scratch
+    void* cub_tmp = nullptr;
+    size_t cub_tmp_bytes = 0;
     bool occ_ok = false;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr, kev0 = nullptr, kev1 = nullptr;
     bool have_params = false;
@@ -595,10 +602,11 @@ __device__ void walk_sparse(const KParams& P, const uint2* list, unsigned qn, un
             uint32_t e = P.occ[s_beg[wid][lo] + (j - s_off[wid][lo])] + 1;  // the path edge out of the occurrence
             // the next entry of the path is loaded one step ahead
             uint32_t code = __ldg(P.e_idx + e);
-            uint32_t w = MODE == 0 ? (uint32_t)__ldg(P.e_w + e) : 1u;
+            uint32_t w = MODE == 0 ? (uint32_t)__ldg(P.e_w + e) : (MODE == 1 ? 1u : 0u);
             for (int step = 0; step < P.sparse_walk; step++) {
                 const uint32_t u = code & kVMask;
-                const uint32_t cand = sat_add(cur, w);
+                if (MODE == 3 && P.scc_label[u] >= 0) break;  // assigned vertices break their paths
+                const uint32_t cand = MODE == 3 ? cur : sat_add(cur, w);
                 const bool last = code & kTail;
                 acc.entries++;
                 acc.edges++;
@@ -622,6 +630,67 @@ __device__ void walk_sparse(const KParams& P, const uint2* list, unsigned qn, un
                 cur = cand;
                 pred = u;
                 e++;
+            }
+        }
+        __syncwarp();
+    }
+}
+
+// Sparse backward rounds of the SCC reachability phase: from each marked
+// vertex v, walk its in-edges backwards (P.occ_off/P.occ hold the non-head
+// entries here: the path edge INTO entry i comes from entry i-1) and mark
+// unassigned predecessors of v's colour, passing the mark on along the path.
+__device__ void walk_sparse_bwd(const KParams& P, const uint2* list, unsigned qn, unsigned* ticket, uint32_t* bnxt,
+                                Acc& acc) {
+    __shared__ uint32_t s_off[kWarps][33];
+    __shared__ uint32_t s_beg[kWarps][32], s_x[kWarps][32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    while (true) {
+        unsigned t = 0;
+        if (lane == 0) t = atomicAdd(ticket, 32u);
+        t = __shfl_sync(0xffffffffu, t, 0);
+        if (t >= qn) break;
+        uint32_t cnt = 0, beg = 0, col = INF;
+        if (t + lane < qn) {
+            const uint2 it = list[t + lane];
+            beg = P.occ_off[it.x] + it.y * kOccChunk;
+            cnt = min(P.occ_off[it.x + 1] - beg, kOccChunk);
+            col = P.vs_u[it.x];
+            acc.units++;
+        }
+        uint32_t inc = cnt;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, off);
+            if (lane >= off) inc += y;
+        }
+        s_off[wid][lane + 1] = inc;
+        if (lane == 0) s_off[wid][0] = 0;
+        s_beg[wid][lane] = beg;
+        s_x[wid][lane] = col;
+        __syncwarp();
+        const uint32_t total = s_off[wid][32];
+        for (uint32_t j = lane; j < total; j += 32) {
+            int lo = 0, hi = 31;
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (s_off[wid][mid] <= j) lo = mid; else hi = mid - 1;
+            }
+            const uint32_t c = s_x[wid][lo];
+            uint32_t e = P.occ[s_beg[wid][lo] + (j - s_off[wid][lo])] - 1;  // the path predecessor
+            for (int step = 0; step < P.sparse_walk; step++) {
+                const uint32_t code = __ldg(P.e_idx + e);
+                const uint32_t u = code & kVMask;
+                acc.entries++;
+                acc.edges++;
+                if (P.scc_label[u] >= 0 || P.vs_u[u] != c || P.mark[u]) break;
+                P.mark[u] = 1;  // idempotent byte store; the signal bit counts it once
+                if (signal_vertex(bnxt, u)) {
+                    acc.upd++;
+                    acc.sig++;
+                }
+                if (code & kHead) break;
+                e--;
             }
         }
         __syncwarp();
@@ -857,13 +926,99 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
 // End-of-round vertex sweep of the accumulative algorithms: a vertex whose
 // total grew by >= eps since its last signal counts as signalled for the next
 // round (the per-vertex stop rule at delta < eps; the device active counter).
-__device__ void accum_sweep(const KParams& P, unsigned& cnt) {
-    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < P.n; v += (int64_t)gridDim.x * blockDim.x) {
-        const unsigned long long T = __ldcg(&P.vs_t[v]);
-        if (T - P.sigma[v] >= P.eps_fx) {
-            P.sigma[v] = T;
-            cnt++;
+// The signalled vertices also form the next round's bitmap (whole words: a
+// warp sweeps 32 consecutive vertices), read by sparse rounds.
+__device__ void accum_sweep(const KParams& P, uint32_t* bnxt, unsigned& cnt) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v0 = blockIdx.x * (int64_t)blockDim.x; v0 < P.n; v0 += stride) {
+        const int64_t v = v0 + threadIdx.x;
+        bool sig = false;
+        if (v < P.n) {
+            const unsigned long long T = __ldcg(&P.vs_t[v]);
+            if (T - P.sigma[v] >= P.eps_fx) {
+                P.sigma[v] = T;
+                cnt++;
+                sig = true;
+            }
         }
+        const unsigned word = __ballot_sync(0xffffffffu, sig);
+        if ((threadIdx.x & 31) == 0 && v < P.n + 31) bnxt[v >> 5] = word;
+    }
+}
+
+// Sparse accumulative rounds (PageRank / Adsorption; DESIGN.md "Sparse
+// rounds").  From every non-tail entry i of a signalled vertex the walk
+// forwards pend_i (if >= eps) along the path edge out of i exactly as the
+// dense walk does, and passes the push on along the path: at entry e of
+// vertex x with incoming push p it reads T(x), adds p to T(x) (RED), forwards
+// c_e * (pend_e + p) and sets S_val[e] += pend_e + p.  Each entry has a single
+// owner in a round (as in the dense walk, where a warp owns a window): the
+// starter at a signalled vertex's entry, or the walk arriving from the path
+// predecessor when the entry's vertex is not signalled.  A walk arriving at a
+// signalled vertex's entry (that entry has its own starter), at a tail, or at
+// the length cap only adds its push to the master; the push stays pending in
+// T(x) - S_val[e], like any push from another path.
+__device__ void walk_sparse_acc(const KParams& P, const uint2* list, unsigned qn, unsigned* ticket,
+                                const uint32_t* bcur, Acc& acc) {
+    __shared__ uint32_t s_off[kWarps][33];
+    __shared__ uint32_t s_beg[kWarps][32];
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const unsigned long long eps = P.eps_fx;
+    while (true) {
+        unsigned t = 0;
+        if (lane == 0) t = atomicAdd(ticket, 32u);
+        t = __shfl_sync(0xffffffffu, t, 0);
+        if (t >= qn) break;
+        uint32_t cnt = 0, beg = 0;
+        if (t + lane < qn) {
+            const uint2 it = list[t + lane];
+            beg = P.occ_off[it.x] + it.y * kOccChunk;
+            cnt = min(P.occ_off[it.x + 1] - beg, kOccChunk);
+            acc.units++;
+        }
+        uint32_t inc = cnt;
+#pragma unroll
+        for (int off = 1; off < 32; off <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, off);
+            if (lane >= off) inc += y;
+        }
+        s_off[wid][lane + 1] = inc;
+        if (lane == 0) s_off[wid][0] = 0;
+        s_beg[wid][lane] = beg;
+        __syncwarp();
+        const uint32_t total = s_off[wid][32];
+        for (uint32_t j = lane; j < total; j += 32) {
+            int lo = 0, hi = 31;
+            while (lo < hi) {
+                const int mid = (lo + hi + 1) >> 1;
+                if (s_off[wid][mid] <= j) lo = mid; else hi = mid - 1;
+            }
+            uint32_t e = P.occ[s_beg[wid][lo] + (j - s_off[wid][lo])];
+            uint32_t x = __ldg(P.e_idx + e) & kVMask;
+            unsigned long long p = 0ull;  // push arriving at entry e
+            for (int step = 0; step <= P.sparse_walk; step++) {
+                const uint32_t code = step ? __ldg(P.e_idx + e) : 0u;
+                const unsigned long long T = __ldcg(&P.vs_t[x]);
+                if (p) {
+                    atomicAdd(&P.vs_t[x], p);
+                    acc.upd++;
+                }
+                acc.entries++;
+                if (step) acc.edges++;
+                // stop: tail, the entry has its own starter, or the cap (the push stays pending)
+                if (step && ((code & kTail) || test_bit(bcur, x) || step == P.sparse_walk)) break;
+                const unsigned long long sv = P.s_val[e];
+                const unsigned long long pd = T > sv ? T - sv : 0ull;
+                const unsigned long long amt = (pd >= eps ? pd : 0ull) + p;
+                if (!amt) break;
+                P.s_val[e] = sv + amt;
+                p = fx_from(__ldg(P.e_coef + e) * fx_to(amt));
+                if (!p) break;
+                e++;
+                x = __ldg(P.e_idx + e) & kVMask;
+            }
+        }
+        __syncwarp();
     }
 }
 
@@ -995,6 +1150,20 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
         const uint32_t* bcur = P.bits + (int64_t)cur * P.nw;
         uint32_t* bnxt = P.bits + (int64_t)nxt * P.nw;
         if (kAccum) {
+            // sparse round: few signalled vertices whose out-edges are at most M / sparse_div
+            bool sparse = false;
+            if (P.occ_off && *((volatile unsigned*)&P.ctr->active[cur]) <= P.sparse_max) {
+                count_bits(P, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
+                grid.sync();
+                sparse = *((volatile unsigned*)&P.ctr->osum[cur]) <= P.sparse_occ;
+                if (sparse) {
+                    compact_bits(P, bcur, P.occ_items, &P.ctr->qcur[cur]);
+                    grid.sync();
+                }
+            }
+            if (sparse) {
+                walk_sparse_acc(P, P.occ_items, *((volatile unsigned*)&P.ctr->qn[cur]), &P.ctr->ticket[cur], bcur, acc);
+            } else {
             if (px.H) {  // round-start snapshot of the proxied masters
                 for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) {
                     px.T[i] = __ldcg(&P.vs_t[i]);
@@ -1009,8 +1178,9 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
                 for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x)
                     if (const unsigned long long a = px_read(&px.acc[2 * i])) atomicAdd(&P.vs_t[i], a);
             }
+            }
             grid.sync();  // all pushes of the round landed
-            accum_sweep(P, acc.sig);
+            accum_sweep(P, bnxt, acc.sig);
         } else {
             unsigned* ticket = &P.ctr->ticket[cur];
             // bucket bound of this round (reading R-DELTA): only distances <= theta are committed
@@ -1020,7 +1190,7 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             // signalled, compact them; walk from them if their out-edges are
             // at most 1/sparse_div of the path entries, else walk the windows
             bool sparse = false;
-            if ((ALGO == DG_SSSP || ALGO == DG_BFS) && P.occ_off &&
+            if ((ALGO == DG_SSSP || ALGO == DG_BFS || ALGO == 100) && P.occ_off &&
                 *((volatile unsigned*)&P.ctr->active[cur]) <= P.sparse_max) {
                 count_bits(P, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
                 grid.sync();
@@ -1033,12 +1203,31 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             if (sparse) {
                 const unsigned qn = *((volatile unsigned*)&P.ctr->qn[cur]);
                 if (ALGO == DG_SSSP) walk_sparse<0>(P, P.occ_items, qn, ticket, bnxt, theta, acc);
-                else walk_sparse<1>(P, P.occ_items, qn, ticket, bnxt, theta, acc);
+                else if (ALGO == DG_BFS) walk_sparse<1>(P, P.occ_items, qn, ticket, bnxt, theta, acc);
+                else walk_sparse<3>(P, P.occ_items, qn, ticket, bnxt, theta, acc);
             } else if (ALGO == DG_SSSP) walk_minplus<0>(P, ticket, bcur, bnxt, theta, acc);
             else if (ALGO == DG_BFS) walk_minplus<1>(P, ticket, bcur, bnxt, theta, acc);
             else if (ALGO == DG_WCC) walk_minplus<2>(P, ticket, bcur, bnxt, INF, acc);
             else if (ALGO == 100) walk_minplus<3>(P, ticket, bcur, bnxt, INF, acc);
-            else if (ALGO == 101) {
+            else if (ALGO == 101 && P.occ_off &&
+                     *((volatile unsigned*)&P.ctr->active[cur]) <= P.sparse_max) {
+                // sparse backward round (same decision as the forward rounds)
+                count_bits(P, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
+                grid.sync();
+                if (*((volatile unsigned*)&P.ctr->osum[cur]) <= P.sparse_occ) {
+                    compact_bits(P, bcur, P.occ_items, &P.ctr->qcur[cur]);
+                    grid.sync();
+                    walk_sparse_bwd(P, P.occ_items, *((volatile unsigned*)&P.ctr->qn[cur]), ticket, bnxt, acc);
+                } else {
+                    while (true) {
+                        unsigned t = 0;
+                        if (lane == 0) t = atomicAdd(ticket, 1u);
+                        t = __shfl_sync(0xffffffffu, t, 0);
+                        if (t >= (unsigned)P.n_part) break;
+                        walk_scc_bwd(P, P.part_off[t], P.part_off[t + 1], bcur, bnxt, acc);
+                    }
+                }
+            } else if (ALGO == 101) {
                 while (true) {
                     unsigned t = 0;
                     if (lane == 0) t = atomicAdd(ticket, 1u);
@@ -1307,16 +1496,18 @@ __global__ void scale_f_kernel(float* x, int64_t n, const double* sum) {
 }
 
 // ---- occurrence index (sparse min-plus rounds): vertex -> its non-tail entries
-__global__ void occ_count_kernel(const uint32_t* e_idx, int64_t M, uint32_t* cnt) {
+// (skip = kTail: out-edges, the entries a path edge leaves; skip = kHead:
+// in-edges, the entries a path edge enters)
+__global__ void occ_count_kernel(const uint32_t* e_idx, int64_t M, uint32_t skip, uint32_t* cnt) {
     GRID_STRIDE(i, M) {
         const uint32_t c = e_idx[i];
-        if (!(c & kTail)) atomicAdd(&cnt[(c & kVMask) + 1], 1u);
+        if (!(c & skip)) atomicAdd(&cnt[(c & kVMask) + 1], 1u);
     }
 }
-__global__ void occ_fill_kernel(const uint32_t* e_idx, int64_t M, uint32_t* cursor, uint32_t* occ) {
+__global__ void occ_fill_kernel(const uint32_t* e_idx, int64_t M, uint32_t skip, uint32_t* cursor, uint32_t* occ) {
     GRID_STRIDE(i, M) {
         const uint32_t c = e_idx[i];
-        if (!(c & kTail)) occ[atomicAdd(&cursor[c & kVMask], 1u)] = (uint32_t)i;
+        if (!(c & skip)) occ[atomicAdd(&cursor[c & kVMask], 1u)] = (uint32_t)i;
     }
 }
 
@@ -1326,6 +1517,17 @@ __global__ void scc_init_kernel(uint32_t* vs, const int32_t* label, const int32_
     GRID_STRIDE(v, n) {
         vs[v] = label[v] < 0 ? (uint32_t)orig[v] : INF;
         mark[v] = 0;
+    }
+}
+// the forward phase starts with every unassigned vertex signalled
+__global__ void scc_bits_kernel(const int32_t* label, int64_t n, uint32_t* b, int64_t nw) {
+    GRID_STRIDE(i, nw) {
+        uint32_t w = 0;
+        for (int k = 0; k < 32; k++) {
+            const int64_t v = i * 32 + k;
+            if (v < n && label[v] < 0) w |= 1u << k;
+        }
+        b[i] = w;
     }
 }
 // roots keep their own id as colour; they seed the backward phase's bitmap
@@ -1381,7 +1583,7 @@ __global__ void pack_sum_kernel(const unsigned long long* vs, const int32_t* bnd
 }
 __global__ void unpack_sum_kernel(unsigned long long* vs, unsigned long long* sigma, const int32_t* bnd, int64_t nb,
                                   unsigned long long* base, const unsigned long long* buf, unsigned long long eps,
-                                  int round, Counters* ctr, int slot) {
+                                  uint32_t* b, Counters* ctr, int slot) {
     unsigned cnt = 0;
     GRID_STRIDE(k, nb) {
         const int v = bnd[k];
@@ -1390,6 +1592,7 @@ __global__ void unpack_sum_kernel(unsigned long long* vs, unsigned long long* si
         vs[v] = t;
         if (t - sigma[v] >= eps) {  // the replica's growth counts as a signal of the next local round
             sigma[v] = t;
+            signal_vertex(b, (uint32_t)v);  // (the bitmap sparse rounds read)
             cnt++;
         }
     }
@@ -1534,38 +1737,62 @@ int64_t sparse_min_entries() {
     return e ? std::atoll(e) : (int64_t)1 << 23;
 }
 
-// Occurrence index: counting sort of the non-tail entries by vertex (built on
-// the device on the first SSSP/BFS run after an upload).
-int ensure_occ(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
-    if (W->occ_ok) return DG_OK;
+// Occurrence index: counting sort of the non-tail (out-edge) or non-head
+// (in-edge, SCC backward) entries by vertex, built on the device on the first
+// run that needs it after an upload.
+// Scratch (cursor, cub temporary) and the index arrays stay allocated across
+// re-uploads of a layout of the same size; only the contents are rebuilt.
+int build_occ(DevWork* W, const DevLayout& D, uint32_t skip, uint32_t*& off, uint32_t*& occ, int64_t& cap,
+              RunState& S, std::string& err) {
     int64_t bytes = 0;
     int rc;
-    uint32_t *cur = nullptr;
-    void* tmp = nullptr;
+    const bool verbose = std::getenv("DG_VERBOSE") != nullptr;
+    if (verbose) CK(cudaEventRecord(W->ev0));
+    if (!off && (rc = dalloc(&off, D.n + 1, bytes, err))) return rc;
+    if (!W->occ_cur && (rc = dalloc(&W->occ_cur, D.n + 1, bytes, err))) return rc;
+    CK(cudaMemsetAsync(off, 0, sizeof(uint32_t) * (D.n + 1)));
+    occ_count_kernel<<<grid_1d(D.M), 256>>>(D.e_idx, D.M, skip, off);
     size_t tmp_bytes = 0;
-    if ((rc = dalloc(&W->occ_off, D.n + 1, bytes, err))) return rc;
-    if ((rc = dalloc(&cur, D.n + 1, bytes, err))) return rc;
-    CK(cudaMemsetAsync(W->occ_off, 0, sizeof(uint32_t) * (D.n + 1)));
-    occ_count_kernel<<<grid_1d(D.M), 256>>>(D.e_idx, D.M, W->occ_off);
-    CK(cub::DeviceScan::InclusiveSum(nullptr, tmp_bytes, W->occ_off, W->occ_off, (int)(D.n + 1)));
-    CK(cudaMalloc(&tmp, tmp_bytes ? tmp_bytes : 1));
-    CK(cub::DeviceScan::InclusiveSum(tmp, tmp_bytes, W->occ_off, W->occ_off, (int)(D.n + 1)));
-    uint32_t total = 0;
-    CK(cudaMemcpy(&total, W->occ_off + D.n, sizeof(uint32_t), cudaMemcpyDeviceToHost));
-    if ((rc = dalloc(&W->occ, (size_t)total + 1, bytes, err)) ||
-        (rc = dalloc(&W->occ_items, (size_t)(D.n + total / kOccChunk + 1), bytes, err))) {
-        cudaFree(cur);
-        cudaFree(tmp);
-        return rc;
+    CK(cub::DeviceScan::InclusiveSum(nullptr, tmp_bytes, off, off, (int)(D.n + 1)));
+    if (tmp_bytes > W->cub_tmp_bytes) {
+        if (W->cub_tmp) cudaFree(W->cub_tmp);
+        CK(cudaMalloc(&W->cub_tmp, tmp_bytes));
+        W->cub_tmp_bytes = tmp_bytes;
     }
-    CK(cudaMemcpyAsync(cur, W->occ_off, sizeof(uint32_t) * D.n, cudaMemcpyDeviceToDevice));
-    occ_fill_kernel<<<grid_1d(D.M), 256>>>(D.e_idx, D.M, cur, W->occ);
+    CK(cub::DeviceScan::InclusiveSum(W->cub_tmp, tmp_bytes, off, off, (int)(D.n + 1)));
+    uint32_t total = 0;
+    CK(cudaMemcpy(&total, off + D.n, sizeof(uint32_t), cudaMemcpyDeviceToHost));
+    if ((int64_t)total + 1 > cap) {
+        dfree(occ);
+        if ((rc = dalloc(&occ, (size_t)total + 1, bytes, err))) return rc;
+        cap = (int64_t)total + 1;
+    }
+    CK(cudaMemcpyAsync(W->occ_cur, off, sizeof(uint32_t) * D.n, cudaMemcpyDeviceToDevice));
+    occ_fill_kernel<<<grid_1d(D.M), 256>>>(D.e_idx, D.M, skip, W->occ_cur, occ);
     CK(cudaGetLastError());
-    CK(cudaDeviceSynchronize());
-    cudaFree(cur);
-    cudaFree(tmp);
     S.stats.kernel_launches += 3;
-    W->occ_ok = true;
+    if (verbose) {
+        CK(cudaEventRecord(W->ev1));
+        CK(cudaEventSynchronize(W->ev1));
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, W->ev0, W->ev1));
+        fprintf(stderr, "[dg] occurrence index (%s): %u entries in %.2f ms\n", skip == kTail ? "out" : "in", total, ms);
+    }
+    return DG_OK;
+}
+int ensure_occ(DevWork* W, const DevLayout& D, RunState& S, bool incoming, std::string& err) {
+    int rc;
+    if (!W->occ_items) {  // every path edge is one out- and one in-occurrence: one item buffer serves both
+        int64_t bytes = 0;
+        if ((rc = dalloc(&W->occ_items, (size_t)(D.n + D.m / kOccChunk + 1), bytes, err))) return rc;
+    }
+    if (incoming) {
+        if (!W->iocc_ok && (rc = build_occ(W, D, kHead, W->iocc_off, W->iocc, W->iocc_cap, S, err))) return rc;
+        W->iocc_ok = true;
+    } else {
+        if (!W->occ_ok && (rc = build_occ(W, D, kTail, W->occ_off, W->occ, W->occ_cap, S, err))) return rc;
+        W->occ_ok = true;
+    }
     return DG_OK;
 }
 
@@ -1598,11 +1825,13 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
         const char* dl = std::getenv("DG_DELTA");  // bucket width knob; default: reading R-DELTA
         P.delta = dl ? (uint32_t)std::atoi(dl) : (uint32_t)S.delta;
         const int64_t sd = sparse_div();
-        if ((algo_k == DG_SSSP || algo_k == DG_BFS) && sd > 0 && D.M >= sparse_min_entries()) {
+        if ((algo_k == DG_SSSP || algo_k == DG_BFS || algo_k == 100 || algo_k == 101 || algo_k == DG_PAGERANK ||
+             algo_k == DG_ADSORPTION) && sd > 0 && D.M >= sparse_min_entries()) {
             int rc;
-            if ((rc = ensure_occ(W, D, S, err))) return rc;
-            P.occ_off = W->occ_off;
-            P.occ = W->occ;
+            const bool in = algo_k == 101;
+            if ((rc = ensure_occ(W, D, S, in, err))) return rc;
+            P.occ_off = in ? W->iocc_off : W->occ_off;
+            P.occ = in ? W->iocc : W->occ;
             P.occ_items = W->occ_items;
             P.sparse_max = (uint32_t)std::min<int64_t>(D.n / 4, 0xFFFFFFFFll);
             P.sparse_occ = (uint32_t)std::min<int64_t>(D.M / sd, 0xFFFFFFFFll);
@@ -1715,13 +1944,15 @@ int run_scc(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, std
     Counters tot{};
     int64_t total_rounds = 0;
     const int rounds = (int)std::min<int64_t>(max_rounds, 1 << 30);
+    const bool verbose = std::getenv("DG_VERBOSE") != nullptr;
+    int32_t rem = (int32_t)D.n;
     for (int64_t it = 0;; it++) {
         // forward colouring: every unassigned vertex starts with its own id, all signalled
         scc_init_kernel<<<g, 256>>>(W->vs_u, W->scc_label, D.orig, W->scc_mark, D.n);
         CK(cudaMemsetAsync(W->bits, 0, sizeof(uint32_t) * 2 * W->nw));
-        bits_all_kernel<<<grid_1d(W->nw), 256>>>(W->bits, W->nw, D.n);
+        scc_bits_kernel<<<grid_1d(W->nw), 256>>>(W->scc_label, D.n, W->bits, W->nw);
         Counters c0{};
-        c0.active[0] = (unsigned)D.n;
+        c0.active[0] = (unsigned)rem;
         if ((rc = write_counters(W, c0, err))) return rc;
         S.stats.kernel_launches += 2;
         if ((rc = launch_path(W, D, 100, rounds, S, err))) return rc;
@@ -1744,9 +1975,11 @@ int run_scc(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, std
         CK(cudaMemset(W->remaining, 0, sizeof(int32_t)));
         scc_assign_kernel<<<g, 256>>>(W->vs_u, W->scc_label, W->scc_mark, D.n, W->remaining);
         S.stats.kernel_launches += 1;
-        int32_t rem = 0;
         CK(cudaMemcpy(&rem, W->remaining, sizeof(int32_t), cudaMemcpyDeviceToHost));
         S.stats.outer_iterations = it + 1;
+        if (verbose)
+            fprintf(stderr, "[dg] scc iteration %lld: forward %d rounds, backward %d rounds, %d unassigned\n",
+                    (long long)it, c1.round, c3.round, rem);
         if (rem == 0) break;
         if (it > D.n) { err = "SCC colouring did not terminate"; return DG_ENOCONV; }
     }
@@ -1868,7 +2101,8 @@ void dev_free_work(DevWork*& W) {
     dfree(W->vs_u); dfree(W->vstamp); dfree(W->vs_f); dfree(W->vs_t); dfree(W->sigma); dfree(W->s_val); dfree(W->bnd_base);
     dfree(W->e_coef); dfree(W->pr_coef); dfree(W->ads_base); dfree(W->bits); dfree(W->vlist[0]); dfree(W->vlist[1]);
     dfree(W->ctr); dfree(W->dsum); dfree(W->scc_label); dfree(W->scc_mark); dfree(W->remaining); dfree(W->out_stage);
-    dfree(W->occ_off); dfree(W->occ); dfree(W->occ_items);
+    dfree(W->occ_off); dfree(W->occ); dfree(W->occ_items); dfree(W->iocc_off); dfree(W->iocc); dfree(W->occ_cur);
+    if (W->cub_tmp) cudaFree(W->cub_tmp);
     if (W->ev0) cudaEventDestroy(W->ev0);
     if (W->ev1) cudaEventDestroy(W->ev1);
     if (W->kev0) cudaEventDestroy(W->kev0);
@@ -1880,8 +2114,7 @@ void dev_free_work(DevWork*& W) {
 void dev_layout_changed(DevWork* W) {
     if (!W) return;
     W->pr_coef_d = -1.0;
-    dfree(W->occ_off); dfree(W->occ); dfree(W->occ_items);
-    W->occ_ok = false;
+    W->occ_ok = W->iocc_ok = false;  // rebuilt on next use (allocations kept: same n, M)
 }
 
 int dev_set_vertex_params(DevWork*& W, const DevLayout& D, const double* p_inj, const double* p_cont,
@@ -1992,7 +2225,7 @@ int dev_boundary_unpack(DevWork* W, const DevLayout& D, RunState& S, const void*
         if (S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION)
             unpack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_t, W->sigma, D.bnd, D.n_bnd, W->bnd_base,
                                                          (const unsigned long long*)buf,
-                                                         (unsigned long long)(S.eps * 4294967296.0), c.round, W->ctr,
+                                                         (unsigned long long)(S.eps * 4294967296.0), b, W->ctr,
                                                          slot);
         else
             unpack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, D.bnd, D.n_bnd, (const uint32_t*)buf, b, W->ctr,

@@ -176,3 +176,35 @@ def test_min_plus_exact_in_sparse_and_dense_rounds(graph, sparse_div, gname, del
     assert np.array_equal(dg.get_states().astype(np.int64), exp)
     if delta == 1:  # level-synchronous in either kind of round
         assert st["vertex_updates"] == int((exp < OA.UNREACHED).sum()) - 1
+    if delta is None:  # SCC forward colouring walks sparse too
+        dg.run("scc")
+        assert np.array_equal(dg.get_states().astype(np.int64), OA.scc_tarjan(g.n, src, dst))
+
+
+@pytest.mark.parametrize("gname", ["rmat", "chains", "uniform_dup"])
+def test_accumulative_in_sparse_and_dense_rounds(graph, sparse_div, gname):
+    # DESIGN.md "Sparse rounds" (accumulative): walks from the signalled
+    # vertices forward pending totals with the same per-entry rule; PageRank and
+    # Adsorption stay within the north_star tolerance (L1 <= 1e-4, per-vertex
+    # relative error <= 1e-3 against the oracle converged to 1e-12)
+    g = {"rmat": graph,
+         "chains": inputs.chains(20000, 26000, chain_len=700, seed=13),
+         "uniform_dup": inputs.uniform(3000, 9000, seed=12, dedupe=False, drop_self=False)}[gname]
+    dg = DiGraph()
+    dg.load_graph(g)
+    dg.build_paths()
+    src, dst, w = g.edges()
+    st = dg.run("pagerank", epsilon=1e-7, damping=0.85)
+    got = dg.get_states().astype(np.float64)
+    exp, _ = OA.pagerank_power(g.n, src, dst, d=0.85, tol=1e-12)
+    assert np.abs(got - exp).sum() <= 1e-4
+    assert (np.abs(got - exp) / exp).max() <= 1e-3
+    assert st["converged"]
+    p_inj, p_cont, inj = inputs.adsorption_params(g.n, seed=3)
+    dg.set_vertex_params(p_inj, p_cont, inj)
+    dg.run("adsorption", epsilon=1e-7)
+    got = dg.get_states().astype(np.float64)
+    exp, _ = OA.adsorption_jacobi(g.n, src, dst, w, p_inj, p_cont, inj, tol=1e-12)
+    assert np.abs(got - exp).sum() / np.abs(exp).sum() <= 1e-4
+    big = exp > 1e-3 * exp.mean()
+    assert (np.abs(got - exp)[big] / exp[big]).max() <= 1e-3
