@@ -67,6 +67,7 @@ struct Counters {
     unsigned int qn[2];      // SSSP/BFS sparse rounds: length of the round's compacted frontier list
     unsigned int osum[2];    // ... and the occurrences (out-edges) of its vertices
     unsigned int qcur[2];    // append cursor of the list
+    unsigned int qn_in[2], osum_in[2], qcur_in[2], ticket_in[2];  // WCC sparse rounds: the in-edge phase
     int round;  // global round number of the next round
     int pad;
 };
@@ -140,6 +141,8 @@ struct KParams {
     const uint32_t* occ_off;  // SSSP/BFS sparse rounds: occurrence index (null: dense rounds only)
     const uint32_t* occ;
     uint2* occ_items;         // the round's frontier items (v, chunk)
+    const uint32_t* iocc_off;  // WCC: the in-edge occurrence index as well
+    const uint32_t* iocc;
     uint32_t sparse_max;      // rounds with at most this many signalled vertices are candidates (n/4)
     uint32_t sparse_occ;      // ... and are walked sparse if their out-edges are at most this many
     int sparse_walk;          // path edges a sparse walk follows at most
@@ -506,13 +509,13 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
 // kOccChunk occurrences, so a hub's out-edges spread over many warps.
 constexpr uint32_t kOccChunk = 32;
 // Pass 1 (count): out-edges and items of the signalled vertices.
-__device__ void count_bits(const KParams& P, const uint32_t* bcur, unsigned* qn, unsigned* osum) {
+__device__ void count_bits(const KParams& P, const uint32_t* off, const uint32_t* bcur, unsigned* qn, unsigned* osum) {
     const int64_t T = (int64_t)gridDim.x * blockDim.x;
     unsigned c = 0, o = 0;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < P.nw; i += T) {
         for (uint32_t x = bcur[i]; x; x &= x - 1) {
             const uint32_t v = (uint32_t)(i * 32 + __ffs(x) - 1);
-            const uint32_t d = P.occ_off[v + 1] - P.occ_off[v];
+            const uint32_t d = off[v + 1] - off[v];
             c += (d + kOccChunk - 1) / kOccChunk;
             o += d;
         }
@@ -527,7 +530,7 @@ __device__ void count_bits(const KParams& P, const uint32_t* bcur, unsigned* qn,
     }
 }
 // Pass 2 (write): the items, appended warp by warp (order is irrelevant).
-__device__ void compact_bits(const KParams& P, const uint32_t* bcur, uint2* list, unsigned* cursor) {
+__device__ void compact_bits(const KParams& P, const uint32_t* off, const uint32_t* bcur, uint2* list, unsigned* cursor) {
     const int lane = threadIdx.x & 31;
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
     const int64_t gw = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
@@ -537,7 +540,7 @@ __device__ void compact_bits(const KParams& P, const uint32_t* bcur, uint2* list
         unsigned c = 0;
         for (uint32_t x = w; x; x &= x - 1) {
             const uint32_t v = (uint32_t)(i * 32 + __ffs(x) - 1);
-            c += (P.occ_off[v + 1] - P.occ_off[v] + kOccChunk - 1) / kOccChunk;
+            c += (off[v + 1] - off[v] + kOccChunk - 1) / kOccChunk;
         }
         unsigned inc = c;
 #pragma unroll
@@ -553,14 +556,15 @@ __device__ void compact_bits(const KParams& P, const uint32_t* bcur, uint2* list
         while (w) {
             const uint32_t v = (uint32_t)(i * 32 + __ffs(w) - 1);
             w &= w - 1;
-            const uint32_t nch = (P.occ_off[v + 1] - P.occ_off[v] + kOccChunk - 1) / kOccChunk;
+            const uint32_t nch = (off[v + 1] - off[v] + kOccChunk - 1) / kOccChunk;
             for (uint32_t k = 0; k < nch; k++) list[base++] = make_uint2(v, k);
         }
     }
 }
 
 template <int MODE>
-__device__ void walk_sparse(const KParams& P, const uint2* list, unsigned qn, unsigned* ticket, uint32_t* bnxt,
+__device__ void walk_sparse(const KParams& P, const uint32_t* off, const uint32_t* occ, const uint2* list, unsigned qn,
+                            unsigned* ticket, uint32_t* bnxt,
                             uint32_t theta, Acc& acc) {
     __shared__ uint32_t s_off[kWarps][33];
     __shared__ uint32_t s_beg[kWarps][32], s_x[kWarps][32], s_v[kWarps][32];
@@ -574,8 +578,8 @@ __device__ void walk_sparse(const KParams& P, const uint2* list, unsigned qn, un
         if (t + lane < qn) {
             const uint2 it = list[t + lane];
             v = it.x;
-            beg = P.occ_off[v] + it.y * kOccChunk;
-            cnt = min(P.occ_off[v + 1] - beg, kOccChunk);
+            beg = off[v] + it.y * kOccChunk;
+            cnt = min(off[v + 1] - beg, kOccChunk);
             x = P.vs_u[v];
             acc.units++;
         }
@@ -599,7 +603,7 @@ __device__ void walk_sparse(const KParams& P, const uint2* list, unsigned qn, un
                 if (s_off[wid][mid] <= j) lo = mid; else hi = mid - 1;
             }
             uint32_t cur = s_x[wid][lo], pred = s_v[wid][lo];
-            uint32_t e = P.occ[s_beg[wid][lo] + (j - s_off[wid][lo])] + 1;  // the path edge out of the occurrence
+            uint32_t e = occ[s_beg[wid][lo] + (j - s_off[wid][lo])] + 1;  // the path edge out of the occurrence
             // the next entry of the path is loaded one step ahead
             uint32_t code = __ldg(P.e_idx + e);
             uint32_t w = MODE == 0 ? (uint32_t)__ldg(P.e_w + e) : (MODE == 1 ? 1u : 0u);
@@ -640,8 +644,10 @@ __device__ void walk_sparse(const KParams& P, const uint2* list, unsigned qn, un
 // vertex v, walk its in-edges backwards (P.occ_off/P.occ hold the non-head
 // entries here: the path edge INTO entry i comes from entry i-1) and mark
 // unassigned predecessors of v's colour, passing the mark on along the path.
-__device__ void walk_sparse_bwd(const KParams& P, const uint2* list, unsigned qn, unsigned* ticket, uint32_t* bnxt,
-                                Acc& acc) {
+// WCC: the same backward walk carries the smallest label (atomicMin) instead.
+template <bool WCC>
+__device__ void walk_sparse_bwd(const KParams& P, const uint32_t* off, const uint32_t* occ, const uint2* list,
+                                unsigned qn, unsigned* ticket, uint32_t* bnxt, Acc& acc) {
     __shared__ uint32_t s_off[kWarps][33];
     __shared__ uint32_t s_beg[kWarps][32], s_x[kWarps][32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -653,8 +659,8 @@ __device__ void walk_sparse_bwd(const KParams& P, const uint2* list, unsigned qn
         uint32_t cnt = 0, beg = 0, col = INF;
         if (t + lane < qn) {
             const uint2 it = list[t + lane];
-            beg = P.occ_off[it.x] + it.y * kOccChunk;
-            cnt = min(P.occ_off[it.x + 1] - beg, kOccChunk);
+            beg = off[it.x] + it.y * kOccChunk;
+            cnt = min(off[it.x + 1] - beg, kOccChunk);
             col = P.vs_u[it.x];
             acc.units++;
         }
@@ -677,17 +683,23 @@ __device__ void walk_sparse_bwd(const KParams& P, const uint2* list, unsigned qn
                 if (s_off[wid][mid] <= j) lo = mid; else hi = mid - 1;
             }
             const uint32_t c = s_x[wid][lo];
-            uint32_t e = P.occ[s_beg[wid][lo] + (j - s_off[wid][lo])] - 1;  // the path predecessor
+            uint32_t e = occ[s_beg[wid][lo] + (j - s_off[wid][lo])] - 1;  // the path predecessor
             for (int step = 0; step < P.sparse_walk; step++) {
                 const uint32_t code = __ldg(P.e_idx + e);
                 const uint32_t u = code & kVMask;
                 acc.entries++;
                 acc.edges++;
-                if (P.scc_label[u] >= 0 || P.vs_u[u] != c || P.mark[u]) break;
-                P.mark[u] = 1;  // idempotent byte store; the signal bit counts it once
-                if (signal_vertex(bnxt, u)) {
+                if (WCC) {
+                    if (c >= __ldcg(&P.vs_u[u]) || c >= atomicMin(&P.vs_u[u], c)) break;
                     acc.upd++;
-                    acc.sig++;
+                    acc.sig += signal_vertex(bnxt, u);
+                } else {
+                    if (P.scc_label[u] >= 0 || P.vs_u[u] != c || P.mark[u]) break;
+                    P.mark[u] = 1;  // idempotent byte store; the signal bit counts it once
+                    if (signal_vertex(bnxt, u)) {
+                        acc.upd++;
+                        acc.sig++;
+                    }
                 }
                 if (code & kHead) break;
                 e--;
@@ -1153,11 +1165,11 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             // sparse round: few signalled vertices whose out-edges are at most M / sparse_div
             bool sparse = false;
             if (P.occ_off && *((volatile unsigned*)&P.ctr->active[cur]) <= P.sparse_max) {
-                count_bits(P, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
+                count_bits(P, P.occ_off, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
                 grid.sync();
                 sparse = *((volatile unsigned*)&P.ctr->osum[cur]) <= P.sparse_occ;
                 if (sparse) {
-                    compact_bits(P, bcur, P.occ_items, &P.ctr->qcur[cur]);
+                    compact_bits(P, P.occ_off, bcur, P.occ_items, &P.ctr->qcur[cur]);
                     grid.sync();
                 }
             }
@@ -1192,32 +1204,56 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             bool sparse = false;
             if ((ALGO == DG_SSSP || ALGO == DG_BFS || ALGO == 100) && P.occ_off &&
                 *((volatile unsigned*)&P.ctr->active[cur]) <= P.sparse_max) {
-                count_bits(P, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
+                count_bits(P, P.occ_off, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
                 grid.sync();
                 sparse = *((volatile unsigned*)&P.ctr->osum[cur]) <= P.sparse_occ;
                 if (sparse) {
-                    compact_bits(P, bcur, P.occ_items, &P.ctr->qcur[cur]);
+                    compact_bits(P, P.occ_off, bcur, P.occ_items, &P.ctr->qcur[cur]);
                     grid.sync();
                 }
             }
             if (sparse) {
                 const unsigned qn = *((volatile unsigned*)&P.ctr->qn[cur]);
-                if (ALGO == DG_SSSP) walk_sparse<0>(P, P.occ_items, qn, ticket, bnxt, theta, acc);
-                else if (ALGO == DG_BFS) walk_sparse<1>(P, P.occ_items, qn, ticket, bnxt, theta, acc);
-                else walk_sparse<3>(P, P.occ_items, qn, ticket, bnxt, theta, acc);
+                if (ALGO == DG_SSSP) walk_sparse<0>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
+                else if (ALGO == DG_BFS) walk_sparse<1>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
+                else walk_sparse<3>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
             } else if (ALGO == DG_SSSP) walk_minplus<0>(P, ticket, bcur, bnxt, theta, acc);
             else if (ALGO == DG_BFS) walk_minplus<1>(P, ticket, bcur, bnxt, theta, acc);
-            else if (ALGO == DG_WCC) walk_minplus<2>(P, ticket, bcur, bnxt, INF, acc);
+            else if (ALGO == DG_WCC) {
+                // sparse WCC round: labels go forward along the out-edges, then
+                // backward along the in-edges of the signalled vertices
+                bool wsparse = false;
+                if (P.occ_off && P.iocc_off && *((volatile unsigned*)&P.ctr->active[cur]) <= P.sparse_max) {
+                    count_bits(P, P.occ_off, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
+                    count_bits(P, P.iocc_off, bcur, &P.ctr->qn_in[cur], &P.ctr->osum_in[cur]);
+                    grid.sync();
+                    wsparse = (uint64_t)*((volatile unsigned*)&P.ctr->osum[cur]) +
+                                  *((volatile unsigned*)&P.ctr->osum_in[cur]) <= P.sparse_occ;
+                }
+                if (wsparse) {
+                    compact_bits(P, P.occ_off, bcur, P.occ_items, &P.ctr->qcur[cur]);
+                    grid.sync();
+                    walk_sparse<2>(P, P.occ_off, P.occ, P.occ_items, *((volatile unsigned*)&P.ctr->qn[cur]), ticket,
+                                   bnxt, INF, acc);
+                    grid.sync();  // the item buffer is reused
+                    compact_bits(P, P.iocc_off, bcur, P.occ_items, &P.ctr->qcur_in[cur]);
+                    grid.sync();
+                    walk_sparse_bwd<true>(P, P.iocc_off, P.iocc, P.occ_items, *((volatile unsigned*)&P.ctr->qn_in[cur]),
+                                          &P.ctr->ticket_in[cur], bnxt, acc);
+                } else {
+                    walk_minplus<2>(P, ticket, bcur, bnxt, INF, acc);
+                }
+            }
             else if (ALGO == 100) walk_minplus<3>(P, ticket, bcur, bnxt, INF, acc);
             else if (ALGO == 101 && P.occ_off &&
                      *((volatile unsigned*)&P.ctr->active[cur]) <= P.sparse_max) {
                 // sparse backward round (same decision as the forward rounds)
-                count_bits(P, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
+                count_bits(P, P.occ_off, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
                 grid.sync();
                 if (*((volatile unsigned*)&P.ctr->osum[cur]) <= P.sparse_occ) {
-                    compact_bits(P, bcur, P.occ_items, &P.ctr->qcur[cur]);
+                    compact_bits(P, P.occ_off, bcur, P.occ_items, &P.ctr->qcur[cur]);
                     grid.sync();
-                    walk_sparse_bwd(P, P.occ_items, *((volatile unsigned*)&P.ctr->qn[cur]), ticket, bnxt, acc);
+                    walk_sparse_bwd<false>(P, P.occ_off, P.occ, P.occ_items, *((volatile unsigned*)&P.ctr->qn[cur]), ticket, bnxt, acc);
                 } else {
                     while (true) {
                         unsigned t = 0;
@@ -1266,6 +1302,7 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             P.ctr->qn[cur] = 0;
             P.ctr->osum[cur] = 0;
             P.ctr->qcur[cur] = 0;
+            P.ctr->qn_in[cur] = P.ctr->osum_in[cur] = P.ctr->qcur_in[cur] = P.ctr->ticket_in[cur] = 0;
         }
         grid.sync();
     }
@@ -1826,10 +1863,15 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
         P.delta = dl ? (uint32_t)std::atoi(dl) : (uint32_t)S.delta;
         const int64_t sd = sparse_div();
         if ((algo_k == DG_SSSP || algo_k == DG_BFS || algo_k == 100 || algo_k == 101 || algo_k == DG_PAGERANK ||
-             algo_k == DG_ADSORPTION) && sd > 0 && D.M >= sparse_min_entries()) {
+             algo_k == DG_ADSORPTION || algo_k == DG_WCC) && sd > 0 && D.M >= sparse_min_entries()) {
             int rc;
             const bool in = algo_k == 101;
             if ((rc = ensure_occ(W, D, S, in, err))) return rc;
+            if (algo_k == DG_WCC) {  // both directions
+                if ((rc = ensure_occ(W, D, S, true, err))) return rc;
+                P.iocc_off = W->iocc_off;
+                P.iocc = W->iocc;
+            }
             P.occ_off = in ? W->iocc_off : W->occ_off;
             P.occ = in ? W->iocc : W->occ;
             P.occ_items = W->occ_items;

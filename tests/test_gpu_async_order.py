@@ -176,9 +176,11 @@ def test_min_plus_exact_in_sparse_and_dense_rounds(graph, sparse_div, gname, del
     assert np.array_equal(dg.get_states().astype(np.int64), exp)
     if delta == 1:  # level-synchronous in either kind of round
         assert st["vertex_updates"] == int((exp < OA.UNREACHED).sum()) - 1
-    if delta is None:  # SCC forward colouring walks sparse too
+    if delta is None:  # SCC colouring and WCC labels walk sparse too
         dg.run("scc")
         assert np.array_equal(dg.get_states().astype(np.int64), OA.scc_tarjan(g.n, src, dst))
+        dg.run("wcc")
+        assert np.array_equal(dg.get_states().astype(np.int64), OA.wcc_label_propagation(g.n, src, dst)[0])
 
 
 @pytest.mark.parametrize("gname", ["rmat", "chains", "uniform_dup"])
@@ -208,3 +210,26 @@ def test_accumulative_in_sparse_and_dense_rounds(graph, sparse_div, gname):
     assert np.abs(got - exp).sum() / np.abs(exp).sum() <= 1e-4
     big = exp > 1e-3 * exp.mean()
     assert (np.abs(got - exp)[big] / exp[big]).max() <= 1e-3
+
+
+def test_edge_cases_in_sparse_rounds(sparse_div):
+    # empty edge set, single vertex, self loop only, source without out-edges,
+    # a two-vertex cycle: every algorithm with sparse rounds forced on / off
+    for n, e in [(1, []), (5, []), (3, [(1, 1)]), (4, [(1, 2), (2, 3)]), (3, [(0, 1), (1, 0), (1, 2)])]:
+        src = np.array([a for a, _ in e], np.int64)
+        dst = np.array([b for _, b in e], np.int64)
+        w = [3] * len(e)
+        g = inputs.from_edges(n, list(src), list(dst), w)
+        dg = DiGraph()
+        dg.load_graph(g)
+        dg.build_paths()
+        dg.run("sssp", source=0)
+        assert np.array_equal(dg.get_states().astype(np.int64), OA.sssp_bellman_ford(n, src, dst, w, 0)[0])
+        dg.run("bfs", source=0)
+        assert np.array_equal(dg.get_states().astype(np.int64), OA.bfs_levels(n, src, dst, 0))
+        dg.run("scc")
+        assert np.array_equal(dg.get_states().astype(np.int64), OA.scc_tarjan(n, src, dst))
+        dg.run("wcc")
+        assert np.array_equal(dg.get_states().astype(np.int64), OA.wcc_label_propagation(n, src, dst)[0])
+        dg.run("pagerank")
+        assert np.abs(dg.get_states() - OA.pagerank_power(n, src, dst)[0]).sum() <= 1e-4
