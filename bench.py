@@ -243,7 +243,7 @@ def main():
     ap.add_argument("--eps", type=float, default=1e-7)
     ap.add_argument("--part-entries", type=int, default=0)
     ap.add_argument("--merge-rule", default="relaxed")
-    ap.add_argument("--n-proxy", type=int, default=2048)
+    ap.add_argument("--n-proxy", type=int, default=4096)
     ap.add_argument("--l2-flush-mb", type=int, default=512)
     ap.add_argument("--no-extras", action="store_true", help="skip ablation/e2e/cpu baseline (profiling runs)")
     args = ap.parse_args()

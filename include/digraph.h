@@ -78,7 +78,7 @@ typedef struct {
 
 /* Fill *p with the defaults (d_max 16, l_merge 64, n_sub 64, order 0,
  * hot_factor 2, part_entries 0 (auto), rank 0, world 1, merge_rule 1,
- * n_proxy 2048). */
+ * n_proxy 4096). */
 void dg_default_params(dg_path_params *p);
 
 /* Statistics of one dg_run (device-side counters). */

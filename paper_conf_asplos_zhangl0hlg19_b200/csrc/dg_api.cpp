@@ -49,7 +49,7 @@ void dg_default_params(dg_path_params* p) {
     p->rank = 0;
     p->world = 1;
     p->merge_rule = 1;
-    p->n_proxy = 2048;
+    p->n_proxy = 4096;
 }
 
 int dg_create(dg_graph** out, int device) {

@@ -73,7 +73,7 @@ class DiGraph:
         return self.load_csr(g.n, g.row_ptr, g.col, g.w)
 
     def build_paths(self, d_max=16, l_merge=64, n_sub=64, order="degree", hot_factor=2.0,
-                    part_entries=0, rank=0, world=1, merge_rule="relaxed", n_proxy=2048):
+                    part_entries=0, rank=0, world=1, merge_rule="relaxed", n_proxy=4096):
         p = default_params()
         p.d_max, p.l_merge, p.n_sub = d_max, l_merge, n_sub
         p.order = 0 if order == "degree" else 1
