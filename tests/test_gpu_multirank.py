@@ -29,8 +29,10 @@ def _graph():
     return inputs.rmat(13, 8192, 80000, seed=31)
 
 
-def _worker(rank, world, port, algo, q):
+def _worker(rank, world, port, algo, q, sparse=False):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    if sparse:  # every round with <= n/4 signalled vertices walks sparse
+        os.environ.update(DG_SPARSE_DIV="1", DG_SPARSE_MIN_M="0")
     dist.init_process_group("gloo", rank=rank, world_size=world)
     torch.cuda.set_device(0)
     from paper_conf_asplos_zhangl0hlg19_b200 import DiGraph, parallel
@@ -46,12 +48,13 @@ def _worker(rank, world, port, algo, q):
     dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("sparse", [False, True])
 @pytest.mark.parametrize("algo", ["sssp", "wcc", "pagerank"])
-def test_two_ranks_on_one_gpu_match_oracle(algo, cuda_required):
+def test_two_ranks_on_one_gpu_match_oracle(algo, sparse, cuda_required):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, algo, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, algo, q, sparse)) for r in range(2)]
     for p in procs:
         p.start()
     got, info, stats = q.get(timeout=600)
