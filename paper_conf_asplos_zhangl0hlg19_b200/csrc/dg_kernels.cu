@@ -487,7 +487,8 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
     }
 }
 
-// Sparse min-plus rounds (SSSP/BFS).  When few
+// Sparse min-plus rounds (SSSP/BFS, the forward half of WCC, SCC's forward
+// colouring).  When few
 // vertices are signalled, probing every window's signal bits costs more than
 // the work: the round instead starts the path walks at the signalled vertices.
 // Every out-edge of v lies on exactly one path, right after one of v's
@@ -520,9 +521,9 @@ __device__ void count_bits(const KParams& P, const uint32_t* off, const uint32_t
             o += d;
         }
     }
-    for (int off = 16; off; off >>= 1) {
-        c += __shfl_xor_sync(0xffffffffu, c, off);
-        o += __shfl_xor_sync(0xffffffffu, o, off);
+    for (int sh = 16; sh; sh >>= 1) {
+        c += __shfl_xor_sync(0xffffffffu, c, sh);
+        o += __shfl_xor_sync(0xffffffffu, o, sh);
     }
     if ((threadIdx.x & 31) == 0 && o) {
         atomicAdd(qn, c);
@@ -544,9 +545,9 @@ __device__ void compact_bits(const KParams& P, const uint32_t* off, const uint32
         }
         unsigned inc = c;
 #pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {
-            const unsigned y = __shfl_up_sync(0xffffffffu, inc, off);
-            if (lane >= off) inc += y;
+        for (int sh = 1; sh < 32; sh <<= 1) {
+            const unsigned y = __shfl_up_sync(0xffffffffu, inc, sh);
+            if (lane >= sh) inc += y;
         }
         const unsigned tot = __shfl_sync(0xffffffffu, inc, 31);
         if (tot == 0) continue;
@@ -585,9 +586,9 @@ __device__ void walk_sparse(const KParams& P, const uint32_t* off, const uint32_
         }
         uint32_t inc = cnt;
 #pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, off);
-            if (lane >= off) inc += y;
+        for (int sh = 1; sh < 32; sh <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, sh);
+            if (lane >= sh) inc += y;
         }
         s_off[wid][lane + 1] = inc;
         if (lane == 0) s_off[wid][0] = 0;
@@ -666,9 +667,9 @@ __device__ void walk_sparse_bwd(const KParams& P, const uint32_t* off, const uin
         }
         uint32_t inc = cnt;
 #pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {
-            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, off);
-            if (lane >= off) inc += y;
+        for (int sh = 1; sh < 32; sh <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, sh);
+            if (lane >= sh) inc += y;
         }
         s_off[wid][lane + 1] = inc;
         if (lane == 0) s_off[wid][0] = 0;
