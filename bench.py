@@ -390,7 +390,7 @@ def main():
             "config": {"workload": WORKLOADS.get((args.algo, args.config), f"{args.algo} on {args.config}"),
                        "graph": g.name, "n": g.n, "m": g.m, "algo": args.algo, "mode": args.mode,
                        "epsilon": args.eps if args.algo == "pagerank" else None,
-                       "delta": ("library default (SSSP 2*max weight, BFS unbounded; DESIGN.md R-DELTA)"
+                       "delta": ("library default (SSSP 2*max weight, BFS 1; DESIGN.md R-DELTA)"
                                  if args.algo in ("sssp", "bfs") else None),
                        "l2": f"flushed between steps ({args.l2_flush_mb} MB write outside the step events)",
                        "parallelism": f"paths partitioned over {world} GPU(s)",

@@ -164,7 +164,8 @@ int dg_set_vertex_params(dg_graph *g, const double *p_inj, const double *p_cont,
  *            SSSP/BFS: bucket width Delta of the rounds (DESIGN.md reading
  *            R-DELTA): a round commits only distances <= (smallest distance
  *            signalled by the previous round) + Delta.  0 = library default
- *            (SSSP: 2 * max edge weight; BFS: unbounded), < 0 = unbounded,
+ *            (SSSP: 2 * max edge weight; BFS: 1, level-synchronous),
+ *            < 0 = unbounded,
  *            > 0 = that width.  Results are exact for every value; it trades
  *            redundant updates against rounds.  Ignored by the others.
  *   mode     DG_MODE_PATH or DG_MODE_VERTEX (ablation)

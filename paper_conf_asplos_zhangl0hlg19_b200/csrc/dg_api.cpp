@@ -195,7 +195,7 @@ static int64_t run_delta(const dg_graph* g, int algo, double param) {
     if (algo != DG_SSSP && algo != DG_BFS) return 0;
     if (param > 0) return (int64_t)param;
     if (param < 0) return 0;
-    return algo == DG_SSSP ? 2 * (int64_t)g->csr.max_w : 0;
+    return algo == DG_SSSP ? 2 * (int64_t)g->csr.max_w : 1;  // BFS: level-synchronous
 }
 
 static int check_run_args(dg_graph* g, int algo, int64_t source, double epsilon, double param, int mode) {
