@@ -36,6 +36,7 @@ extern "C" {
 #define DG_ENOMEM (-2)   /* host or device allocation failed                */
 #define DG_ENOCUDA (-3)  /* no CUDA device / kernel launch failed           */
 #define DG_ENOCONV (-4)  /* max_rounds reached before convergence           */
+#define DG_ETIMEOUT (-5) /* a peer rank never reached a boundary exchange  */
 
 /* Unreachable vertex distance for SSSP/BFS (reading R-INF). */
 #define DG_INF 0x7FFFFFFFu
@@ -239,6 +240,35 @@ int dg_boundary_unpack(dg_graph *g, const void *buf, int64_t *active);
 
 /* Finish the run: normalisation (PageRank) and statistics. */
 int dg_run_end(dg_graph *g, dg_run_stats *stats);
+
+/* ---- peer-memory boundary exchange (replaces pack + all-reduce + unpack) ----
+ * PAPER.md line 96 ("state propagation between paths is done through state
+ * synchronization of vertex replicas ... in batches") and line 184 (mirrors
+ * send their new states to their masters).  Every rank owns one exchange
+ * region in its own device memory (256 B of epoch flags + 2 x n_boundary
+ * uint64 slots), mapped into every other rank by CUDA IPC; an exchange packs
+ * this rank's boundary values into its slot, publishes an epoch number into
+ * every peer's flag word, waits (on the device) for every peer's epoch, then
+ * reduces all ranks' slots elementwise straight from peer memory (MIN for
+ * SSSP/BFS/WCC, SUM of fixed-point growth for PageRank/Adsorption) and
+ * applies the result like dg_boundary_unpack.  No host collective moves the
+ * boundary states.  All ranks must hold the same layout (same boundary set)
+ * and call dg_boundary_exchange the same number of times.
+ *
+ * dg_p2p_alloc: after dg_build_paths(rank, world) and dg_upload; allocates
+ *   the region (the library owns it; freed by dg_destroy or the next
+ *   dg_p2p_alloc) and writes its IPC handle to HOST `handle` (64 bytes).
+ *   2 <= world <= 16.  The caller distributes the handles (any transport).
+ * dg_p2p_open: HOST `handles` = world x 64 bytes in rank order (this rank's
+ *   own entry is ignored); maps every peer's region.  Ranks on the same GPU
+ *   in different processes are allowed (tests); two ranks in one process are
+ *   not (CUDA IPC).
+ * dg_boundary_exchange: during a run (after dg_rounds); *active = vertices
+ *   this rank re-signalled.  DG_ETIMEOUT if a peer has not arrived after 60 s
+ *   (the device wait gives up instead of hanging). */
+int dg_p2p_alloc(dg_graph *g, int world, int rank, void *handle);
+int dg_p2p_open(dg_graph *g, const void *handles);
+int dg_boundary_exchange(dg_graph *g, int64_t *active);
 
 #ifdef __cplusplus
 }

@@ -16,6 +16,7 @@ struct dg_graph {
     dg::HostLayout layout;
     dg::DevLayout dev;
     dg::DevWork* work = nullptr;
+    dg::P2P* p2p = nullptr;  // peer-memory exchange region (dg_p2p_alloc)
     dg::RunState run;
     bool loaded = false;
     bool uploaded = false;
@@ -65,6 +66,7 @@ int dg_create(dg_graph** out, int device) {
 
 void dg_destroy(dg_graph* g) {
     if (!g) return;
+    dg::dev_p2p_free(g->p2p);
     dg::dev_free_work(g->work);
     dg::dev_free_layout(g->dev, true);
     dg::dev_unpin_all(g->dev);
@@ -77,6 +79,7 @@ int dg_load_csr(dg_graph* g, int64_t n, int64_t m, const int64_t* row_ptr, const
     if (n < 0 || n >= (int64_t)dg::kVMask || m < 0) return fail(DG_EINVAL, "dg_load_csr: bad n or m");
     if (!row_ptr || (m > 0 && !col)) return fail(DG_EINVAL, "dg_load_csr: NULL row_ptr/col");
     if (row_ptr[0] != 0 || row_ptr[n] != m) return fail(DG_EINVAL, "dg_load_csr: row_ptr[0] != 0 or row_ptr[n] != m");
+    dg::dev_p2p_free(g->p2p);
     dg::dev_free_work(g->work);
     dg::dev_free_layout(g->dev, true);
     dg::dev_unpin_all(g->dev);
@@ -106,6 +109,7 @@ int dg_load_csr(dg_graph* g, int64_t n, int64_t m, const int64_t* row_ptr, const
         return fail(DG_ENOMEM, "dg_load_csr: out of host memory");
     }
     g->layout = dg::HostLayout();
+    dg::dev_p2p_free(g->p2p);
     dg::dev_free_work(g->work);
     dg::dev_free_layout(g->dev, true);
     g->loaded = true;
@@ -123,6 +127,7 @@ int dg_build_paths(dg_graph* g, const dg_path_params* p) {
         q.rank < 0 || q.rank >= q.world || q.l_merge < 0 || q.merge_rule < 0 || q.merge_rule > 1 ||
         q.n_proxy < 0 || q.n_proxy > 16384)
         return fail(DG_EINVAL, "dg_build_paths: bad parameters");
+    dg::dev_p2p_free(g->p2p);
     dg::dev_free_work(g->work);
     dg::dev_free_layout(g->dev, true);
     dg::dev_unpin_all(g->dev);
@@ -134,6 +139,7 @@ int dg_build_paths(dg_graph* g, const dg_path_params* p) {
     } catch (const std::exception& e) {
         return fail(DG_EINVAL, std::string("dg_build_paths: ") + e.what());
     }
+    dg::dev_p2p_free(g->p2p);
     dg::dev_free_work(g->work);
     dg::dev_free_layout(g->dev, true);
     g->uploaded = false;
@@ -347,6 +353,32 @@ int dg_boundary_unpack(dg_graph* g, const void* buf, int64_t* active) {
     if (!buf && !g->layout.boundary.empty()) return fail(DG_EINVAL, "dg_boundary_unpack: NULL buffer");
     std::string err;
     int rc = dg::dev_boundary_unpack(g->work, g->dev, g->run, buf, active, err);
+    return rc ? fail(rc, err) : DG_OK;
+}
+
+int dg_p2p_alloc(dg_graph* g, int world, int rank, void* handle) {
+    if (!g || !g->layout.built || !handle) return fail(DG_EINVAL, "dg_p2p_alloc: no layout built or NULL handle");
+    if (!g->uploaded) return fail(DG_EINVAL, "dg_p2p_alloc: dg_upload first");
+    if (int rc0 = select_dev(g)) return rc0;
+    std::string err;
+    int rc = dg::dev_p2p_alloc(g->p2p, g->dev, world, rank, handle, err);
+    return rc ? fail(rc, err) : DG_OK;
+}
+
+int dg_p2p_open(dg_graph* g, const void* handles) {
+    if (!g || !handles) return fail(DG_EINVAL, "dg_p2p_open: NULL argument");
+    if (!g->p2p) return fail(DG_EINVAL, "dg_p2p_open: dg_p2p_alloc first");
+    if (int rc0 = select_dev(g)) return rc0;
+    std::string err;
+    int rc = dg::dev_p2p_open(g->p2p, handles, err);
+    return rc ? fail(rc, err) : DG_OK;
+}
+
+int dg_boundary_exchange(dg_graph* g, int64_t* active) {
+    if (!g || !g->multi_active || !active) return fail(DG_EINVAL, "dg_boundary_exchange: no run in progress");
+    if (int rc0 = select_dev(g)) return rc0;
+    std::string err;
+    int rc = dg::dev_boundary_exchange(g->work, g->dev, g->run, g->p2p, active, err);
     return rc ? fail(rc, err) : DG_OK;
 }
 

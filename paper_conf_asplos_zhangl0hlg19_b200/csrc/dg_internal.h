@@ -102,6 +102,11 @@ int dev_rounds(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, 
 int dev_boundary_pack(DevWork* W, const DevLayout& D, RunState& S, void* buf, std::string& err);
 int dev_boundary_unpack(DevWork* W, const DevLayout& D, RunState& S, const void* buf, int64_t* active, std::string& err);
 int dev_run_end(DevWork* W, const DevLayout& D, RunState& S, std::string& err);
+struct P2P;  // peer-memory boundary exchange (dg_kernels.cu)
+int dev_p2p_alloc(P2P*& X, const DevLayout& D, int world, int rank, void* handle, std::string& err);
+int dev_p2p_open(P2P* X, const void* handles, std::string& err);
+void dev_p2p_free(P2P*& X);
+int dev_boundary_exchange(DevWork* W, const DevLayout& D, RunState& S, P2P* X, int64_t* active, std::string& err);
 int dev_normalize(void* buf, int64_t n, std::string& err);
 int dev_get_states(DevWork* W, const DevLayout& D, const RunState& S, void* out, int64_t n, int out_is_device,
                    std::string& err);

@@ -562,6 +562,19 @@ __device__ void compact_bits(const KParams& P, const uint32_t* off, const uint32
         }
     }
 }
+// A round's sparse decision: few signalled vertices whose out-edges are at
+// most M / sparse_div; a sparse round compacts the frontier into P.occ_items.
+// (Counting at the end of the previous round, folded into its last barrier,
+// and compacting there were both measured: no gain / slower.)
+__device__ bool sparse_round(const KParams& P, cg::grid_group& grid, int cur, const uint32_t* bcur) {
+    if (!P.occ_off || *((volatile unsigned*)&P.ctr->active[cur]) > P.sparse_max) return false;
+    count_bits(P, P.occ_off, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
+    grid.sync();
+    if (*((volatile unsigned*)&P.ctr->osum[cur]) > P.sparse_occ) return false;
+    compact_bits(P, P.occ_off, bcur, P.occ_items, &P.ctr->qcur[cur]);
+    grid.sync();
+    return true;
+}
 
 template <int MODE>
 __device__ void walk_sparse(const KParams& P, const uint32_t* off, const uint32_t* occ, const uint2* list, unsigned qn,
@@ -1164,18 +1177,8 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
         uint32_t* bnxt = P.bits + (int64_t)nxt * P.nw;
         if (kAccum) {
             // sparse round: few signalled vertices whose out-edges are at most M / sparse_div
-            bool sparse = false;
-            if (P.occ_off && *((volatile unsigned*)&P.ctr->active[cur]) <= P.sparse_max) {
-                count_bits(P, P.occ_off, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
-                grid.sync();
-                sparse = *((volatile unsigned*)&P.ctr->osum[cur]) <= P.sparse_occ;
-                if (sparse) {
-                    compact_bits(P, P.occ_off, bcur, P.occ_items, &P.ctr->qcur[cur]);
-                    grid.sync();
-                }
-            }
-            if (sparse) {
-                walk_sparse_acc(P, P.occ_items, *((volatile unsigned*)&P.ctr->qn[cur]), &P.ctr->ticket[cur], bcur, acc);
+            if (sparse_round(P, grid, cur, bcur)) {
+                walk_sparse_acc(P, P.occ_items, *((volatile unsigned*)&P.ctr->qcur[cur]), &P.ctr->ticket[cur], bcur, acc);
             } else {
             if (px.H) {  // round-start snapshot of the proxied masters
                 for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) {
@@ -1202,19 +1205,9 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             // sparse round: when few vertices are
             // signalled, compact them; walk from them if their out-edges are
             // at most 1/sparse_div of the path entries, else walk the windows
-            bool sparse = false;
-            if ((ALGO == DG_SSSP || ALGO == DG_BFS || ALGO == 100) && P.occ_off &&
-                *((volatile unsigned*)&P.ctr->active[cur]) <= P.sparse_max) {
-                count_bits(P, P.occ_off, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
-                grid.sync();
-                sparse = *((volatile unsigned*)&P.ctr->osum[cur]) <= P.sparse_occ;
-                if (sparse) {
-                    compact_bits(P, P.occ_off, bcur, P.occ_items, &P.ctr->qcur[cur]);
-                    grid.sync();
-                }
-            }
+            const bool sparse = (ALGO == DG_SSSP || ALGO == DG_BFS || ALGO == 100) && sparse_round(P, grid, cur, bcur);
             if (sparse) {
-                const unsigned qn = *((volatile unsigned*)&P.ctr->qn[cur]);
+                const unsigned qn = *((volatile unsigned*)&P.ctr->qcur[cur]);
                 if (ALGO == DG_SSSP) walk_sparse<0>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
                 else if (ALGO == DG_BFS) walk_sparse<1>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
                 else walk_sparse<3>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
@@ -1246,24 +1239,9 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
                 }
             }
             else if (ALGO == 100) walk_minplus<3>(P, ticket, bcur, bnxt, INF, acc);
-            else if (ALGO == 101 && P.occ_off &&
-                     *((volatile unsigned*)&P.ctr->active[cur]) <= P.sparse_max) {
+            else if (ALGO == 101 && sparse_round(P, grid, cur, bcur)) {
                 // sparse backward round (same decision as the forward rounds)
-                count_bits(P, P.occ_off, bcur, &P.ctr->qn[cur], &P.ctr->osum[cur]);
-                grid.sync();
-                if (*((volatile unsigned*)&P.ctr->osum[cur]) <= P.sparse_occ) {
-                    compact_bits(P, P.occ_off, bcur, P.occ_items, &P.ctr->qcur[cur]);
-                    grid.sync();
-                    walk_sparse_bwd<false>(P, P.occ_off, P.occ, P.occ_items, *((volatile unsigned*)&P.ctr->qn[cur]), ticket, bnxt, acc);
-                } else {
-                    while (true) {
-                        unsigned t = 0;
-                        if (lane == 0) t = atomicAdd(ticket, 1u);
-                        t = __shfl_sync(0xffffffffu, t, 0);
-                        if (t >= (unsigned)P.n_part) break;
-                        walk_scc_bwd(P, P.part_off[t], P.part_off[t + 1], bcur, bnxt, acc);
-                    }
-                }
+                walk_sparse_bwd<false>(P, P.occ_off, P.occ, P.occ_items, *((volatile unsigned*)&P.ctr->qcur[cur]), ticket, bnxt, acc);
             } else if (ALGO == 101) {
                 while (true) {
                     unsigned t = 0;
@@ -1536,16 +1514,59 @@ __global__ void scale_f_kernel(float* x, int64_t n, const double* sum) {
 // ---- occurrence index (sparse min-plus rounds): vertex -> its non-tail entries
 // (skip = kTail: out-edges, the entries a path edge leaves; skip = kHead:
 // in-edges, the entries a path edge enters)
-__global__ void occ_count_kernel(const uint32_t* e_idx, int64_t M, uint32_t skip, uint32_t* cnt) {
-    GRID_STRIDE(i, M) {
-        const uint32_t c = e_idx[i];
-        if (!(c & skip)) atomicAdd(&cnt[(c & kVMask) + 1], 1u);
-    }
+// Each block takes one contiguous chunk of entries.  The kOccHubs
+// highest-degree vertices (internal ids [0, kOccHubs)) are counted in shared
+// memory: their occurrences would otherwise serialise on a few global
+// counters (R-MAT hubs hold hundreds of thousands of entries).
+constexpr uint32_t kOccHubs = 4096;
+constexpr int kOccBlocksPerSM = 8;
+__device__ __forceinline__ void occ_chunk(int64_t M, int64_t& beg, int64_t& end) {
+    const int64_t chunk = (M + gridDim.x - 1) / gridDim.x;
+    beg = (int64_t)blockIdx.x * chunk;
+    end = beg + chunk < M ? beg + chunk : M;
 }
-__global__ void occ_fill_kernel(const uint32_t* e_idx, int64_t M, uint32_t skip, uint32_t* cursor, uint32_t* occ) {
-    GRID_STRIDE(i, M) {
+__global__ void __launch_bounds__(256) occ_count_kernel(const uint32_t* e_idx, int64_t M, uint32_t skip,
+                                                        uint32_t hubs, uint32_t* cnt) {
+    __shared__ uint32_t s[kOccHubs];
+    for (uint32_t h = threadIdx.x; h < hubs; h += blockDim.x) s[h] = 0;
+    __syncthreads();
+    int64_t beg, end;
+    occ_chunk(M, beg, end);
+    for (int64_t i = beg + threadIdx.x; i < end; i += blockDim.x) {
+        const uint32_t c = __ldcs(e_idx + i);
+        if (c & skip) continue;
+        const uint32_t v = c & kVMask;
+        if (v < hubs) atomicAdd(&s[v], 1u);
+        else atomicAdd(&cnt[v + 1], 1u);
+    }
+    __syncthreads();
+    for (uint32_t h = threadIdx.x; h < hubs; h += blockDim.x)
+        if (s[h]) atomicAdd(&cnt[h + 1], s[h]);
+}
+// Same chunks: the block recounts its hub occurrences, reserves one range per
+// hub with a single global atomic, then places every occurrence (hubs from
+// their shared-memory cursor, the others from the global one).
+__global__ void __launch_bounds__(256) occ_fill_kernel(const uint32_t* e_idx, int64_t M, uint32_t skip,
+                                                       uint32_t hubs, uint32_t* cursor, uint32_t* occ) {
+    __shared__ uint32_t s[kOccHubs];
+    for (uint32_t h = threadIdx.x; h < hubs; h += blockDim.x) s[h] = 0;
+    __syncthreads();
+    int64_t beg, end;
+    occ_chunk(M, beg, end);
+    for (int64_t i = beg + threadIdx.x; i < end; i += blockDim.x) {
         const uint32_t c = e_idx[i];
-        if (!(c & skip)) occ[atomicAdd(&cursor[c & kVMask], 1u)] = (uint32_t)i;
+        if (!(c & skip) && (c & kVMask) < hubs) atomicAdd(&s[c & kVMask], 1u);
+    }
+    __syncthreads();
+    for (uint32_t h = threadIdx.x; h < hubs; h += blockDim.x)
+        if (s[h]) s[h] = atomicAdd(&cursor[h], s[h]);
+    __syncthreads();
+    for (int64_t i = beg + threadIdx.x; i < end; i += blockDim.x) {
+        const uint32_t c = __ldcs(e_idx + i);
+        if (c & skip) continue;
+        const uint32_t v = c & kVMask;
+        const uint32_t pos = v < hubs ? atomicAdd(&s[v], 1u) : atomicAdd(&cursor[v], 1u);
+        occ[pos] = (uint32_t)i;
     }
 }
 
@@ -1631,6 +1652,90 @@ __global__ void unpack_sum_kernel(unsigned long long* vs, unsigned long long* si
         if (t - sigma[v] >= eps) {  // the replica's growth counts as a signal of the next local round
             sigma[v] = t;
             signal_vertex(b, (uint32_t)v);  // (the bitmap sparse rounds read)
+            cnt++;
+        }
+    }
+    for (int off = 16; off; off >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, off);
+    if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(&ctr->active[slot], cnt);
+}
+
+// ---- peer-memory boundary exchange (replaces pack + NCCL all-reduce + unpack)
+// Every rank owns one exchange region in its HBM, mapped into every peer by
+// CUDA IPC (NVLink/NVSwitch loads and stores between B200s):
+//   [flags: kP2PMaxRanks x u64 epochs written by the peers | error word]
+//   [slot 0: n_bnd x u64][slot 1: n_bnd x u64]      (double buffer by epoch parity)
+// Exchange e: (1) pack this rank's boundary values into its own slot e&1;
+// (2) one warp publishes epoch e into every peer's flag word for this rank
+// (release, system scope) and waits until every peer published e here
+// (acquire); (3) every rank reduces all ranks' slot e&1 elementwise (MIN, or
+// SUM of growth) straight from peer memory and applies it like unpack.  A
+// rank rewrites slot e&1 only at exchange e+2, after every peer published
+// e+1, i.e. after every peer's exchange-e reduce completed (stream order).
+constexpr int kP2PMaxRanks = 16;
+constexpr size_t kP2PHeader = 256;  // bytes: flags + error word
+struct PeerSlots {
+    const void* p[kP2PMaxRanks];
+};
+__global__ void p2p_pack_min_kernel(const uint32_t* vs, const int32_t* bnd, int64_t nb, unsigned long long* slot) {
+    GRID_STRIDE(k, nb) slot[k] = vs[bnd[k]];
+}
+__global__ void p2p_pack_sum_kernel(const unsigned long long* vs, const int32_t* bnd, int64_t nb,
+                                    const unsigned long long* base, unsigned long long* slot) {
+    GRID_STRIDE(k, nb) slot[k] = vs[bnd[k]] - base[k];
+}
+__global__ void p2p_signal_wait_kernel(PeerSlots flags, int world, int rank, unsigned long long epoch,
+                                       unsigned long long* own_flags, unsigned long long timeout_ns) {
+    const int q = threadIdx.x;
+    if (q < world && q != rank) {
+        __threadfence_system();
+        unsigned long long* f = (unsigned long long*)flags.p[q] + rank;
+        asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(f), "l"(epoch) : "memory");
+    }
+    __syncwarp();
+    if (q < world && q != rank) {
+        unsigned long long t0, t, v;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+        while (true) {
+            asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(own_flags + q) : "memory");
+            if (v >= epoch) break;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+            if (t - t0 > timeout_ns) {  // a peer never arrived: report instead of hanging the GPU
+                atomicExch(own_flags + kP2PMaxRanks, 1ull);
+                break;
+            }
+            __nanosleep(256);
+        }
+    }
+}
+__global__ void p2p_reduce_min_kernel(PeerSlots slots, int world, uint32_t* vs, const int32_t* bnd, int64_t nb,
+                                      uint32_t* b, Counters* ctr, int slot) {
+    unsigned cnt = 0;
+    GRID_STRIDE(k, nb) {
+        unsigned long long m = ~0ull;
+        for (int r = 0; r < world; r++) m = min(m, __ldcv((const unsigned long long*)slots.p[r] + k));
+        const int v = bnd[k];
+        if ((uint32_t)m < vs[v]) {
+            vs[v] = (uint32_t)m;
+            cnt += signal_vertex(b, (uint32_t)v);
+        }
+    }
+    for (int off = 16; off; off >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, off);
+    if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(&ctr->active[slot], cnt);
+}
+__global__ void p2p_reduce_sum_kernel(PeerSlots slots, int world, unsigned long long* vs, unsigned long long* sigma,
+                                      const int32_t* bnd, int64_t nb, unsigned long long* base, unsigned long long eps,
+                                      uint32_t* b, Counters* ctr, int slot) {
+    unsigned cnt = 0;
+    GRID_STRIDE(k, nb) {
+        unsigned long long g = 0;
+        for (int r = 0; r < world; r++) g += __ldcv((const unsigned long long*)slots.p[r] + k);
+        const int v = bnd[k];
+        const unsigned long long t = base[k] + g;
+        base[k] = t;
+        vs[v] = t;
+        if (t - sigma[v] >= eps) {
+            sigma[v] = t;
+            signal_vertex(b, (uint32_t)v);
             cnt++;
         }
     }
@@ -1789,7 +1894,12 @@ int build_occ(DevWork* W, const DevLayout& D, uint32_t skip, uint32_t*& off, uin
     if (!off && (rc = dalloc(&off, D.n + 1, bytes, err))) return rc;
     if (!W->occ_cur && (rc = dalloc(&W->occ_cur, D.n + 1, bytes, err))) return rc;
     CK(cudaMemsetAsync(off, 0, sizeof(uint32_t) * (D.n + 1)));
-    occ_count_kernel<<<grid_1d(D.M), 256>>>(D.e_idx, D.M, skip, off);
+    int dev = 0, sms = 148;
+    CK(cudaGetDevice(&dev));
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    const int oblocks = (int)std::max<int64_t>(1, std::min<int64_t>((int64_t)sms * kOccBlocksPerSM, (D.M + 255) / 256));
+    const uint32_t hubs = (uint32_t)std::min<int64_t>(D.n, kOccHubs);
+    occ_count_kernel<<<oblocks, 256>>>(D.e_idx, D.M, skip, hubs, off);
     size_t tmp_bytes = 0;
     CK(cub::DeviceScan::InclusiveSum(nullptr, tmp_bytes, off, off, (int)(D.n + 1)));
     if (tmp_bytes > W->cub_tmp_bytes) {
@@ -1798,15 +1908,15 @@ int build_occ(DevWork* W, const DevLayout& D, uint32_t skip, uint32_t*& off, uin
         W->cub_tmp_bytes = tmp_bytes;
     }
     CK(cub::DeviceScan::InclusiveSum(W->cub_tmp, tmp_bytes, off, off, (int)(D.n + 1)));
-    uint32_t total = 0;
-    CK(cudaMemcpy(&total, off + D.n, sizeof(uint32_t), cudaMemcpyDeviceToHost));
-    if ((int64_t)total + 1 > cap) {
+    // capacity M + 1 bounds the occurrences (every path has a head and a
+    // tail), so the build needs no device->host round trip
+    if (D.M + 1 > cap) {
         dfree(occ);
-        if ((rc = dalloc(&occ, (size_t)total + 1, bytes, err))) return rc;
-        cap = (int64_t)total + 1;
+        if ((rc = dalloc(&occ, (size_t)D.M + 1, bytes, err))) return rc;
+        cap = D.M + 1;
     }
     CK(cudaMemcpyAsync(W->occ_cur, off, sizeof(uint32_t) * D.n, cudaMemcpyDeviceToDevice));
-    occ_fill_kernel<<<grid_1d(D.M), 256>>>(D.e_idx, D.M, skip, W->occ_cur, occ);
+    occ_fill_kernel<<<oblocks, 256>>>(D.e_idx, D.M, skip, hubs, W->occ_cur, occ);
     CK(cudaGetLastError());
     S.stats.kernel_launches += 3;
     if (verbose) {
@@ -1814,6 +1924,8 @@ int build_occ(DevWork* W, const DevLayout& D, uint32_t skip, uint32_t*& off, uin
         CK(cudaEventSynchronize(W->ev1));
         float ms = 0;
         CK(cudaEventElapsedTime(&ms, W->ev0, W->ev1));
+        uint32_t total = 0;
+        CK(cudaMemcpy(&total, off + D.n, sizeof(uint32_t), cudaMemcpyDeviceToHost));
         fprintf(stderr, "[dg] occurrence index (%s): %u entries in %.2f ms\n", skip == kTail ? "out" : "in", total, ms);
     }
     return DG_OK;
@@ -2276,6 +2388,101 @@ int dev_boundary_unpack(DevWork* W, const DevLayout& D, RunState& S, const void*
         S.stats.kernel_launches++;
         CK(cudaGetLastError());
     }
+    if ((rc = read_counters(W, c, err))) return rc;
+    *active = c.active[slot];
+    return DG_OK;
+}
+
+struct P2P {
+    int world = 0, rank = 0;
+    int64_t nb = 0;
+    unsigned long long epoch = 0;   // exchanges done (identical on every rank)
+    unsigned char* own = nullptr;   // this rank's exchange region (cudaMalloc)
+    unsigned char* peer[kP2PMaxRanks] = {};  // every rank's region in this address space (own included)
+    bool opened = false;
+};
+
+int dev_p2p_alloc(P2P*& X, const DevLayout& D, int world, int rank, void* handle, std::string& err) {
+    if (world < 2 || world > kP2PMaxRanks || rank < 0 || rank >= world) {
+        err = "p2p: world must be 2.." + std::to_string(kP2PMaxRanks) + " and 0 <= rank < world";
+        return DG_EINVAL;
+    }
+    dev_p2p_free(X);
+    X = new P2P();
+    X->world = world;
+    X->rank = rank;
+    X->nb = D.n_bnd;
+    const size_t bytes = kP2PHeader + 2 * sizeof(unsigned long long) * (size_t)std::max<int64_t>(D.n_bnd, 1);
+    CK(cudaMalloc(&X->own, bytes));
+    CK(cudaMemset(X->own, 0, bytes));  // epochs 0 before any peer can see the region
+    CK(cudaDeviceSynchronize());
+    cudaIpcMemHandle_t h;
+    CK(cudaIpcGetMemHandle(&h, X->own));
+    std::memcpy(handle, &h, sizeof(h));
+    return DG_OK;
+}
+
+int dev_p2p_open(P2P* X, const void* handles, std::string& err) {
+    if (!X) { err = "p2p: dg_p2p_alloc first"; return DG_EINVAL; }
+    for (int r = 0; r < X->world; r++) {
+        if (r == X->rank) { X->peer[r] = X->own; continue; }
+        if (X->peer[r]) continue;
+        cudaIpcMemHandle_t h;
+        std::memcpy(&h, (const unsigned char*)handles + (size_t)r * sizeof(h), sizeof(h));
+        void* ptr = nullptr;
+        CK(cudaIpcOpenMemHandle(&ptr, h, cudaIpcMemLazyEnablePeerAccess));
+        X->peer[r] = (unsigned char*)ptr;
+    }
+    X->opened = true;
+    return DG_OK;
+}
+
+void dev_p2p_free(P2P*& X) {
+    if (!X) return;
+    for (int r = 0; r < X->world; r++)
+        if (X->peer[r] && r != X->rank) cudaIpcCloseMemHandle(X->peer[r]);
+    if (X->own) cudaFree(X->own);
+    delete X;
+    X = nullptr;
+}
+
+int dev_boundary_exchange(DevWork* W, const DevLayout& D, RunState& S, P2P* X, int64_t* active, std::string& err) {
+    if (!X || !X->opened) { err = "dg_boundary_exchange: peers not opened (dg_p2p_open)"; return DG_EINVAL; }
+    if (X->nb != D.n_bnd) { err = "dg_boundary_exchange: layout changed since dg_p2p_alloc"; return DG_EINVAL; }
+    Counters c;
+    int rc;
+    if ((rc = read_counters(W, c, err))) return rc;
+    const int slot = c.round & 1;  // the bitmap the next local round reads
+    const unsigned long long e = ++X->epoch;
+    const size_t off = kP2PHeader + (size_t)(e & 1) * sizeof(unsigned long long) * (size_t)std::max<int64_t>(D.n_bnd, 1);
+    PeerSlots flags{}, slots{};
+    for (int r = 0; r < X->world; r++) {
+        flags.p[r] = X->peer[r];
+        slots.p[r] = X->peer[r] + off;
+    }
+    const bool sum = S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION;
+    unsigned long long* mine = (unsigned long long*)(X->own + off);
+    if (D.n_bnd) {
+        if (sum) p2p_pack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_t, D.bnd, D.n_bnd, W->bnd_base, mine);
+        else p2p_pack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, D.bnd, D.n_bnd, mine);
+    }
+    unsigned long long* own_flags = (unsigned long long*)X->own;
+    p2p_signal_wait_kernel<<<1, 32>>>(flags, X->world, X->rank, e, own_flags, 60ull * 1000000000ull);
+    if (D.n_bnd) {
+        uint32_t* b = W->bits + (int64_t)slot * W->nw;
+        if (sum)
+            p2p_reduce_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(slots, X->world, W->vs_t, W->sigma, D.bnd, D.n_bnd,
+                                                             W->bnd_base, (unsigned long long)(S.eps * 4294967296.0),
+                                                             b, W->ctr, slot);
+        else
+            p2p_reduce_min_kernel<<<grid_1d(D.n_bnd), 256>>>(slots, X->world, W->vs_u, D.bnd, D.n_bnd, b, W->ctr,
+                                                             slot);
+    }
+    S.stats.kernel_launches += D.n_bnd ? 3 : 1;
+    CK(cudaGetLastError());
+    unsigned long long timed_out = 0;
+    CK(cudaMemcpy(&timed_out, own_flags + kP2PMaxRanks, sizeof(timed_out), cudaMemcpyDeviceToHost));
+    if (timed_out) { err = "dg_boundary_exchange: a peer did not arrive within 60 s"; return DG_ETIMEOUT; }
     if ((rc = read_counters(W, c, err))) return rc;
     *active = c.active[slot];
     return DG_OK;

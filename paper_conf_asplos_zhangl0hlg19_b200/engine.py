@@ -66,6 +66,7 @@ class DiGraph:
         check(self._L.dg_load_csr(self._h, self.n, self.m, _p(self._row_ptr), _p(self._col), _p(self._w)),
               "dg_load_csr")
         self._row_ptr = self._col = self._w = None  # dg_load_csr copied them
+        self.p2p_key = None  # the library freed any exchange region
         return self
 
     def load_graph(self, g):
@@ -81,6 +82,7 @@ class DiGraph:
         p.merge_rule = {"paper": 0, "relaxed": 1}[merge_rule]
         p.n_proxy = n_proxy
         check(self._L.dg_build_paths(self._h, ctypes.byref(p)), "dg_build_paths")
+        self.p2p_key = None  # the library freed any exchange region
         return self
 
     def upload(self):
@@ -167,6 +169,26 @@ class DiGraph:
         a = ctypes.c_int64()
         check(self._L.dg_boundary_unpack(self._h, ctypes.c_void_p(buf.data_ptr()), ctypes.byref(a)),
               "dg_boundary_unpack")
+        return a.value
+
+    # ---- peer-memory boundary exchange (include/digraph.h dg_p2p_*) ----
+    P2P_HANDLE_BYTES = 64
+
+    def p2p_alloc(self, world, rank):
+        """Allocate this rank's exchange region; returns its IPC handle (bytes)."""
+        h = ctypes.create_string_buffer(self.P2P_HANDLE_BYTES)
+        check(self._L.dg_p2p_alloc(self._h, int(world), int(rank), h), "dg_p2p_alloc")
+        return h.raw
+
+    def p2p_open(self, handles):
+        """Map every peer's region; ``handles`` = list of IPC handles in rank order."""
+        blob = b"".join(handles)
+        assert len(blob) == self.P2P_HANDLE_BYTES * len(handles)
+        check(self._L.dg_p2p_open(self._h, ctypes.create_string_buffer(blob, len(blob))), "dg_p2p_open")
+
+    def boundary_exchange(self):
+        a = ctypes.c_int64()
+        check(self._L.dg_boundary_exchange(self._h, ctypes.byref(a)), "dg_boundary_exchange")
         return a.value
 
     def normalize_states(self, buf):

@@ -9,10 +9,15 @@ batches"):
      one NCCL all-reduce of the boundary over NVLink -- is amortised over a
      few rounds while replicas stay at most a few rounds apart), or fewer if
      its local active counter reaches zero;
-  2. boundary states are packed (device kernel) and all-reduced with NCCL:
-     MIN for SSSP/BFS/WCC, SUM of pending deltas for PageRank/Adsorption;
-  3. unpack (device kernel) re-activates partitions of changed vertices;
-  4. the activated-partition counts are all-reduced; zero everywhere = done.
+  2. boundary states are exchanged: MIN for SSSP/BFS/WCC, SUM of pending
+     deltas for PageRank/Adsorption.  ``exchange="p2p"`` (default): one
+     dg_boundary_exchange -- pack, device-side epoch flags and an elementwise
+     reduction read straight from every peer's HBM (CUDA IPC over
+     NVLink/NVSwitch), unpack; no host collective moves boundary states.
+     ``exchange="collective"``: pack kernel, ``dist.all_reduce`` of the
+     buffer (NCCL on GPUs, gloo in the CPU tests), unpack kernel;
+  3. unpack re-activates the changed vertices;
+  4. the activated counts are all-reduced (8 bytes); zero everywhere = done.
 
 The engine argument only needs the ``DiGraph`` protocol methods (run_begin,
 rounds, boundary_pack, boundary_unpack, run_end, get_states), so the host
@@ -33,25 +38,49 @@ def boundary_buffer(n_boundary, algo, device):
     return torch.zeros(max(int(n_boundary), 1), dtype=dtype, device=device)
 
 
+def p2p_setup(engine, group=None):
+    """Allocate this rank's exchange region and map every peer's (once per
+    layout): the 64-byte IPC handles travel through ``dist.all_gather_object``."""
+    world, rank = dist.get_world_size(group), dist.get_rank(group)
+    key = (world, rank, len(engine.boundary_vertices()))
+    if getattr(engine, "p2p_key", None) == key:
+        return
+    h = engine.p2p_alloc(world, rank)
+    hs = [None] * world
+    dist.all_gather_object(hs, h, group=group)
+    engine.p2p_open(hs)
+    engine.p2p_key = key
+
+
 def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_rounds=4,
-                    max_outer=1_000_000, device=None, group=None):
-    """Run ``algo`` to global convergence.  Returns (stats, sync_info)."""
+                    max_outer=1_000_000, device=None, group=None, exchange=None):
+    """Run ``algo`` to global convergence.  Returns (stats, sync_info).
+    ``exchange``: "p2p" (default on CUDA devices) or "collective"."""
     if algo not in SUM_ALGOS + MIN_ALGOS:
         raise ValueError(f"{algo}: no multi-rank protocol (SCC is single-rank)")
     device = device if device is not None else (torch.device("cuda", torch.cuda.current_device())
                                                 if torch.cuda.is_available() else torch.device("cpu"))
+    if exchange is None:
+        exchange = "p2p" if device.type == "cuda" else "collective"
+    if exchange not in ("p2p", "collective"):
+        raise ValueError(f"exchange={exchange!r}: 'p2p' or 'collective'")
     nb = len(engine.boundary_vertices())
     buf = boundary_buffer(nb, algo, device)
     op = dist.ReduceOp.SUM if algo in SUM_ALGOS else dist.ReduceOp.MIN
     active = torch.zeros(1, dtype=torch.int64, device=device)
     engine.run_begin(algo, source=source, epsilon=epsilon, damping=damping)
+    if exchange == "p2p":
+        p2p_setup(engine, group)
     syncs, bytes_per_sync = 0, buf.numel() * buf.element_size()
     for _ in range(max_outer):
         engine.rounds(local_rounds)
-        if nb:
-            engine.boundary_pack(buf)
-        dist.all_reduce(buf, op=op, group=group)
-        act = engine.boundary_unpack(buf)
+        if exchange == "p2p":
+            act = engine.boundary_exchange()
+        else:
+            if nb:
+                engine.boundary_pack(buf)
+            dist.all_reduce(buf, op=op, group=group)
+            act = engine.boundary_unpack(buf)
         syncs += 1
         active.fill_(int(act))
         dist.all_reduce(active, op=dist.ReduceOp.SUM, group=group)
@@ -60,7 +89,9 @@ def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_ro
     else:
         raise RuntimeError("multi-rank run did not converge")
     stats = engine.run_end()
-    return stats, {"syncs": syncs, "boundary": nb, "nvlink_bytes_per_sync": bytes_per_sync}
+    if exchange == "p2p":  # every rank reads each peer's 8-byte slot per boundary vertex
+        bytes_per_sync = 8 * nb * (dist.get_world_size(group) - 1)
+    return stats, {"syncs": syncs, "boundary": nb, "nvlink_bytes_per_sync": bytes_per_sync, "exchange": exchange}
 
 
 def gather_states(engine, algo, n, device=None, group=None):

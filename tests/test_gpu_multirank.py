@@ -1,7 +1,8 @@
-"""-m gpu: the real multi-rank device path (dg_run_begin / dg_rounds /
-dg_boundary_pack / dg_boundary_unpack kernels + parallel.py) with two ranks
-time-sharing cuda:0.  NCCL refuses two ranks on one GPU, so the collective
-here is gloo on CUDA tensors; on an 8-GPU box bench.py uses NCCL."""
+"""-m gpu: the real multi-rank device path (dg_run_begin / dg_rounds and
+either the peer-memory exchange dg_boundary_exchange -- CUDA IPC between the
+two processes, device-side epoch flags -- or dg_boundary_pack / all-reduce /
+dg_boundary_unpack) with two ranks time-sharing cuda:0.  NCCL refuses two
+ranks on one GPU, so the host collective here is gloo on CUDA tensors."""
 import os
 import socket
 
@@ -29,7 +30,7 @@ def _graph():
     return inputs.rmat(13, 8192, 80000, seed=31)
 
 
-def _worker(rank, world, port, algo, q, sparse=False):
+def _worker(rank, world, port, algo, q, sparse=False, exchange="p2p"):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     if sparse:  # every round with <= n/4 signalled vertices walks sparse
         os.environ.update(DG_SPARSE_DIV="1", DG_SPARSE_MIN_M="0")
@@ -40,7 +41,7 @@ def _worker(rank, world, port, algo, q, sparse=False):
     dg = DiGraph(device=0)
     dg.load_graph(g).build_paths(part_entries=256, rank=rank, world=world)
     dev = torch.device("cuda", 0)
-    stats, info = parallel.run_distributed(dg, algo, source=0, epsilon=1e-7, device=dev)
+    stats, info = parallel.run_distributed(dg, algo, source=0, epsilon=1e-7, device=dev, exchange=exchange)
     out = parallel.gather_states(dg, algo, g.n, device=dev)
     if rank == 0:
         q.put((out.cpu().numpy().copy(), info, stats))
@@ -48,13 +49,14 @@ def _worker(rank, world, port, algo, q, sparse=False):
     dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("exchange", ["p2p", "collective"])
 @pytest.mark.parametrize("sparse", [False, True])
 @pytest.mark.parametrize("algo", ["sssp", "wcc", "pagerank"])
-def test_two_ranks_on_one_gpu_match_oracle(algo, sparse, cuda_required):
+def test_two_ranks_on_one_gpu_match_oracle(algo, sparse, exchange, cuda_required):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, algo, q, sparse)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, algo, q, sparse, exchange)) for r in range(2)]
     for p in procs:
         p.start()
     got, info, stats = q.get(timeout=600)
@@ -63,7 +65,7 @@ def test_two_ranks_on_one_gpu_match_oracle(algo, sparse, cuda_required):
         assert p.exitcode == 0
     g = _graph()
     src, dst, w = g.edges()
-    assert info["boundary"] > 0
+    assert info["boundary"] > 0 and info["exchange"] == exchange
     if algo == "sssp":
         exp, _ = OA.sssp_bellman_ford(g.n, src, dst, w, 0)
         assert np.array_equal(got.view(np.uint32).astype(np.int64), exp)

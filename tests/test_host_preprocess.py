@@ -158,3 +158,19 @@ def test_bad_arguments_are_rejected():
         dg.load_csr(3, np.array([0, 1, 2, 9]), np.array([1, 2, 0]))
     with pytest.raises(DGError, match="DG_EINVAL"):
         dg.load_csr(3, np.array([0, 1, 2, 3]), np.array([1, 2, 7]))
+
+
+def test_p2p_exchange_lifecycle_is_checked():
+    """dg_p2p_alloc needs an uploaded layout, dg_p2p_open an allocated region,
+    dg_boundary_exchange a run in progress (include/digraph.h)."""
+    dg = DiGraph()
+    with pytest.raises(DGError, match="DG_EINVAL"):
+        dg.p2p_alloc(2, 0)
+    dg.load_graph(fig4_graph())
+    dg.build_paths(rank=0, world=2)
+    with pytest.raises(DGError, match="DG_EINVAL"):
+        dg.p2p_alloc(2, 0)  # not uploaded
+    with pytest.raises(DGError, match="DG_EINVAL"):
+        dg.p2p_open([b"\0" * 64, b"\0" * 64])
+    with pytest.raises(DGError, match="DG_EINVAL"):
+        dg.boundary_exchange()
