@@ -373,7 +373,7 @@ def main():
                          "d2h_bytes_per_step": d2h, "ms_per_step": e2e_s * 1e3}
     if not args.no_extras and rank == 0 and world == 1:
         # vertex-centric ablation (north_star: total vertex updates next to it)
-        if args.algo in ("pagerank", "sssp", "bfs"):
+        if args.algo in ("pagerank", "sssp", "bfs", "wcc"):
             other = "vertex" if args.mode == "path" else "path"
             ab_st = dg.run(args.algo, mode=other, **run_kw)
             extras["ablation"] = {"mode": other, "ms": ab_st["time_ms"], "rounds": ab_st["rounds"],

@@ -169,7 +169,8 @@ int dg_set_vertex_params(dg_graph *g, const double *p_inj, const double *p_cont,
  *            < 0 = unbounded,
  *            > 0 = that width.  Results are exact for every value; it trades
  *            redundant updates against rounds.  Ignored by the others.
- *   mode     DG_MODE_PATH or DG_MODE_VERTEX (ablation)
+ *   mode     DG_MODE_PATH or DG_MODE_VERTEX (ablation: SSSP, BFS, PageRank,
+ *            WCC -- WCC pushes labels over both edge directions)
  *   max_rounds  safety cap (<= 0: 1,000,000)
  *   stats    may be NULL
  * States stay on the device until dg_get_states.  Single-rank only: with

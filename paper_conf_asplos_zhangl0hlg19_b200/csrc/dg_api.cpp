@@ -166,12 +166,38 @@ static int ensure_uploaded(dg_graph* g) {
     return g->uploaded ? DG_OK : dg_upload(g);
 }
 
+// The CSR of both edge directions (internal ids), for the WCC ablation:
+// vertex x lists its out-neighbours, then its in-neighbours.
+static void build_sym_csr(dg::HostLayout& L, int64_t n) {
+    if (!L.srow_ptr.empty()) return;
+    std::vector<int64_t> rp(n + 1, 0);
+    for (int64_t u = 0; u < n; u++) {
+        rp[u + 1] += L.prow_ptr[u + 1] - L.prow_ptr[u];
+        for (int64_t e = L.prow_ptr[u]; e < L.prow_ptr[u + 1]; e++) rp[L.pcol[e] + 1]++;
+    }
+    for (int64_t u = 0; u < n; u++) rp[u + 1] += rp[u];
+    std::vector<int32_t> col(rp[n]);
+    std::vector<int64_t> cur(rp.begin(), rp.end() - 1);
+    for (int64_t u = 0; u < n; u++)
+        for (int64_t e = L.prow_ptr[u]; e < L.prow_ptr[u + 1]; e++) col[cur[u]++] = L.pcol[e];
+    for (int64_t u = 0; u < n; u++)
+        for (int64_t e = L.prow_ptr[u]; e < L.prow_ptr[u + 1]; e++) col[cur[L.pcol[e]]++] = (int32_t)u;
+    L.srow_ptr.swap(rp);
+    L.scol.swap(col);
+}
+
 // the parts of the device layout an algorithm reads beyond the path entries
 static int ensure_parts(dg_graph* g, int algo, int mode) {
-    const bool need_csr = mode == DG_MODE_VERTEX || algo == DG_ADSORPTION;
+    const bool need_sym = mode == DG_MODE_VERTEX && algo == DG_WCC;
+    const bool need_csr = (mode == DG_MODE_VERTEX && !need_sym) || algo == DG_ADSORPTION;
     const bool need_ew = (mode == DG_MODE_PATH && algo == DG_SSSP) || algo == DG_ADSORPTION;
     std::string err;
-    int rc = dg::dev_ensure_parts(g->dev, g->csr, g->layout, need_csr, need_ew, err);
+    try {
+        if (need_sym) build_sym_csr(g->layout, g->csr.n);
+    } catch (const std::bad_alloc&) {
+        return fail(DG_ENOMEM, "dg_run: out of host memory (WCC ablation CSR)");
+    }
+    int rc = dg::dev_ensure_parts(g->dev, g->csr, g->layout, need_csr, need_ew, need_sym, err);
     return rc ? fail(rc, err) : DG_OK;
 }
 
@@ -213,8 +239,8 @@ static int check_run_args(dg_graph* g, int algo, int64_t source, double epsilon,
     if (algo == DG_PAGERANK && !(param > 0 && param < 1)) return fail(DG_EINVAL, "dg_run: damping must be in (0,1)");
     if ((algo == DG_PAGERANK || algo == DG_ADSORPTION) && !(epsilon > 0))
         return fail(DG_EINVAL, "dg_run: epsilon must be > 0");
-    if (mode == DG_MODE_VERTEX && algo != DG_SSSP && algo != DG_BFS && algo != DG_PAGERANK)
-        return fail(DG_EINVAL, "dg_run: the vertex-centric ablation supports SSSP, BFS and PageRank");
+    if (mode == DG_MODE_VERTEX && algo != DG_SSSP && algo != DG_BFS && algo != DG_PAGERANK && algo != DG_WCC)
+        return fail(DG_EINVAL, "dg_run: the vertex-centric ablation supports SSSP, BFS, PageRank and WCC");
     return DG_OK;
 }
 

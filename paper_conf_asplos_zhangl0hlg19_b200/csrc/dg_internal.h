@@ -47,6 +47,8 @@ struct HostLayout {
     std::vector<int32_t> new_id, orig;  // original -> internal, internal -> original
     std::vector<int64_t> prow_ptr;
     std::vector<int32_t> pcol, pw, poutdeg;
+    std::vector<int64_t> srow_ptr;       // both directions (WCC ablation), built on first use
+    std::vector<int32_t> scol;
     // multi-rank
     std::vector<int32_t> boundary;      // internal ids of vertices present on >1 rank (ascending)
     // stats
@@ -69,9 +71,10 @@ struct DevLayout {
     // CSR (for the vertex-centric ablation and per-vertex coefficients)
     int64_t* row_ptr = nullptr; int32_t* col = nullptr; int32_t* w = nullptr;
     int32_t* outdeg = nullptr;
+    int64_t* srow_ptr = nullptr; int32_t* scol = nullptr;  // both directions (WCC ablation)
     int64_t bytes = 0;      // device bytes allocated
     int64_t h2d_bytes = 0;  // bytes copied host -> device since the last dg_upload
-    bool csr_ok = false, ew_ok = false;  // lazily uploaded parts present
+    bool csr_ok = false, ew_ok = false, sym_ok = false;  // lazily uploaded parts present
     std::vector<void*> pinned;  // host buffers page-locked with cudaHostRegister
 };
 void dev_unpin_all(DevLayout& D);
@@ -92,7 +95,8 @@ struct RunState {
 int dev_select(int device, std::string& err);
 int dev_upload_csr(DevLayout& D, const HostCSR& g, const HostLayout& L, std::string& err);
 int dev_upload_layout(DevLayout& D, const HostLayout& L, std::string& err);
-int dev_ensure_parts(DevLayout& D, const HostCSR& g, const HostLayout& L, bool need_csr, bool need_ew, std::string& err);
+int dev_ensure_parts(DevLayout& D, const HostCSR& g, const HostLayout& L, bool need_csr, bool need_ew, bool need_sym,
+                     std::string& err);
 void dev_free_layout(DevLayout& D, bool csr_too);
 int dev_set_vertex_params(DevWork*& W, const DevLayout& D, const double* p_inj, const double* p_cont,
                           const double* inj, std::string& err);

@@ -1372,7 +1372,8 @@ __global__ void __launch_bounds__(kBlock) vertex_kernel(KParams P) {
                     acc.upd++;
                     push = old < P.eps && old + a >= P.eps;
                 } else {
-                    uint32_t cand = sat_add(s_dist[wid][lo], ALGO == DG_BFS ? 1u : (uint32_t)P.w[e]);
+                    const uint32_t cand = ALGO == DG_WCC ? s_dist[wid][lo]
+                                        : sat_add(s_dist[wid][lo], ALGO == DG_BFS ? 1u : (uint32_t)P.w[e]);
                     if (cand < P.vs_u[x]) {
                         uint32_t old = atomicMin(&P.vs_u[x], cand);
                         if (cand < old) { acc.upd++; push = true; }
@@ -2010,7 +2011,12 @@ int launch_vertex(DevWork* W, const DevLayout& D, int algo, int rounds, RunState
     P.eps = (float)S.eps;
     P.max_rounds = rounds;
     void* fn = algo == DG_PAGERANK ? (void*)vertex_kernel<DG_PAGERANK>
-             : algo == DG_BFS ? (void*)vertex_kernel<DG_BFS> : (void*)vertex_kernel<DG_SSSP>;
+             : algo == DG_BFS ? (void*)vertex_kernel<DG_BFS>
+             : algo == DG_WCC ? (void*)vertex_kernel<DG_WCC> : (void*)vertex_kernel<DG_SSSP>;
+    if (algo == DG_WCC) {  // labels cross every edge in both directions
+        P.row_ptr = D.srow_ptr;
+        P.col = D.scol;
+    }
     return coop_launch(W, fn, P, S, err);
 }
 
@@ -2022,6 +2028,11 @@ int init_states(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
         // frontier: the source (SSSP/BFS) or every vertex (PageRank)
         if (algo == DG_PAGERANK) {
             init_pr_kernel<<<g, 256>>>(W->vs_f, D.outdeg, D.n, (float)S.param);
+            fill_iota_kernel<<<g, 256>>>(W->vlist[0], D.n);
+            c.active[0] = (unsigned)D.n;
+            S.stats.kernel_launches += 2;
+        } else if (algo == DG_WCC) {  // every vertex starts with its own label, all in the frontier
+            init_u_kernel<<<g, 256>>>(W->vs_u, W->vstamp, D.orig, D.n, algo, 0);
             fill_iota_kernel<<<g, 256>>>(W->vlist[0], D.n);
             c.active[0] = (unsigned)D.n;
             S.stats.kernel_launches += 2;
@@ -2186,7 +2197,7 @@ int dev_upload_csr(DevLayout& D, const HostCSR& g, const HostLayout& L, std::str
     return DG_OK;
 }
 
-int dev_ensure_parts(DevLayout& D, const HostCSR& g, const HostLayout& L, bool need_csr, bool need_ew,
+int dev_ensure_parts(DevLayout& D, const HostCSR& g, const HostLayout& L, bool need_csr, bool need_ew, bool need_sym,
                      std::string& err) {
     int rc;
     g_h2d_counter = &D.h2d_bytes;
@@ -2201,6 +2212,14 @@ int dev_ensure_parts(DevLayout& D, const HostCSR& g, const HostLayout& L, bool n
             if ((rc = h2d(D.w, L.pw.data(), g.m, err))) return rc;
         }
         D.csr_ok = true;
+    }
+    if (need_sym && !D.sym_ok) {  // the CSR of both directions (dg_api.cpp builds it on the host)
+        const int64_t ms = (int64_t)L.scol.size();
+        if ((rc = dalloc_once(&D.srow_ptr, g.n + 1, D.bytes, err))) return rc;
+        if ((rc = dalloc_once(&D.scol, ms + kPad, D.bytes, err))) return rc;
+        if ((rc = h2d(D.srow_ptr, L.srow_ptr.data(), g.n + 1, err))) return rc;
+        if ((rc = h2d(D.scol, L.scol.data(), ms, err))) return rc;
+        D.sym_ok = true;
     }
     if (need_ew && !D.ew_ok) {
         if ((rc = dalloc_once(&D.e_w, D.M + kPad, D.bytes, err))) return rc;
@@ -2245,7 +2264,11 @@ void dev_unpin_all(DevLayout& D) {
 
 void dev_free_layout(DevLayout& D, bool csr_too) {
     dfree(D.e_idx); dfree(D.e_w); dfree(D.part_off); dfree(D.bnd);
-    if (csr_too) { dfree(D.row_ptr); dfree(D.col); dfree(D.w); dfree(D.outdeg); dfree(D.new_id); dfree(D.orig); }
+    if (csr_too) {
+        dfree(D.row_ptr); dfree(D.col); dfree(D.w); dfree(D.outdeg); dfree(D.new_id); dfree(D.orig);
+        dfree(D.srow_ptr); dfree(D.scol);
+        D.sym_ok = false;
+    }
     D.bytes = 0;
     D.M = D.n_part = D.n_bnd = 0;
     D.csr_ok = D.ew_ok = false;

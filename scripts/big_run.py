@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """Large-config run (configs[2..4] at N=1): generate once, preprocess once,
 time each algorithm to convergence (3 timed runs after 2 warm-ups), and one
-vertex-centric ablation run for SSSP / BFS / PageRank (vertex updates next to
+vertex-centric ablation run for SSSP / BFS / PageRank / WCC (vertex updates next to
 the path kernel's).  Prints one JSON object.
 
   python scripts/big_run.py <config> <algo,algo,...> [--no-ablation]
@@ -40,7 +40,7 @@ for algo in algos:
                  "vertex_updates": st["vertex_updates"], "entries_processed": st["entries_processed"],
                  "kernel_ms": st["kernel_ms"]}
     print(f"[big] {algo}: {res[algo]}", file=sys.stderr, flush=True)
-    if ablation and algo in ("pagerank", "sssp", "bfs"):
+    if ablation and algo in ("pagerank", "sssp", "bfs", "wcc"):
         st = dg.run(algo, source=0, mode="vertex")
         res[algo]["ablation_vertex_centric"] = {"ms": st["time_ms"], "rounds": st["rounds"],
                                                 "vertex_updates": st["vertex_updates"],

@@ -86,6 +86,12 @@ def test_wcc_fullsize_exact(lj):
     A = sp.csr_matrix((np.ones(len(src)), (src, dst)), shape=(g.n, g.n))
     _, lab = connected_components(A, directed=True, connection="weak")
     assert np.array_equal(got, canonical(lab))
+    # the vertex-centric ablation (labels over both directions) agrees and
+    # needs more label writes than the path walk
+    st_v = dg.run("wcc", mode="vertex")
+    assert np.array_equal(dg.get_states().astype(np.int64), got)
+    st_p = dg.run("wcc")
+    assert st_p["vertex_updates"] <= st_v["vertex_updates"], (st_p, st_v)
 
 
 def test_scc_fullsize_exact(lj):

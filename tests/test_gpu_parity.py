@@ -105,10 +105,11 @@ def test_pagerank_within_tolerance(name, kw, mode):
 
 
 @pytest.mark.parametrize("name", ["rmat12", "uniform_dup", "chains"])
-def test_wcc_bit_exact(name):
+@pytest.mark.parametrize("mode", ["path", "vertex"])
+def test_wcc_bit_exact(name, mode):
     g = G(name)
     dg = engine(g)
-    dg.run("wcc")
+    dg.run("wcc", mode=mode)
     got = dg.get_states().astype(np.int64)
     src, dst, _ = g.edges()
     exp, _ = OA.wcc_label_propagation(g.n, src, dst)
