@@ -38,18 +38,37 @@ def boundary_buffer(n_boundary, algo, device):
     return torch.zeros(max(int(n_boundary), 1), dtype=dtype, device=device)
 
 
-def p2p_setup(engine, group=None):
+def p2p_setup(engine, group=None, device=None):
     """Allocate this rank's exchange region and map every peer's (once per
-    layout): the 64-byte IPC handles travel through ``dist.all_gather_object``."""
+    layout): the 64-byte IPC handles travel through ``dist.all_gather_object``.
+    Returns None when every rank mapped every peer, else the first error (all
+    ranks agree, so they all fall back to the collective exchange together --
+    e.g. when each process sees only its own GPU and CUDA IPC cannot map a
+    peer's memory)."""
     world, rank = dist.get_world_size(group), dist.get_rank(group)
     key = (world, rank, len(engine.boundary_vertices()))
     if getattr(engine, "p2p_key", None) == key:
-        return
-    h = engine.p2p_alloc(world, rank)
+        return None
+    err = None
+    try:
+        h = engine.p2p_alloc(world, rank)
+    except Exception as e:  # noqa: BLE001 -- reported to every rank below
+        h, err = b"", f"dg_p2p_alloc: {e}"
     hs = [None] * world
     dist.all_gather_object(hs, h, group=group)
-    engine.p2p_open(hs)
-    engine.p2p_key = key
+    if err is None and all(len(x) == len(h) for x in hs):
+        try:
+            engine.p2p_open(hs)
+        except Exception as e:  # noqa: BLE001
+            err = f"dg_p2p_open: {e}"
+    elif err is None:
+        err = "a peer failed dg_p2p_alloc"
+    errs = [None] * world
+    dist.all_gather_object(errs, err, group=group)
+    first = next((e for e in errs if e), None)
+    if first is None:
+        engine.p2p_key = key
+    return first
 
 
 def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_rounds=4,
@@ -69,8 +88,14 @@ def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_ro
     op = dist.ReduceOp.SUM if algo in SUM_ALGOS else dist.ReduceOp.MIN
     active = torch.zeros(1, dtype=torch.int64, device=device)
     engine.run_begin(algo, source=source, epsilon=epsilon, damping=damping)
+    p2p_error = None
     if exchange == "p2p":
-        p2p_setup(engine, group)
+        p2p_error = p2p_setup(engine, group)
+        if p2p_error:
+            import sys
+            print(f"[parallel] peer-memory exchange unavailable ({p2p_error}); using the collective",
+                  file=sys.stderr, flush=True)
+            exchange = "collective"
     syncs, bytes_per_sync = 0, buf.numel() * buf.element_size()
     for _ in range(max_outer):
         engine.rounds(local_rounds)
@@ -91,7 +116,10 @@ def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_ro
     stats = engine.run_end()
     if exchange == "p2p":  # every rank reads each peer's 8-byte slot per boundary vertex
         bytes_per_sync = 8 * nb * (dist.get_world_size(group) - 1)
-    return stats, {"syncs": syncs, "boundary": nb, "nvlink_bytes_per_sync": bytes_per_sync, "exchange": exchange}
+    info = {"syncs": syncs, "boundary": nb, "nvlink_bytes_per_sync": bytes_per_sync, "exchange": exchange}
+    if p2p_error:
+        info["p2p_error"] = p2p_error
+    return stats, info
 
 
 def gather_states(engine, algo, n, device=None, group=None):

@@ -160,13 +160,27 @@ def _free_port():
     return port
 
 
-def _worker(rank, world, port, algo, q):
+class NoPeerEngine(CpuPathEngine):
+    """Peer mapping fails on rank 1 only (as when a process cannot see its
+    peers' GPUs): every rank must fall back to the collective together."""
+
+    def p2p_alloc(self, world, rank):
+        if rank == 1:
+            raise RuntimeError("no peer access")
+        return b"h" * 64
+
+    def p2p_open(self, handles):
+        raise AssertionError("must not be reached: rank 1 failed dg_p2p_alloc")
+
+
+def _worker(rank, world, port, algo, q, exchange=None):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     from paper_conf_asplos_zhangl0hlg19_b200 import parallel
     g = inputs.rmat(10, 1024, 6000, seed=21, weights=(1, 20))
-    eng = CpuPathEngine(g, rank, world)
-    stats, info = parallel.run_distributed(eng, algo, source=0, epsilon=1e-7, device=torch.device("cpu"))
+    eng = (NoPeerEngine if exchange == "p2p" else CpuPathEngine)(g, rank, world)
+    stats, info = parallel.run_distributed(eng, algo, source=0, epsilon=1e-7, device=torch.device("cpu"),
+                                           exchange=exchange)
     out = parallel.gather_states(eng, algo, g.n, device=torch.device("cpu"))
     if rank == 0:
         q.put((out.numpy().copy(), info))
@@ -174,12 +188,12 @@ def _worker(rank, world, port, algo, q):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("algo", ["sssp", "wcc", "pagerank"])
-def test_two_rank_protocol_matches_oracle(algo):
+@pytest.mark.parametrize("algo,exchange", [("sssp", None), ("wcc", None), ("pagerank", None), ("sssp", "p2p")])
+def test_two_rank_protocol_matches_oracle(algo, exchange):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, 2, port, algo, q)) for r in range(2)]
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, algo, q, exchange)) for r in range(2)]
     for p in procs:
         p.start()
     got, info = q.get(timeout=300)
@@ -189,6 +203,8 @@ def test_two_rank_protocol_matches_oracle(algo):
     g = inputs.rmat(10, 1024, 6000, seed=21, weights=(1, 20))
     src, dst, w = g.edges()
     assert info["boundary"] > 0 and info["syncs"] >= 1
+    assert info["exchange"] == "collective"
+    assert ("p2p_error" in info) == (exchange == "p2p")
     if algo == "sssp":
         exp, _ = OA.sssp_bellman_ford(g.n, src, dst, w, 0)
         assert np.array_equal(got.astype(np.int64), exp)
