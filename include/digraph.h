@@ -271,6 +271,20 @@ int dg_p2p_alloc(dg_graph *g, int world, int rank, void *handle);
 int dg_p2p_open(dg_graph *g, const void *handles);
 int dg_boundary_exchange(dg_graph *g, int64_t *active);
 
+/* The whole multi-rank run in ONE kernel launch per rank (after
+ * dg_run_begin and dg_p2p_open, before dg_run_end): the persistent
+ * propagation kernel performs the same peer-memory exchange itself after
+ * every `local_rounds` rounds (or as soon as this rank has no work), and
+ * stops when every rank published zero activity (no signalled vertex and
+ * no boundary value changed since the previous exchange) at the same
+ * exchange -- the global convergence test runs on the devices, no host
+ * collective.  SSSP, BFS, WCC, PageRank, Adsorption.  Every rank must call
+ * it together (the kernels rendezvous through the epoch flags).
+ *   *exchanges  exchanges performed; *converged 1 if globally converged
+ *   (0: max_rounds reached).  DG_ETIMEOUT if a peer did not arrive within
+ *   60 s. */
+int dg_run_fused(dg_graph *g, int64_t local_rounds, int64_t max_rounds, int64_t *exchanges, int64_t *converged);
+
 #ifdef __cplusplus
 }
 #endif

@@ -24,7 +24,7 @@ EXPORTS = [
     "dg_build_paths", "dg_upload", "dg_set_vertex_params", "dg_run", "dg_get_states",
     "dg_get_layout_info", "dg_export_paths", "dg_boundary_size", "dg_boundary_vertices",
     "dg_run_begin", "dg_rounds", "dg_boundary_pack", "dg_boundary_unpack", "dg_run_end",
-    "dg_normalize_states", "dg_p2p_alloc", "dg_p2p_open", "dg_boundary_exchange",
+    "dg_normalize_states", "dg_p2p_alloc", "dg_p2p_open", "dg_boundary_exchange", "dg_run_fused",
 ]
 
 
@@ -99,6 +99,7 @@ def lib():
         "dg_p2p_alloc": (i32, [P, i32, i32, P]),
         "dg_p2p_open": (i32, [P, P]),
         "dg_boundary_exchange": (i32, [P, pp(i64)]),
+        "dg_run_fused": (i32, [P, i64, i64, pp(i64), pp(i64)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)

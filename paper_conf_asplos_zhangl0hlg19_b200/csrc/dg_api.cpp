@@ -408,6 +408,15 @@ int dg_boundary_exchange(dg_graph* g, int64_t* active) {
     return rc ? fail(rc, err) : DG_OK;
 }
 
+int dg_run_fused(dg_graph* g, int64_t local_rounds, int64_t max_rounds, int64_t* exchanges, int64_t* converged) {
+    if (!g || !g->multi_active || !exchanges || !converged) return fail(DG_EINVAL, "dg_run_fused: no run in progress");
+    if (int rc0 = select_dev(g)) return rc0;
+    std::string err;
+    int rc = dg::dev_run_fused(g->work, g->dev, g->run, g->p2p, local_rounds, max_rounds <= 0 ? 1000000 : max_rounds,
+                               exchanges, converged, err);
+    return rc ? fail(rc, err) : DG_OK;
+}
+
 int dg_run_end(dg_graph* g, dg_run_stats* stats) {
     if (!g || !g->multi_active) return fail(DG_EINVAL, "dg_run_end: no run in progress");
     if (int rc0 = select_dev(g)) return rc0;

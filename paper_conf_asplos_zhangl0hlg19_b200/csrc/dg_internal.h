@@ -111,6 +111,8 @@ int dev_p2p_alloc(P2P*& X, const DevLayout& D, int world, int rank, void* handle
 int dev_p2p_open(P2P* X, const void* handles, std::string& err);
 void dev_p2p_free(P2P*& X);
 int dev_boundary_exchange(DevWork* W, const DevLayout& D, RunState& S, P2P* X, int64_t* active, std::string& err);
+int dev_run_fused(DevWork* W, const DevLayout& D, RunState& S, P2P* X, int64_t local_rounds, int64_t max_rounds,
+                  int64_t* exchanges, int64_t* converged, std::string& err);
 int dev_normalize(void* buf, int64_t n, std::string& err);
 int dev_get_states(DevWork* W, const DevLayout& D, const RunState& S, void* out, int64_t n, int out_is_device,
                    std::string& err);

@@ -70,6 +70,11 @@ struct Counters {
     unsigned int qn_in[2], osum_in[2], qcur_in[2], ticket_in[2];  // WCC sparse rounds: the in-edge phase
     int round;  // global round number of the next round
     int pad;
+    // fused multi-rank runs (path_kernel with P.mr.world > 1)
+    unsigned long long mr_dirty;  // boundary values changed since the last exchange (this rank)
+    unsigned long long mr_total;  // all ranks' published activity at the last exchange
+    unsigned long long mr_ex;     // exchanges done by the last launch
+    unsigned long long mr_err;    // a peer did not arrive (timeout)
 };
 
 struct DevWork {
@@ -106,6 +111,24 @@ struct DevWork {
     bool occ_ok = false;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr, kev0 = nullptr, kev1 = nullptr;
     bool have_params = false;
+};
+
+// Peer-memory exchange region (see "peer-memory boundary exchange" below):
+// header (u64 words): [0, kP2PMaxRanks) epochs written by the peers, [16]
+// error word, [17 + parity] this rank's published activity; then two slots.
+constexpr int kP2PMaxRanks = 16;
+constexpr size_t kP2PHeader = 256;
+constexpr int kP2PErr = kP2PMaxRanks, kP2PCount = kP2PMaxRanks + 1;
+// Fused multi-rank run: the exchange happens inside path_kernel's round loop.
+struct MultiRank {
+    const unsigned char* region[kP2PMaxRanks];  // every rank's region in this address space (own included)
+    unsigned long long* own;                    // this rank's region
+    const int32_t* bnd;                         // boundary vertices (internal ids), identical on every rank
+    unsigned long long* base;                   // SUM: total after the last exchange
+    uint32_t* last;                             // MIN: reduced value of the last exchange
+    int64_t nb;
+    unsigned long long slot_bytes, epoch0, timeout_ns, eps_fx;
+    int world, rank, every, sum;
 };
 
 struct KParams {
@@ -146,6 +169,7 @@ struct KParams {
     uint32_t sparse_max;      // rounds with at most this many signalled vertices are candidates (n/4)
     uint32_t sparse_occ;      // ... and are walked sparse if their out-edges are at most this many
     int sparse_walk;          // path edges a sparse walk follows at most
+    MultiRank mr;             // world > 1: fused multi-rank run
 };
 
 // ------------------------------------------------------------------ helpers
@@ -1144,7 +1168,113 @@ __device__ void walk_scc_bwd(const KParams& P, int64_t beg, int64_t end, const u
 // hub) then the per-warp 2 x 128-entry master ring (kWarps x 4 KB).
 constexpr size_t kGbufBytes = (size_t)kWarps * 2 * 128 * sizeof(uint4);
 
-template <int ALGO, int MINB = DG_PATH_MINB>
+// ---- fused multi-rank exchange (P.mr.world > 1; DESIGN.md "Peer-memory
+// exchange"): the same protocol as dg_boundary_exchange, run by the
+// persistent kernel between rounds, plus the global termination test.
+// Exchange e: every thread packs boundary values into this rank's slot e&1
+// and counts the ones that differ from the last exchange's result; warp 0 of
+// block 0 publishes (activity = signalled vertices + changed boundary values)
+// and epoch e to every peer, waits for every peer's epoch e and sums their
+// activities; every thread then reduces all ranks' slot e&1 into its masters
+// (signalling changed vertices into bitmap ncur).  Activity 0 on every rank
+// means no rank has work and no boundary value changed since the last
+// exchange -- the reduction cannot change anything: the run is converged.
+__device__ __forceinline__ bool mr_exchange(const KParams& P, cg::grid_group& grid, int ncur, unsigned long long e) {
+    const MultiRank& M = P.mr;
+    const int lane = threadIdx.x & 31;
+    const int64_t T = (int64_t)gridDim.x * blockDim.x, t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const size_t off = kP2PHeader + (size_t)(e & 1) * M.slot_bytes;
+    unsigned long long* mine = (unsigned long long*)((unsigned char*)M.own + off);
+    unsigned dirty = 0;
+    for (int64_t k = t0; k < M.nb; k += T) {
+        const int v = M.bnd[k];
+        if (M.sum) {
+            const unsigned long long g = P.vs_t[v] - M.base[k];
+            mine[k] = g;
+            dirty += g != 0;
+        } else {
+            const uint32_t x = P.vs_u[v];
+            mine[k] = x;
+            dirty += x != M.last[k];
+        }
+    }
+    for (int sh = 16; sh; sh >>= 1) dirty += __shfl_xor_sync(0xffffffffu, dirty, sh);
+    if (lane == 0 && dirty) atomicAdd(&P.ctr->mr_dirty, (unsigned long long)dirty);
+    grid.sync();
+    if (blockIdx.x == 0 && threadIdx.x < 32) {
+        const int q = lane;
+        if (q == 0) {
+            const unsigned long long act = *((volatile unsigned*)&P.ctr->active[ncur]) +
+                                           *((volatile unsigned long long*)&P.ctr->mr_dirty);
+            *((volatile unsigned long long*)&M.own[kP2PCount + (e & 1)]) = act;
+            P.ctr->mr_dirty = 0;
+            __threadfence_system();
+        }
+        __syncwarp();
+        if (q < M.world && q != M.rank) {
+            __threadfence_system();
+            unsigned long long* f = (unsigned long long*)M.region[q] + M.rank;
+            asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(f), "l"(e) : "memory");
+        }
+        bool late = false;
+        unsigned long long c = 0;
+        if (q < M.world && q != M.rank) {
+            unsigned long long ts, t, v;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(ts));
+            while (true) {
+                asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(M.own + q) : "memory");
+                if (v >= e) break;
+                asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+                if (t - ts > M.timeout_ns) { late = true; break; }
+                __nanosleep(256);
+            }
+            const unsigned long long* pc = (const unsigned long long*)M.region[q] + kP2PCount + (e & 1);
+            asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(c) : "l"(pc) : "memory");
+        } else if (q == M.rank) {
+            c = *((volatile unsigned long long*)&M.own[kP2PCount + (e & 1)]);
+        }
+        for (int sh = 16; sh; sh >>= 1) c += __shfl_xor_sync(0xffffffffu, c, sh);
+        const bool any_late = __any_sync(0xffffffffu, late);
+        if (q == 0) {
+            P.ctr->mr_total = any_late ? 0ull : c;
+            if (any_late) P.ctr->mr_err = 1;
+        }
+    }
+    grid.sync();
+    if (*((volatile unsigned long long*)&P.ctr->mr_err)) return true;
+    uint32_t* b = P.bits + (int64_t)ncur * P.nw;
+    unsigned cnt = 0;
+    for (int64_t k = t0; k < M.nb; k += T) {
+        const int v = M.bnd[k];
+        if (M.sum) {
+            unsigned long long g = 0;
+            for (int r = 0; r < M.world; r++) g += __ldcv((const unsigned long long*)(M.region[r] + off) + k);
+            const unsigned long long t = M.base[k] + g;
+            M.base[k] = t;
+            P.vs_t[v] = t;
+            if (t - P.sigma[v] >= M.eps_fx) {
+                P.sigma[v] = t;
+                cnt += signal_vertex(b, (uint32_t)v);
+            }
+        } else {
+            unsigned long long m = ~0ull;
+            for (int r = 0; r < M.world; r++) m = min(m, __ldcv((const unsigned long long*)(M.region[r] + off) + k));
+            M.last[k] = (uint32_t)m;
+            if ((uint32_t)m < P.vs_u[v]) {
+                P.vs_u[v] = (uint32_t)m;
+                cnt += signal_vertex(b, (uint32_t)v);
+            }
+        }
+    }
+    for (int sh = 16; sh; sh >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, sh);
+    if (lane == 0 && cnt) atomicAdd(&P.ctr->active[ncur], cnt);
+    grid.sync();
+    return *((volatile unsigned long long*)&P.ctr->mr_total) == 0;
+}
+
+// MR: fused multi-rank run (P.mr.world > 1) -- a separate instantiation, so a
+// single-rank run carries none of its code or registers
+template <int ALGO, int MINB = DG_PATH_MINB, bool MR = false>
 __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
     cg::grid_group grid = cg::this_grid();
     const int lane = threadIdx.x & 31;
@@ -1168,14 +1298,24 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
         px.acc = reinterpret_cast<unsigned*>(px.T + px.H);
     }
     Acc acc;
-    int r = 0;
+    constexpr bool multi = MR;
+    int r = 0, since = 0;
+    unsigned long long ex = 0;
     for (; r < P.max_rounds; r++) {
         const int round = P.ctr->round + r;  // ctr->round only changes after the loop
         const int cur = round & 1, nxt = cur ^ 1;
-        if (*((volatile unsigned*)&P.ctr->active[cur]) == 0) break;
+        // a rank of a fused multi-rank run keeps going without local work: it
+        // idles through rounds to the next exchange (mr_exchange)
+        const bool idle = *((volatile unsigned*)&P.ctr->active[cur]) == 0;
+        if (idle && !multi) break;
         const uint32_t* bcur = P.bits + (int64_t)cur * P.nw;
         uint32_t* bnxt = P.bits + (int64_t)nxt * P.nw;
-        if (kAccum) {
+        if (multi && idle) {
+            if (kAccum)  // no sweep writes the next bitmap this round
+                for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.nw;
+                     i += (int64_t)gridDim.x * blockDim.x)
+                    bnxt[i] = 0u;
+        } else if (kAccum) {
             // sparse round: few signalled vertices whose out-edges are at most M / sparse_div
             if (sparse_round(P, grid, cur, bcur)) {
                 walk_sparse_acc(P, P.occ_items, *((volatile unsigned*)&P.ctr->qcur[cur]), &P.ctr->ticket[cur], bcur, acc);
@@ -1284,6 +1424,13 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             P.ctr->qn_in[cur] = P.ctr->osum_in[cur] = P.ctr->qcur_in[cur] = P.ctr->ticket_in[cur] = 0;
         }
         grid.sync();
+        if (multi && (++since >= P.mr.every || *((volatile unsigned*)&P.ctr->active[nxt]) == 0)) {
+            since = 0;
+            if (mr_exchange(P, grid, nxt, P.mr.epoch0 + ++ex)) {
+                r++;
+                break;
+            }
+        }
     }
     unsigned long long su = acc.upd, se = acc.edges, sn = acc.entries;
     for (int off = 16; off; off >>= 1) {
@@ -1298,7 +1445,10 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
         atomicAdd(&P.ctr->entries, sn);
     }
     grid.sync();
-    if (blockIdx.x == 0 && threadIdx.x == 0) P.ctr->round += r;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        P.ctr->round += r;
+        P.ctr->mr_ex = ex;
+    }
 }
 
 // ------------------------------------------------------------------ vertex-centric ablation
@@ -1672,8 +1822,6 @@ __global__ void unpack_sum_kernel(unsigned long long* vs, unsigned long long* si
 // SUM of growth) straight from peer memory and applies it like unpack.  A
 // rank rewrites slot e&1 only at exchange e+2, after every peer published
 // e+1, i.e. after every peer's exchange-e reduce completed (stream order).
-constexpr int kP2PMaxRanks = 16;
-constexpr size_t kP2PHeader = 256;  // bytes: flags + error word
 struct PeerSlots {
     const void* p[kP2PMaxRanks];
 };
@@ -1948,13 +2096,24 @@ int ensure_occ(DevWork* W, const DevLayout& D, RunState& S, bool incoming, std::
 }
 
 // Launch the persistent path kernel for at most `rounds` rounds.
-int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState& S, std::string& err) {
+int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState& S, std::string& err,
+                const MultiRank* mr = nullptr) {
     KParams P = make_params(D, W);
+    if (mr) P.mr = *mr;
     P.eps = (float)S.eps;
     P.eps_fx = (unsigned long long)(S.eps * 4294967296.0);
     P.max_rounds = rounds;
     void* fn = nullptr;
-    switch (algo_k) {
+    if (mr) {
+        switch (algo_k) {
+            case DG_SSSP: fn = (void*)path_kernel<DG_SSSP, DG_PATH_MINB, true>; break;
+            case DG_BFS: fn = (void*)path_kernel<DG_BFS, DG_PATH_MINB, true>; break;
+            case DG_WCC: fn = (void*)path_kernel<DG_WCC, DG_PATH_MINB, true>; break;
+            case DG_PAGERANK: fn = (void*)path_kernel<DG_PAGERANK, 2, true>; break;
+            case DG_ADSORPTION: fn = (void*)path_kernel<DG_ADSORPTION, 2, true>; break;
+            default: err = "fused multi-rank run: bad algo"; return DG_EINVAL;
+        }
+    } else switch (algo_k) {
         case DG_SSSP: fn = (void*)path_kernel<DG_SSSP>; break;
         case DG_BFS: fn = (void*)path_kernel<DG_BFS>; break;
         case DG_WCC: fn = (void*)path_kernel<DG_WCC>; break;
@@ -2422,6 +2581,7 @@ struct P2P {
     unsigned long long epoch = 0;   // exchanges done (identical on every rank)
     unsigned char* own = nullptr;   // this rank's exchange region (cudaMalloc)
     unsigned char* peer[kP2PMaxRanks] = {};  // every rank's region in this address space (own included)
+    uint32_t* last = nullptr;       // fused runs, MIN: reduced boundary values of the last exchange
     bool opened = false;
 };
 
@@ -2465,6 +2625,7 @@ void dev_p2p_free(P2P*& X) {
     for (int r = 0; r < X->world; r++)
         if (X->peer[r] && r != X->rank) cudaIpcCloseMemHandle(X->peer[r]);
     if (X->own) cudaFree(X->own);
+    if (X->last) cudaFree(X->last);
     delete X;
     X = nullptr;
 }
@@ -2508,6 +2669,47 @@ int dev_boundary_exchange(DevWork* W, const DevLayout& D, RunState& S, P2P* X, i
     if (timed_out) { err = "dg_boundary_exchange: a peer did not arrive within 60 s"; return DG_ETIMEOUT; }
     if ((rc = read_counters(W, c, err))) return rc;
     *active = c.active[slot];
+    return DG_OK;
+}
+
+// A whole multi-rank run in one launch per rank: the exchanges (every
+// `local_rounds` rounds, or as soon as this rank has no work) and the global
+// termination test run inside path_kernel (mr_exchange).
+int dev_run_fused(DevWork* W, const DevLayout& D, RunState& S, P2P* X, int64_t local_rounds, int64_t max_rounds,
+                  int64_t* exchanges, int64_t* converged, std::string& err) {
+    if (!X || !X->opened) { err = "dg_run_fused: peers not opened (dg_p2p_open)"; return DG_EINVAL; }
+    if (X->nb != D.n_bnd) { err = "dg_run_fused: layout changed since dg_p2p_alloc"; return DG_EINVAL; }
+    if (S.algo != DG_SSSP && S.algo != DG_BFS && S.algo != DG_WCC && S.algo != DG_PAGERANK &&
+        S.algo != DG_ADSORPTION) {
+        err = "dg_run_fused: SSSP, BFS, WCC, PageRank or Adsorption";
+        return DG_EINVAL;
+    }
+    const size_t nbs = (size_t)std::max<int64_t>(D.n_bnd, 1);
+    if (!X->last) CK(cudaMalloc(&X->last, sizeof(uint32_t) * nbs));
+    CK(cudaMemset(X->last, 0xFF, sizeof(uint32_t) * nbs));  // differs from every state: the first exchange is dirty
+    MultiRank M{};
+    for (int r = 0; r < X->world; r++) M.region[r] = X->peer[r];
+    M.own = (unsigned long long*)X->own;
+    M.bnd = D.bnd;
+    M.base = W->bnd_base;
+    M.last = X->last;
+    M.nb = D.n_bnd;
+    M.slot_bytes = sizeof(unsigned long long) * nbs;
+    M.epoch0 = X->epoch;
+    M.timeout_ns = 60ull * 1000000000ull;
+    M.eps_fx = (unsigned long long)(S.eps * 4294967296.0);
+    M.world = X->world;
+    M.rank = X->rank;
+    M.every = (int)std::max<int64_t>(1, local_rounds);
+    M.sum = S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION;
+    int rc;
+    if ((rc = launch_path(W, D, S.algo, (int)std::min<int64_t>(max_rounds, 1 << 30), S, err, &M))) return rc;
+    Counters c;
+    if ((rc = read_counters(W, c, err))) return rc;
+    X->epoch += c.mr_ex;
+    *exchanges = (int64_t)c.mr_ex;
+    if (c.mr_err) { err = "dg_run_fused: a peer did not arrive within 60 s"; return DG_ETIMEOUT; }
+    *converged = c.mr_ex > 0 && c.mr_total == 0;
     return DG_OK;
 }
 

@@ -191,6 +191,14 @@ class DiGraph:
         check(self._L.dg_boundary_exchange(self._h, ctypes.byref(a)), "dg_boundary_exchange")
         return a.value
 
+    def run_fused(self, local_rounds=4, max_rounds=0):
+        """The whole multi-rank run in one launch (dg_run_fused); returns
+        (exchanges, converged)."""
+        ex, conv = ctypes.c_int64(), ctypes.c_int64()
+        check(self._L.dg_run_fused(self._h, int(local_rounds), int(max_rounds), ctypes.byref(ex), ctypes.byref(conv)),
+              "dg_run_fused")
+        return ex.value, bool(conv.value)
+
     def normalize_states(self, buf):
         check(self._L.dg_normalize_states(self._h, ctypes.c_void_p(buf.data_ptr()), buf.numel()),
               "dg_normalize_states")

@@ -10,7 +10,11 @@ batches"):
      few rounds while replicas stay at most a few rounds apart), or fewer if
      its local active counter reaches zero;
   2. boundary states are exchanged: MIN for SSSP/BFS/WCC, SUM of pending
-     deltas for PageRank/Adsorption.  ``exchange="p2p"`` (default): one
+     deltas for PageRank/Adsorption.  ``exchange="fused"`` (default on
+     GPUs): the whole run is ONE dg_run_fused launch per rank -- the
+     persistent kernel does the peer-memory exchange below between its
+     rounds and tests global convergence on the devices (steps 1-4 without
+     any host involvement).  ``exchange="p2p"``: one
      dg_boundary_exchange -- pack, device-side epoch flags and an elementwise
      reduction read straight from every peer's HBM (CUDA IPC over
      NVLink/NVSwitch), unpack; no host collective moves boundary states.
@@ -74,22 +78,22 @@ def p2p_setup(engine, group=None, device=None):
 def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_rounds=4,
                     max_outer=1_000_000, device=None, group=None, exchange=None):
     """Run ``algo`` to global convergence.  Returns (stats, sync_info).
-    ``exchange``: "p2p" (default on CUDA devices) or "collective"."""
+    ``exchange``: "fused" (default on CUDA devices), "p2p" or "collective"."""
     if algo not in SUM_ALGOS + MIN_ALGOS:
         raise ValueError(f"{algo}: no multi-rank protocol (SCC is single-rank)")
     device = device if device is not None else (torch.device("cuda", torch.cuda.current_device())
                                                 if torch.cuda.is_available() else torch.device("cpu"))
     if exchange is None:
-        exchange = "p2p" if device.type == "cuda" else "collective"
-    if exchange not in ("p2p", "collective"):
-        raise ValueError(f"exchange={exchange!r}: 'p2p' or 'collective'")
+        exchange = "fused" if device.type == "cuda" else "collective"
+    if exchange not in ("fused", "p2p", "collective"):
+        raise ValueError(f"exchange={exchange!r}: 'fused', 'p2p' or 'collective'")
     nb = len(engine.boundary_vertices())
     buf = boundary_buffer(nb, algo, device)
     op = dist.ReduceOp.SUM if algo in SUM_ALGOS else dist.ReduceOp.MIN
     active = torch.zeros(1, dtype=torch.int64, device=device)
     engine.run_begin(algo, source=source, epsilon=epsilon, damping=damping)
     p2p_error = None
-    if exchange == "p2p":
+    if exchange in ("fused", "p2p"):
         p2p_error = p2p_setup(engine, group)
         if p2p_error:
             import sys
@@ -97,6 +101,11 @@ def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_ro
                   file=sys.stderr, flush=True)
             exchange = "collective"
     syncs, bytes_per_sync = 0, buf.numel() * buf.element_size()
+    if exchange == "fused":
+        syncs, converged = engine.run_fused(local_rounds)
+        if not converged:
+            raise RuntimeError("multi-rank run did not converge")
+        max_outer = 0
     for _ in range(max_outer):
         engine.rounds(local_rounds)
         if exchange == "p2p":
@@ -112,9 +121,10 @@ def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_ro
         if int(active.item()) == 0:
             break
     else:
-        raise RuntimeError("multi-rank run did not converge")
+        if exchange != "fused":
+            raise RuntimeError("multi-rank run did not converge")
     stats = engine.run_end()
-    if exchange == "p2p":  # every rank reads each peer's 8-byte slot per boundary vertex
+    if exchange in ("fused", "p2p"):  # every rank reads each peer's 8-byte slot per boundary vertex
         bytes_per_sync = 8 * nb * (dist.get_world_size(group) - 1)
     info = {"syncs": syncs, "boundary": nb, "nvlink_bytes_per_sync": bytes_per_sync, "exchange": exchange}
     if p2p_error:

@@ -30,7 +30,7 @@ def _graph():
     return inputs.rmat(13, 8192, 80000, seed=31)
 
 
-def _worker(rank, world, port, algo, q, sparse=False, exchange="p2p"):
+def _worker(rank, world, port, algo, q, sparse=False, exchange="fused"):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     if sparse:  # every round with <= n/4 signalled vertices walks sparse
         os.environ.update(DG_SPARSE_DIV="1", DG_SPARSE_MIN_M="0")
@@ -49,7 +49,7 @@ def _worker(rank, world, port, algo, q, sparse=False, exchange="p2p"):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("exchange", ["p2p", "collective"])
+@pytest.mark.parametrize("exchange", ["fused", "p2p", "collective"])
 @pytest.mark.parametrize("sparse", [False, True])
 @pytest.mark.parametrize("algo", ["sssp", "wcc", "pagerank"])
 def test_two_ranks_on_one_gpu_match_oracle(algo, sparse, exchange, cuda_required):
