@@ -173,12 +173,49 @@ class NoPeerEngine(CpuPathEngine):
         raise AssertionError("must not be reached: rank 1 failed dg_p2p_alloc")
 
 
+class FusedModelEngine(CpuPathEngine):
+    """Host model of dg_run_fused's protocol (path_kernel + mr_exchange):
+    between local round batches every rank publishes its activity =
+    signalled work + boundary values that differ from the previous
+    exchange's result (MIN) or non-zero growth (SUM); the boundary is
+    reduced; the run stops when the summed activity of an exchange is 0.
+    Here a rendezvous is a gloo collective, in the kernel an epoch flag."""
+
+    def p2p_alloc(self, world, rank):
+        return b"m" * 64
+
+    def p2p_open(self, handles):
+        pass
+
+    def run_fused(self, local_rounds=4, max_rounds=0):
+        nb = len(self.bnd)
+        minalgo = self.algo in ("sssp", "wcc")
+        last = None
+        for ex in range(1, 100000):
+            act = self.rounds(local_rounds)
+            buf = torch.zeros(max(nb, 1), dtype=torch.int32 if minalgo else torch.int64)
+            if nb:
+                self.boundary_pack(buf)
+            vals = buf.numpy()[:nb].astype(np.int64)
+            dirty = int((vals != last).sum()) if (minalgo and last is not None) else (
+                nb if minalgo else int((vals != 0).sum()))
+            total = torch.tensor([act + dirty], dtype=torch.int64)
+            dist.all_reduce(total)
+            dist.all_reduce(buf, op=dist.ReduceOp.MIN if minalgo else dist.ReduceOp.SUM)
+            self.boundary_unpack(buf)
+            if minalgo:
+                last = buf.numpy()[:nb].astype(np.int64)
+            if int(total.item()) == 0:
+                return ex, True
+        return ex, False
+
+
 def _worker(rank, world, port, algo, q, exchange=None):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     from paper_conf_asplos_zhangl0hlg19_b200 import parallel
     g = inputs.rmat(10, 1024, 6000, seed=21, weights=(1, 20))
-    eng = (NoPeerEngine if exchange == "p2p" else CpuPathEngine)(g, rank, world)
+    eng = {"p2p": NoPeerEngine, "fused": FusedModelEngine}.get(exchange, CpuPathEngine)(g, rank, world)
     stats, info = parallel.run_distributed(eng, algo, source=0, epsilon=1e-7, device=torch.device("cpu"),
                                            exchange=exchange)
     out = parallel.gather_states(eng, algo, g.n, device=torch.device("cpu"))
@@ -188,7 +225,8 @@ def _worker(rank, world, port, algo, q, exchange=None):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("algo,exchange", [("sssp", None), ("wcc", None), ("pagerank", None), ("sssp", "p2p")])
+@pytest.mark.parametrize("algo,exchange", [("sssp", None), ("wcc", None), ("pagerank", None), ("sssp", "p2p"),
+                                           ("sssp", "fused"), ("wcc", "fused"), ("pagerank", "fused")])
 def test_two_rank_protocol_matches_oracle(algo, exchange):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -203,7 +241,7 @@ def test_two_rank_protocol_matches_oracle(algo, exchange):
     g = inputs.rmat(10, 1024, 6000, seed=21, weights=(1, 20))
     src, dst, w = g.edges()
     assert info["boundary"] > 0 and info["syncs"] >= 1
-    assert info["exchange"] == "collective"
+    assert info["exchange"] == ("fused" if exchange == "fused" else "collective")
     assert ("p2p_error" in info) == (exchange == "p2p")
     if algo == "sssp":
         exp, _ = OA.sssp_bellman_ford(g.n, src, dst, w, 0)
