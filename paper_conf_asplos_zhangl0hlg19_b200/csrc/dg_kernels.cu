@@ -1712,12 +1712,20 @@ __global__ void __launch_bounds__(256) occ_fill_kernel(const uint32_t* e_idx, in
     for (uint32_t h = threadIdx.x; h < hubs; h += blockDim.x)
         if (s[h]) s[h] = atomicAdd(&cursor[h], s[h]);
     __syncthreads();
-    for (int64_t i = beg + threadIdx.x; i < end; i += blockDim.x) {
-        const uint32_t c = __ldcs(e_idx + i);
-        if (c & skip) continue;
-        const uint32_t v = c & kVMask;
-        const uint32_t pos = v < hubs ? atomicAdd(&s[v], 1u) : atomicAdd(&cursor[v], 1u);
-        occ[pos] = (uint32_t)i;
+    // four entries per thread and step: their atomics are in flight together
+    constexpr int kU = 4;
+    for (int64_t i0 = beg + (int64_t)threadIdx.x * kU; i0 < end; i0 += (int64_t)blockDim.x * kU) {
+        uint32_t c[kU], pos[kU];
+#pragma unroll
+        for (int u = 0; u < kU; u++) c[u] = i0 + u < end ? __ldcs(e_idx + i0 + u) : skip;
+#pragma unroll
+        for (int u = 0; u < kU; u++) {
+            const uint32_t v = c[u] & kVMask;
+            pos[u] = (c[u] & skip) ? 0u : (v < hubs ? atomicAdd(&s[v], 1u) : atomicAdd(&cursor[v], 1u));
+        }
+#pragma unroll
+        for (int u = 0; u < kU; u++)
+            if (!(c[u] & skip)) occ[pos[u]] = (uint32_t)(i0 + u);
     }
 }
 
