@@ -259,7 +259,8 @@ int dg_run_end(dg_graph *g, dg_run_stats *stats);
  * dg_p2p_alloc: after dg_build_paths(rank, world) and dg_upload; allocates
  *   the region (the library owns it; freed by dg_destroy or the next
  *   dg_p2p_alloc) and writes its IPC handle to HOST `handle` (64 bytes).
- *   2 <= world <= 16.  The caller distributes the handles (any transport).
+ *   2 <= world <= 16; world and rank must be the layout's (dg_build_paths).
+ *   The caller distributes the handles (any transport).
  * dg_p2p_open: HOST `handles` = world x 64 bytes in rank order (this rank's
  *   own entry is ignored); maps every peer's region.  Ranks on the same GPU
  *   in different processes are allowed (tests); two ranks in one process are

@@ -385,6 +385,8 @@ int dg_boundary_unpack(dg_graph* g, const void* buf, int64_t* active) {
 int dg_p2p_alloc(dg_graph* g, int world, int rank, void* handle) {
     if (!g || !g->layout.built || !handle) return fail(DG_EINVAL, "dg_p2p_alloc: no layout built or NULL handle");
     if (!g->uploaded) return fail(DG_EINVAL, "dg_p2p_alloc: dg_upload first");
+    if (world != g->layout.params.world || rank != g->layout.params.rank)
+        return fail(DG_EINVAL, "dg_p2p_alloc: world/rank differ from the layout's (dg_build_paths)");
     if (int rc0 = select_dev(g)) return rc0;
     std::string err;
     int rc = dg::dev_p2p_alloc(g->p2p, g->dev, world, rank, handle, err);
