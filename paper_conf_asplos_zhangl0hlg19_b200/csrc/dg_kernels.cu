@@ -471,6 +471,14 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
             // path predecessor of entry 0 (previous lane's last entry, or the carry's vertex)
             uint32_t pred0 = __shfl_up_sync(0xffffffffu, vtx[3], 1);
             if (lane == 0) pred0 = carry_vtx;
+            // the lane's (up to four) atomicMins are issued back to back and
+            // are in flight together; their results are consumed afterwards
+            uint32_t old[4];
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                old[k] = 0u;
+                if (live[k] && val[k] < a[k] && val[k] <= theta) old[k] = atomicMin(&P.vs_u[vtx[k]], val[k]);
+            }
 #pragma unroll
             for (int k = 0; k < 4; k++) {
                 if (!live[k]) continue;
@@ -483,8 +491,7 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
                         acc.sig += signal_vertex(bnxt, k ? vtx[k - 1] : pred0);
                         continue;
                     }
-                    const uint32_t old = atomicMin(&P.vs_u[vtx[k]], val[k]);
-                    if (val[k] < old) {
+                    if (val[k] < old[k]) {
                         acc.upd++;
                         if (k == 3) changed3 = true;
                         acc.sig += signal_vertex(bnxt, vtx[k]);
