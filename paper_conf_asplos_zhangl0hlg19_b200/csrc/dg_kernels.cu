@@ -494,7 +494,11 @@ __device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t*
                     if (val[k] < old[k]) {
                         acc.upd++;
                         if (k == 3) changed3 = true;
-                        acc.sig += signal_vertex(bnxt, vtx[k]);
+                        // fire-and-forget signal (RED): the active counter may count a
+                        // vertex lowered twice in one round twice -- an upper bound,
+                        // which is all its uses need (non-zero test, sparse threshold)
+                        atomicOr(&bnxt[vtx[k] >> 5], 1u << (vtx[k] & 31));
+                        acc.sig++;
                         acc.vmin = min(acc.vmin, val[k]);
                     }
                 }
