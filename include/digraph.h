@@ -94,6 +94,9 @@ typedef struct {
     int64_t entries_processed;    /* path entries walked (path mode)               */
     int64_t csr_edges;            /* CSR out-edges pushed (delta algorithms, ablation) */
     double kernel_ms;             /* device time of the propagation kernels only   */
+    int64_t dense_rounds;         /* path mode: rounds that streamed every window's
+                                     entries (the others walked sparse from the
+                                     signalled vertices); for the byte model      */
 } dg_run_stats;
 
 /* Static description of the built layout (sizes; for tests and benchmarks). */
@@ -130,7 +133,9 @@ const char *dg_last_error(void);
  *   col      HOST int32[m], destination of edge k (source = the row)
  *   weight   HOST int32[m] edge weights (>= 0) or NULL (all weights 1)
  * The arrays are copied (host copy for preprocessing, device copy for the
- * vertex-centric ablation).  Invalidates a previous layout. */
+ * vertex-centric ablation).  On success it invalidates a previous graph,
+ * layout and device state; on failure (DG_EINVAL / DG_ENOMEM) the handle is
+ * left exactly as it was. */
 int dg_load_csr(dg_graph *g, int64_t n, int64_t m, const int64_t *row_ptr,
                 const int32_t *col, const int32_t *weight);
 
@@ -167,12 +172,15 @@ int dg_set_vertex_params(dg_graph *g, const double *p_inj, const double *p_cont,
  *            signalled by the previous round) + Delta.  0 = library default
  *            (SSSP: 2 * max edge weight; BFS: 1, level-synchronous),
  *            < 0 = unbounded,
- *            > 0 = that width.  Results are exact for every value; it trades
- *            redundant updates against rounds.  Ignored by the others.
+ *            > 0 = that width (values above 2^31-1 act as unbounded).
+ *            Results are exact for every value; it trades redundant
+ *            updates against rounds.  Ignored by the others.
  *   mode     DG_MODE_PATH or DG_MODE_VERTEX (ablation: SSSP, BFS, PageRank,
  *            WCC -- WCC pushes labels over both edge directions)
  *   max_rounds  safety cap (<= 0: 1,000,000)
  *   stats    may be NULL
+ * DG_ENOCONV if max_rounds ended the run (for SCC: any forward or backward
+ * phase) before convergence; the states are then not final.
  * States stay on the device until dg_get_states.  Single-rank only: with
  * world > 1 use dg_rounds / dg_boundary_* (multi-GPU protocol). */
 int dg_run(dg_graph *g, int algo, int64_t source, double epsilon, double param,
@@ -226,7 +234,9 @@ int dg_boundary_vertices(const dg_graph *g, int32_t *out);
 /* Start a multi-round run (resets states as dg_run does). */
 int dg_run_begin(dg_graph *g, int algo, int64_t source, double epsilon, double param);
 
-/* Run up to max_rounds local rounds; *active = partitions still active. */
+/* Run up to max_rounds local rounds; *active is non-zero iff work remains
+ * (an upper bound on the vertices signalled for the next round: a vertex
+ * lowered twice in a round may count twice). */
 int dg_rounds(dg_graph *g, int64_t max_rounds, int64_t *active);
 
 /* Pack boundary states into DEVICE buffer `buf` (n_boundary elements, see
@@ -235,8 +245,9 @@ int dg_rounds(dg_graph *g, int64_t max_rounds, int64_t *active);
  * always sends its new state to its master"). */
 int dg_boundary_pack(dg_graph *g, void *buf);
 
-/* Apply the all-reduced DEVICE buffer; vertices whose state changed
- * re-activate their partitions.  *active = partitions activated. */
+/* Apply the all-reduced DEVICE buffer; vertices whose state changed are
+ * signalled for the next local round.  *active is non-zero iff work remains
+ * (an upper bound on the signalled vertices, as for dg_rounds). */
 int dg_boundary_unpack(dg_graph *g, const void *buf, int64_t *active);
 
 /* Finish the run: normalisation (PageRank) and statistics. */

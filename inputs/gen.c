@@ -127,18 +127,29 @@ static int cmp_i32(const void *x, const void *y) {
  * (u,v); drop_self: drop u->u.  keep_m > 0: if more edges survive, keep the
  * keep_m ones with the smallest hash(u,v) (deterministic thinning to an exact
  * edge count).  row_ptr has n+1 entries; col must hold m entries.
- * Returns the final edge count. */
+ * Returns the final edge count.  Every pass is parallel; the output does not
+ * depend on the thread count (rows are sorted after an unordered fill, and the
+ * thinning threshold is the exact keep_m-th smallest hash). */
+static inline uint64_t thin_hash(uint64_t seed, int64_t v, int32_t x) {
+    return h3(seed ^ 0x7f4a7c15ull, (uint64_t)v, (uint64_t)x);
+}
+static int cmp_u64(const void *x, const void *y) {
+    uint64_t a = *(const uint64_t *)x, b = *(const uint64_t *)y;
+    return (a > b) - (a < b);
+}
 int64_t dgi_build_csr(int64_t n, int64_t m, const int32_t *src, const int32_t *dst,
                       int dedupe, int drop_self, int64_t keep_m, uint64_t seed,
                       int64_t *row_ptr, int32_t *col) {
     int64_t *cnt = (int64_t *)calloc((size_t)n + 1, sizeof(int64_t));
+    #pragma omp parallel for schedule(static)
     for (int64_t k = 0; k < m; k++)
-        if (!(drop_self && src[k] == dst[k])) cnt[src[k] + 1]++;
+        if (!(drop_self && src[k] == dst[k])) __atomic_fetch_add(&cnt[src[k] + 1], 1, __ATOMIC_RELAXED);
     for (int64_t v = 0; v < n; v++) cnt[v + 1] += cnt[v];
     int64_t *fill = (int64_t *)malloc(sizeof(int64_t) * (size_t)n);
     memcpy(fill, cnt, sizeof(int64_t) * (size_t)n);
+    #pragma omp parallel for schedule(static)
     for (int64_t k = 0; k < m; k++)
-        if (!(drop_self && src[k] == dst[k])) col[fill[src[k]]++] = dst[k];
+        if (!(drop_self && src[k] == dst[k])) col[__atomic_fetch_add(&fill[src[k]], 1, __ATOMIC_RELAXED)] = dst[k];
     free(fill);
     /* sort (and dedupe) each row in place */
     int64_t *keep = (int64_t *)malloc(sizeof(int64_t) * ((size_t)n + 1));
@@ -151,49 +162,67 @@ int64_t dgi_build_csr(int64_t n, int64_t m, const int32_t *src, const int32_t *d
             if (!dedupe || i == b || col[i] != col[i - 1]) col[w++] = col[i];
         keep[v] = w - b;
     }
-    /* optional thinning: global threshold on hash(u,v) via sampling + exact pass */
     int64_t total = 0;
+    #pragma omp parallel for reduction(+:total) schedule(static)
     for (int64_t v = 0; v < n; v++) total += keep[v];
+    /* optional thinning: the exact keep_m-th smallest hash(u,v) by a two-pass
+     * radix select (histogram of the top 16 bits, then the one bucket sorted) */
     uint64_t thresh = UINT64_MAX;
     if (keep_m > 0 && total > keep_m) {
-        /* exact k-th smallest hash by collecting all hashes (fine up to ~2e9) */
-        uint64_t *hs = (uint64_t *)malloc(sizeof(uint64_t) * (size_t)total);
-        int64_t *off = (int64_t *)malloc(sizeof(int64_t) * ((size_t)n + 1));
-        off[0] = 0;
-        for (int64_t v = 0; v < n; v++) off[v + 1] = off[v] + keep[v];
+        enum { NB = 1 << 16 };
+        uint64_t *hist = (uint64_t *)calloc(NB, sizeof(uint64_t));
+        #pragma omp parallel
+        {
+            uint64_t *h = (uint64_t *)calloc(NB, sizeof(uint64_t));
+            #pragma omp for schedule(dynamic, 1024)
+            for (int64_t v = 0; v < n; v++)
+                for (int64_t i = 0; i < keep[v]; i++) h[thin_hash(seed, v, col[cnt[v] + i]) >> 48]++;
+            #pragma omp critical
+            for (int b2 = 0; b2 < NB; b2++) hist[b2] += h[b2];
+            free(h);
+        }
+        int64_t kth = keep_m - 1, below = 0;
+        int bucket = 0;
+        while (below + (int64_t)hist[bucket] <= kth) below += (int64_t)hist[bucket++];
+        int64_t nb = (int64_t)hist[bucket], pos = 0;
+        uint64_t *cand = (uint64_t *)malloc(sizeof(uint64_t) * (size_t)(nb > 0 ? nb : 1));
         #pragma omp parallel for schedule(dynamic, 1024)
         for (int64_t v = 0; v < n; v++)
-            for (int64_t i = 0; i < keep[v]; i++)
-                hs[off[v] + i] = h3(seed ^ 0x7f4a7c15ull, (uint64_t)v, (uint64_t)col[cnt[v] + i]);
-        /* quickselect */
-        int64_t lo = 0, hi = total - 1, kth = keep_m - 1;
-        uint64_t st = seed;
-        while (lo < hi) {
-            st = mix64(st);
-            uint64_t pivot = hs[lo + (int64_t)(st % (uint64_t)(hi - lo + 1))];
-            int64_t i = lo, j = hi;
-            while (i <= j) {
-                while (hs[i] < pivot) i++;
-                while (hs[j] > pivot) j--;
-                if (i <= j) { uint64_t t = hs[i]; hs[i] = hs[j]; hs[j] = t; i++; j--; }
+            for (int64_t i = 0; i < keep[v]; i++) {
+                uint64_t x = thin_hash(seed, v, col[cnt[v] + i]);
+                if ((int)(x >> 48) == bucket) cand[__atomic_fetch_add(&pos, 1, __ATOMIC_RELAXED)] = x;
             }
-            if (kth <= j) hi = j; else if (kth >= i) lo = i; else break;
-        }
-        thresh = hs[kth];
-        free(hs); free(off);
+        qsort(cand, (size_t)nb, sizeof(uint64_t), cmp_u64);
+        thresh = cand[kth - below];
+        free(cand); free(hist);
     }
-    /* compact rows */
+    /* compact rows: kept count per row, offsets, parallel copy into a
+     * temporary (rows move left, so an in-place parallel copy could overwrite
+     * a row not yet read), then back into col */
+    int64_t *kc = (int64_t *)malloc(sizeof(int64_t) * ((size_t)n + 1));
+    #pragma omp parallel for schedule(dynamic, 1024)
+    for (int64_t v = 0; v < n; v++) {
+        int64_t c = keep[v];
+        if (thresh != UINT64_MAX) {
+            c = 0;
+            for (int64_t i = 0; i < keep[v]; i++) c += thin_hash(seed, v, col[cnt[v] + i]) <= thresh;
+        }
+        kc[v] = c;
+    }
     row_ptr[0] = 0;
+    for (int64_t v = 0; v < n; v++) row_ptr[v + 1] = row_ptr[v] + kc[v];
+    int32_t *tmp = (int32_t *)malloc(sizeof(int32_t) * (size_t)(row_ptr[n] > 0 ? row_ptr[n] : 1));
+    #pragma omp parallel for schedule(dynamic, 1024)
     for (int64_t v = 0; v < n; v++) {
         int64_t b = cnt[v], w = row_ptr[v];
         for (int64_t i = 0; i < keep[v]; i++) {
             int32_t x = col[b + i];
-            if (thresh != UINT64_MAX &&
-                h3(seed ^ 0x7f4a7c15ull, (uint64_t)v, (uint64_t)x) > thresh) continue;
-            col[w++] = x;
+            if (thresh != UINT64_MAX && thin_hash(seed, v, x) > thresh) continue;
+            tmp[w++] = x;
         }
-        row_ptr[v + 1] = w;
     }
+    memcpy(col, tmp, sizeof(int32_t) * (size_t)row_ptr[n]);
+    free(tmp); free(kc);
     free(cnt); free(keep);
     return row_ptr[n];
 }

@@ -40,7 +40,8 @@ class dg_run_stats(ctypes.Structure):
                 ("vertex_updates", ctypes.c_int64), ("edges_processed", ctypes.c_int64),
                 ("units_processed", ctypes.c_int64), ("kernel_launches", ctypes.c_int64),
                 ("outer_iterations", ctypes.c_int64), ("entries_processed", ctypes.c_int64),
-                ("csr_edges", ctypes.c_int64), ("kernel_ms", ctypes.c_double)]
+                ("csr_edges", ctypes.c_int64), ("kernel_ms", ctypes.c_double),
+                ("dense_rounds", ctypes.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

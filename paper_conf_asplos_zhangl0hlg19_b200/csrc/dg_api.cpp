@@ -79,14 +79,10 @@ int dg_load_csr(dg_graph* g, int64_t n, int64_t m, const int64_t* row_ptr, const
     if (n < 0 || n >= (int64_t)dg::kVMask || m < 0) return fail(DG_EINVAL, "dg_load_csr: bad n or m");
     if (!row_ptr || (m > 0 && !col)) return fail(DG_EINVAL, "dg_load_csr: NULL row_ptr/col");
     if (row_ptr[0] != 0 || row_ptr[n] != m) return fail(DG_EINVAL, "dg_load_csr: row_ptr[0] != 0 or row_ptr[n] != m");
-    dg::dev_p2p_free(g->p2p);
-    dg::dev_free_work(g->work);
-    dg::dev_free_layout(g->dev, true);
-    dg::dev_unpin_all(g->dev);
-    g->uploaded = false;
+    // validate into a local CSR and swap it in only on success: a failed load
+    // leaves the handle (previous graph, layout and device state) untouched
+    dg::HostCSR c;
     try {
-        dg::HostCSR& c = g->csr;
-        c = dg::HostCSR();
         c.n = n; c.m = m;
         c.row_ptr.assign(row_ptr, row_ptr + n + 1);
         c.col.assign(col, col + m);
@@ -108,10 +104,13 @@ int dg_load_csr(dg_graph* g, int64_t n, int64_t m, const int64_t* row_ptr, const
     } catch (const std::bad_alloc&) {
         return fail(DG_ENOMEM, "dg_load_csr: out of host memory");
     }
-    g->layout = dg::HostLayout();
+    // the old device state goes first: its host buffers are page-locked
     dg::dev_p2p_free(g->p2p);
     dg::dev_free_work(g->work);
     dg::dev_free_layout(g->dev, true);
+    dg::dev_unpin_all(g->dev);
+    g->csr = std::move(c);
+    g->layout = dg::HostLayout();
     g->loaded = true;
     g->uploaded = false;
     g->ran = false;

@@ -61,7 +61,8 @@ constexpr int kPad = 256;  // zero entries after every per-entry array
 // device counters of a run
 struct Counters {
     unsigned long long updates, edges, units, entries, pushes;
-    unsigned int active[2];  // path mode: vertices signalled into bitmap[k]; vertex mode: frontier sizes
+    unsigned int active[2];  // path mode: non-zero iff bitmap[k] has a signalled vertex (an upper bound on
+                             // their number: a vertex lowered twice counts twice); vertex mode: frontier sizes
     unsigned int ticket[2];
     unsigned int minval[2];  // SSSP/BFS: smallest distance signalled into bitmap[k] (bucket base of its round)
     unsigned int qn[2];      // SSSP/BFS sparse rounds: length of the round's compacted frontier list
@@ -75,6 +76,7 @@ struct Counters {
     unsigned long long mr_total;  // all ranks' published activity at the last exchange
     unsigned long long mr_ex;     // exchanges done by the last launch
     unsigned long long mr_err;    // a peer did not arrive (timeout)
+    unsigned long long dense_rounds;  // rounds that streamed every window's path entries (not sparse)
 };
 
 struct DevWork {
@@ -880,7 +882,15 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
                         if (a) atomicAdd(&P.vs_t[i], a);
                     }
                     __syncwarp();
-                    for (int64_t i = lane; i < px.H; i += 32) px.T[i] = *(volatile unsigned long long*)&P.vs_t[i];
+                    // snapshot refresh: eight independent L2 loads in flight per lane
+                    for (int64_t i0 = lane; i0 < px.H; i0 += 32 * 8) {
+                        unsigned long long t8[8];
+#pragma unroll
+                        for (int u = 0; u < 8; u++) t8[u] = i0 + 32 * u < px.H ? __ldcg(&P.vs_t[i0 + 32 * u]) : 0ull;
+#pragma unroll
+                        for (int u = 0; u < 8; u++)
+                            if (i0 + 32 * u < px.H) px.T[i0 + 32 * u] = t8[u];
+                    }
                 }
             }
         }
@@ -1321,6 +1331,7 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
         if (idle && !multi) break;
         const uint32_t* bcur = P.bits + (int64_t)cur * P.nw;
         uint32_t* bnxt = P.bits + (int64_t)nxt * P.nw;
+        bool dense = !(multi && idle);  // this round streams every window (for the byte model)
         if (multi && idle) {
             if (kAccum)  // no sweep writes the next bitmap this round
                 for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.nw;
@@ -1329,6 +1340,7 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
         } else if (kAccum) {
             // sparse round: few signalled vertices whose out-edges are at most M / sparse_div
             if (sparse_round(P, grid, cur, bcur)) {
+                dense = false;
                 walk_sparse_acc(P, P.occ_items, *((volatile unsigned*)&P.ctr->qcur[cur]), &P.ctr->ticket[cur], bcur, acc);
             } else {
             if (px.H) {  // round-start snapshot of the proxied masters
@@ -1358,6 +1370,7 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             // at most 1/sparse_div of the path entries, else walk the windows
             const bool sparse = (ALGO == DG_SSSP || ALGO == DG_BFS || ALGO == 100) && sparse_round(P, grid, cur, bcur);
             if (sparse) {
+                dense = false;
                 const unsigned qn = *((volatile unsigned*)&P.ctr->qcur[cur]);
                 if (ALGO == DG_SSSP) walk_sparse<0>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
                 else if (ALGO == DG_BFS) walk_sparse<1>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
@@ -1376,6 +1389,7 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
                                   *((volatile unsigned*)&P.ctr->osum_in[cur]) <= P.sparse_occ;
                 }
                 if (wsparse) {
+                    dense = false;
                     compact_bits(P, P.occ_off, bcur, P.occ_items, &P.ctr->qcur[cur]);
                     grid.sync();
                     walk_sparse<2>(P, P.occ_off, P.occ, P.occ_items, *((volatile unsigned*)&P.ctr->qn[cur]), ticket,
@@ -1392,6 +1406,7 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             else if (ALGO == 100) walk_minplus<3>(P, ticket, bcur, bnxt, INF, acc);
             else if (ALGO == 101 && sparse_round(P, grid, cur, bcur)) {
                 // sparse backward round (same decision as the forward rounds)
+                dense = false;
                 walk_sparse_bwd<false>(P, P.occ_off, P.occ, P.occ_items, *((volatile unsigned*)&P.ctr->qcur[cur]), ticket, bnxt, acc);
             } else if (ALGO == 101) {
                 while (true) {
@@ -1406,7 +1421,10 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
         // publish this round's newly signalled vertices (the device active counter)
         unsigned s = acc.sig;
         for (int off = 16; off; off >>= 1) s += __shfl_xor_sync(0xffffffffu, s, off);
-        if (lane == 0 && s) atomicAdd(&P.ctr->active[nxt], s);
+        // a warp adds at most 2^19: with at most 148 x 4 x 8 warps the 32-bit
+        // counter cannot wrap to 0 (it is an upper bound on the signalled
+        // vertices, used only for its non-zero test and the sparse threshold)
+        if (lane == 0 && s) atomicAdd(&P.ctr->active[nxt], min(s, 1u << 19));
         acc.sig = 0;
         if ((ALGO == DG_SSSP || ALGO == DG_BFS) && P.delta) {
             uint32_t mv = acc.vmin;
@@ -1425,10 +1443,11 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             // a round whose pending relaxations were all beyond the bucket keeps the
             // bucket base; otherwise the next bucket starts at the smallest new distance
             if ((ALGO == DG_SSSP || ALGO == DG_BFS) && P.ctr->minval[nxt] == INF)
-                P.ctr->minval[nxt] = P.ctr->minval[cur] == INF ? INF : P.ctr->minval[cur] + P.delta;
+                P.ctr->minval[nxt] = sat_add(P.ctr->minval[cur], P.delta);
             P.ctr->active[cur] = 0;
             P.ctr->ticket[cur] = 0;
             P.ctr->minval[cur] = INF;
+            if (dense) P.ctr->dense_rounds++;
             P.ctr->qn[cur] = 0;
             P.ctr->osum[cur] = 0;
             P.ctr->qcur[cur] = 0;
@@ -2145,14 +2164,20 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
         default: err = "bad algo"; return DG_EINVAL;
     }
     const bool accum = algo_k == DG_PAGERANK || algo_k == DG_ADSORPTION;
-    const size_t smem = accum ? kGbufBytes + (size_t)D.n_proxy * 16 : 0;
+    // ids are degree-descending, so any H' <= the built n_proxy also names
+    // the H' highest-degree vertices: DG_N_PROXY caps the proxies per launch
+    // (developer knob)
+    if (const char* np = std::getenv("DG_N_PROXY")) P.n_proxy = std::min<int64_t>(P.n_proxy, std::max(0, std::atoi(np)));
     if (!accum) P.n_proxy = 0;
+    const size_t smem = accum ? kGbufBytes + (size_t)P.n_proxy * 16 : 0;
     if (accum) P.e_coef = algo_k == DG_ADSORPTION ? W->e_coef : W->pr_coef;
     {
         const char* e = std::getenv("DG_PROXY_REFRESH");  // developer knob
         P.px_refresh = e ? std::atoi(e) : DG_PROXY_REFRESH;
         const char* dl = std::getenv("DG_DELTA");  // bucket width knob; default: reading R-DELTA
-        P.delta = dl ? (uint32_t)std::atoi(dl) : (uint32_t)S.delta;
+        // clamped to INF: sat_add and the bucket advance assume operands <= INF
+        const long long dv = dl ? std::atoll(dl) : (long long)S.delta;
+        P.delta = (uint32_t)std::min<long long>(std::max<long long>(dv, 0), (long long)INF);
         const int64_t sd = sparse_div();
         if ((algo_k == DG_SSSP || algo_k == DG_BFS || algo_k == 100 || algo_k == 101 || algo_k == DG_PAGERANK ||
              algo_k == DG_ADSORPTION || algo_k == DG_WCC) && sd > 0 && D.M >= sparse_min_entries()) {
@@ -2268,6 +2293,7 @@ int collect_stats(DevWork* W, RunState& S, std::string& err) {
     S.stats.units_processed = (int64_t)c.units;
     S.stats.entries_processed = (int64_t)c.entries;
     S.stats.csr_edges = (int64_t)c.pushes;
+    S.stats.dense_rounds = (int64_t)c.dense_rounds;
     return DG_OK;
 }
 
@@ -2302,6 +2328,10 @@ int run_scc(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, std
         if ((rc = launch_path(W, D, 100, rounds, S, err))) return rc;
         Counters c1;
         if ((rc = read_counters(W, c1, err))) return rc;
+        if (c1.active[c1.round & 1] != 0) {  // colours not final: roots would be wrong
+            err = "SCC forward colouring: max_rounds reached before convergence";
+            return DG_ENOCONV;
+        }
         // backward reachability from the roots within their colours
         CK(cudaMemsetAsync(W->bits, 0, sizeof(uint32_t) * 2 * W->nw));
         Counters c2{};
@@ -2311,11 +2341,16 @@ int run_scc(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, std
         if ((rc = launch_path(W, D, 101, rounds, S, err))) return rc;
         Counters c3;
         if ((rc = read_counters(W, c3, err))) return rc;
+        if (c3.active[c3.round & 1] != 0) {
+            err = "SCC backward reachability: max_rounds reached before convergence";
+            return DG_ENOCONV;
+        }
         total_rounds += c1.round + c3.round;
         tot.updates += c1.updates + c3.updates;
         tot.edges += c1.edges + c3.edges;
         tot.units += c1.units + c3.units;
         tot.entries += c1.entries + c3.entries;
+        tot.dense_rounds += c1.dense_rounds + c3.dense_rounds;
         CK(cudaMemset(W->remaining, 0, sizeof(int32_t)));
         scc_assign_kernel<<<g, 256>>>(W->vs_u, W->scc_label, W->scc_mark, D.n, W->remaining);
         S.stats.kernel_launches += 1;
@@ -2332,6 +2367,7 @@ int run_scc(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, std
     S.stats.edges_processed = (int64_t)tot.edges;
     S.stats.units_processed = (int64_t)tot.units;
     S.stats.entries_processed = (int64_t)tot.entries;
+    S.stats.dense_rounds = (int64_t)tot.dense_rounds;
     return DG_OK;
 }
 

@@ -62,10 +62,11 @@ class DiGraph:
         self._row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
         self._col = np.ascontiguousarray(col, dtype=np.int32)
         self._w = None if weight is None else np.ascontiguousarray(weight, dtype=np.int32)
-        self.n, self.m = int(n), int(self._row_ptr[-1])
-        check(self._L.dg_load_csr(self._h, self.n, self.m, _p(self._row_ptr), _p(self._col), _p(self._w)),
-              "dg_load_csr")
+        n_new, m_new = int(n), int(self._row_ptr[-1])
+        rc = self._L.dg_load_csr(self._h, n_new, m_new, _p(self._row_ptr), _p(self._col), _p(self._w))
         self._row_ptr = self._col = self._w = None  # dg_load_csr copied them
+        check(rc, "dg_load_csr")  # on failure the handle keeps the previous graph
+        self.n, self.m = n_new, m_new
         self.p2p_key = None  # the library freed any exchange region
         return self
 

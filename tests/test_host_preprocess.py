@@ -160,6 +160,28 @@ def test_bad_arguments_are_rejected():
         dg.load_csr(3, np.array([0, 1, 2, 3]), np.array([1, 2, 7]))
 
 
+def test_failed_load_keeps_the_previous_graph():
+    """A dg_load_csr that fails validation leaves the handle as it was
+    (include/digraph.h): the previous graph and its layout stay usable, so a
+    later upload cannot read host arrays sized for the rejected graph."""
+    dg = DiGraph()
+    g = fig4_graph()
+    dg.load_graph(g).build_paths()
+    before = dg.layout_info()
+    big = 100
+    for rp, col, w in [
+        (np.r_[0, np.full(big, 1)], np.array([big + 5]), None),        # column out of range
+        (np.r_[0, np.full(big, 1)], np.array([3]), np.array([-1])),     # negative weight
+        (np.r_[0, 2, 1, np.full(big - 2, 2)], np.array([1, 2]), None),  # decreasing row_ptr
+    ]:
+        with pytest.raises(DGError, match="DG_EINVAL"):
+            dg.load_csr(big, rp, col, w)
+        assert dg.n == g.n and dg.m == g.m
+        assert dg.layout_info() == before
+    ex = dg.export_paths()
+    assert len(ex["vertices"]) == before["n_entries"]
+
+
 def test_p2p_exchange_lifecycle_is_checked():
     """dg_p2p_alloc needs an uploaded layout, dg_p2p_open an allocated region,
     dg_boundary_exchange a run in progress (include/digraph.h)."""

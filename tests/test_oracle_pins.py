@@ -287,6 +287,31 @@ def test_algorithm1_is_an_edge_disjoint_cover(seed, n_sub, order):
     assert len(merged) <= len(paths)
 
 
+def test_subgraph_bounds_hand_example():
+    """Reading R-SUB by hand: lo_k = first v with row_ptr[v] >= floor(k*m/T).
+    out-degrees [4, 0, 1, 1, 2, 0], m = 8, T = 4: targets 2, 4, 6 -> v = 1,
+    1, 4 (row_ptr = [0, 4, 4, 5, 6, 8, 8])."""
+    row_ptr = np.array([0, 4, 4, 5, 6, 8, 8])
+    assert P.subgraph_bounds(6, row_ptr, 4) == [0, 1, 1, 4, 6]
+    assert P.subgraph_bounds(6, row_ptr, 1) == [0, 6]
+    assert P.subgraph_bounds(3, np.array([0, 0, 0, 0]), 3) == [0, 0, 0, 3]  # no edges
+
+
+def test_algorithm1_subgraphs_split_paths_by_hand():
+    """Each thread divides only its local subgraph: an edge
+    belongs to the subgraph of its source, and a traversal stops at a vertex
+    of another subgraph (no local edges -> line 19).  Chain 0->1->2->3->4,
+    order "id", derived by hand: T=1 one path; T=2 (bounds [0,2,5]) splits at
+    vertex 2; T=3 (bounds [0,1,2,5]) splits at 1 and 2."""
+    n = 5
+    src = np.arange(4); dst = np.arange(1, 5)
+    row_ptr, col, _, _ = to_csr(n, src, dst)
+    run = lambda t: P.graphp_decompose(n, row_ptr, col, d_max=16, n_sub=t, order="id")[0]
+    assert run(1) == [[0, 1, 2, 3, 4]]
+    assert run(2) == [[0, 1, 2], [2, 3, 4]]
+    assert run(3) == [[0, 1], [1, 2], [2, 3, 4]]
+
+
 def test_algorithm1_depth_bound_on_chain():
     n = 41  # chain 0 -> 1 -> ... -> 40
     src = np.arange(40); dst = np.arange(1, 41)
