@@ -60,7 +60,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L);
 
 // ---------------- device side ----------------
 struct DevLayout {
-    int64_t n = 0, m = 0, M = 0, n_part = 0, n_bnd = 0;
+    int64_t n = 0, m = 0, M = 0, n_part = 0, n_bnd = 0, max_part = 0;
     uint32_t* e_idx = nullptr;
     int32_t* e_w = nullptr;
     int64_t* part_off = nullptr;

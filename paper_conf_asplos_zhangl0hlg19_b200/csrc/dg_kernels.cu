@@ -100,6 +100,7 @@ struct DevWork {
     uint8_t* scc_mark = nullptr;
     int32_t* remaining = nullptr;
     uint32_t* out_stage = nullptr;         // dg_get_states staging buffer (n words)
+    unsigned* qtick = nullptr;             // per-CTA partition queue counters (2 x kMaxGrid x kQStride)
     uint32_t* occ_off = nullptr;           // vertex -> its non-tail path entries (sparse rounds), n+1
     uint32_t* occ = nullptr;               // entry indices grouped by vertex
     uint2* occ_items = nullptr;            // frontier items (v, chunk of <= kOccChunk occurrences)
@@ -172,6 +173,9 @@ struct KParams {
     uint32_t sparse_occ;      // ... and are walked sparse if their out-edges are at most this many
     int sparse_walk;          // path edges a sparse walk follows at most
     MultiRank mr;             // world > 1: fused multi-rank run
+    unsigned* qtick;            // per-CTA partition queue counters, 2 x grid x kQStride (null: global ticket)
+    unsigned long long* trace;  // DG_TRACE: per round {end time ns, vertices signalled into it, dense, out-edges}
+    int trace_cap;
 };
 
 // ------------------------------------------------------------------ helpers
@@ -287,28 +291,97 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 __device__ __forceinline__ void cp_async_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
 __device__ __forceinline__ void cp_async_wait0() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 
-// A warp's stream of 128-entry windows over the partitions it takes from the
-// round's ticket (priority order): base < 0 marks the end of the stream.
-// Entry offsets are 32-bit (dev_upload_layout checks M + padding < 2^32) so
-// the three cursors of the software pipeline stay in 9 registers.
+// Partition dispatch of a dense round ("work stealing
+// for balanced load between SMXs", line 192 priority order; north_star (3)
+// "per-SM hot-first priority work queue").  The partitions are in priority
+// order; CTA c owns the queue {c, c+G, c+2G, ...} (G = grid size), so every
+// queue is itself hot-first and all CTAs advance through the priority order
+// together.  A CTA's warps take partitions from its own queue (one atomic on
+// the CTA's own counter, on its own 32-byte line); once it is empty they steal
+// single partitions from the other CTAs' queues, starting at the next CTA, and
+// a per-CTA shared cursor skips victims found empty.  DG_DISPATCH=0 (developer
+// knob) restores one global ticket.
+struct Queue {
+    unsigned* qt;        // per-CTA counters of this round (stride kQStride)
+    unsigned* global;    // the single global ticket (DG_DISPATCH=0)
+    unsigned* s_state;   // shared: [0] next victim offset, [1] own queue empty
+};
+constexpr int kQStride = 8;
+constexpr int kMaxGrid = 4096;  // CTAs of a persistent launch (148 SMs x resident CTAs)
+constexpr unsigned kNoPart = 0xFFFFFFFFu;
+__device__ __forceinline__ unsigned queue_len(unsigned n_part, unsigned c, unsigned G) {
+    return n_part > c ? (n_part - c - 1) / G + 1 : 0u;
+}
+// The rank (in priority order) of the warp's next partition, or kNoPart; all
+// lanes call it.  Own queue: one atomic by lane 0.  Stealing: the warp probes
+// 32 victims' counters at once with plain loads, then takes from the first
+// with partitions left (atomic); a batch found empty advances the CTA's shared
+// cursor, so each CTA scans the other queues about once per round.
+__device__ __forceinline__ unsigned take_rank(const KParams& P, const Queue& q) {
+    const unsigned np = (unsigned)P.n_part;
+    const int lane = threadIdx.x & 31;
+    unsigned t = kNoPart;
+    if (!q.qt) {
+        if (lane == 0) {
+            const unsigned k = atomicAdd(q.global, 1u);
+            t = k < np ? k : kNoPart;
+        }
+        return __shfl_sync(0xffffffffu, t, 0);
+    }
+    const unsigned G = gridDim.x, c = blockIdx.x;
+    if (lane == 0 && !*(volatile unsigned*)&q.s_state[1]) {
+        const unsigned k = atomicAdd(&q.qt[c * kQStride], 1u);
+        if (k < queue_len(np, c, G)) t = c + k * G;
+        else q.s_state[1] = 1u;
+    }
+    t = __shfl_sync(0xffffffffu, t, 0);
+    if (t != kNoPart) return t;
+    while (true) {
+        const unsigned j0 = *(volatile unsigned*)&q.s_state[0];
+        if (j0 >= G) return kNoPart;
+        const unsigned j = j0 + lane;
+        const unsigned v = c + j < G ? c + j : c + j - G;
+        const bool left = j < G && __ldcg(&q.qt[v * kQStride]) < queue_len(np, v, G);
+        unsigned mask = __ballot_sync(0xffffffffu, left);
+        while (mask) {
+            const int l = __ffs(mask) - 1;
+            mask &= mask - 1;
+            const unsigned vv = __shfl_sync(0xffffffffu, v, l);
+            unsigned k = 0;
+            if (lane == 0) k = atomicAdd(&q.qt[vv * kQStride], 1u);
+            k = __shfl_sync(0xffffffffu, k, 0);
+            if (k < queue_len(np, vv, G)) return vv + k * G;
+        }
+        if (lane == 0) atomicMax(&q.s_state[0], j0 + 32);
+        __syncwarp();
+    }
+}
+__device__ __forceinline__ unsigned next_partition(const KParams& P, const Queue& q) {
+    unsigned t = take_rank(P, q);
+    if (t == kNoPart) return kNoPart;
+    if (P.part_order == 1) t = (unsigned)P.n_part - 1 - t;  // developer knob: dispatch-order experiments
+    else if (P.part_order > 1) t = (unsigned)(((unsigned long long)t * P.part_order) % (unsigned long long)P.n_part);
+    return t;
+}
+
+// A warp's stream of 128-entry windows over the partitions it takes from its
+// queue: base == kNoWin marks the end of the stream.  Entry offsets are 32-bit
+// (dev_upload_layout checks M + padding < 2^32) so the three cursors of the
+// software pipeline stay in 9 registers.
 constexpr uint32_t kNoWin = 0xFFFFFFFFu;
 struct Win {
     uint32_t base, beg, end;
 };
-__device__ __forceinline__ Win win_first_of(const KParams& P, unsigned* ticket) {
-    unsigned t = 0;
-    if ((threadIdx.x & 31) == 0) t = atomicAdd(ticket, 1u);
-    t = __shfl_sync(0xffffffffu, t, 0);
-    if (t >= (unsigned)P.n_part) return Win{kNoWin, 0, 0};
-    if (P.part_order == 1) t = (unsigned)P.n_part - 1 - t;  // developer knob: dispatch-order experiments
-    else if (P.part_order > 1) t = (unsigned)(((unsigned long long)t * P.part_order) % (unsigned long long)P.n_part);
+__device__ __forceinline__ Win win_first_of(const KParams& P, const Queue& q) {
+    const unsigned t = next_partition(P, q);
+    if (t == kNoPart) return Win{kNoWin, 0, 0};
     const uint32_t beg = (uint32_t)P.part_off[t], end = (uint32_t)P.part_off[t + 1];
     return Win{beg & ~3u, beg, end};
 }
-__device__ __forceinline__ Win win_next(const KParams& P, const Win& w, unsigned* ticket) {
+__device__ __forceinline__ Win win_next(const KParams& P, const Win& w, const Queue& q) {
     if (w.base == kNoWin) return w;
     if (w.base + 128 < w.end) return Win{w.base + 128, w.beg, w.end};
-    return win_first_of(P, ticket);
+    return win_first_of(P, q);
 }
 
 // Min-plus walk.  MODE 0 SSSP (weights), 1 BFS (unit weights), 2 WCC (weight 0,
@@ -320,7 +393,7 @@ __device__ __forceinline__ Win win_next(const KParams& P, const Win& w, unsigned
 // asynchronous semantics of any concurrent update; atomicMin stays the
 // authority), as are the indices of window w+2.
 template <int MODE>
-__device__ void walk_minplus(const KParams& P, unsigned* ticket, const uint32_t* bcur, uint32_t* bnxt,
+__device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32_t* bcur, uint32_t* bnxt,
                              uint32_t theta, Acc& acc) {
     const int lane = threadIdx.x & 31;
     const uint4 kFill = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
@@ -785,29 +858,41 @@ __device__ __forceinline__ float fx_to(unsigned long long v) { return __ull2floa
 // pushed new states of its local mirrors ... sent to the master when the
 // partition assigned to this SMX has been handled".  Per CTA: the round-start
 // totals and the CTA's unflushed pushes.
-// The pushes accumulate in two 32-bit words per hub (lo, hi) because shared
-// memory has native 32-bit atomic adds only (a 64-bit add is a CAS loop): lo
-// takes the push, its carry goes to hi.  A concurrent reader can see a carry
-// not yet applied (an under-estimate: pend only shrinks, safe) and a flush can
-// leave a pending carry for the next flush (the total is conserved).
+// Reads of a hub use the CTA's snapshot T only (refreshed every px_refresh
+// partitions): the CTA's own unflushed pushes are a 1/G share of what the hub
+// receives and, like every other push, are seen after the next refresh.
+// Pushes accumulate write-only in three 32-bit limbs per hub with
+// fire-and-forget shared REDs (shared memory has native 32-bit atomic adds
+// only; a 64-bit add is a CAS loop): limb 0 takes bits 0-15 of the push,
+// limb 1 bits 16-31, limb 2 bits 32-47.  A push >= 2^48 (2^16 in rank units)
+// goes straight to the master.  No limb can wrap: fewer than 2^16 pushes reach
+// a hub between two flushes of it (launch_path bounds px_refresh by the
+// largest partition), and every limb addend is < 2^16.
+constexpr int kPxLimbs = 3;
 struct Proxies {
-    unsigned long long* T;
-    unsigned* acc;  // 2 words per hub
+    unsigned long long* T;  // snapshot of the hub totals
+    unsigned* acc;          // kPxLimbs words per hub
     int64_t H;
 };
-__device__ __forceinline__ void px_add(unsigned* a, unsigned long long p) {
-    const unsigned lo = (unsigned)p, hi = (unsigned)(p >> 32);
-    const unsigned old = atomicAdd(&a[0], lo);
-    const unsigned c = hi + (old + lo < old ? 1u : 0u);
-    if (c) atomicAdd(&a[1], c);
+__device__ __forceinline__ void red_shared_u32(unsigned* a, unsigned v) {
+    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"((unsigned)__cvta_generic_to_shared(a)), "r"(v) : "memory");
 }
-__device__ __forceinline__ unsigned long long px_read(const unsigned* a) {
-    const unsigned lo = *(const volatile unsigned*)&a[0], hi = *(const volatile unsigned*)&a[1];
-    return ((unsigned long long)hi << 32) + lo;
+__device__ __forceinline__ void px_push(unsigned* a, unsigned long long p, unsigned long long* master) {
+    if (p >> 48) {
+        atomicAdd(master, p);
+        return;
+    }
+    const unsigned l0 = (unsigned)p & 0xFFFFu, l1 = (unsigned)(p >> 16) & 0xFFFFu, l2 = (unsigned)(p >> 32);
+    if (l0) red_shared_u32(&a[0], l0);
+    if (l1) red_shared_u32(&a[1], l1);
+    if (l2) red_shared_u32(&a[2], l2);
+}
+__device__ __forceinline__ unsigned long long px_combine(unsigned l0, unsigned l1, unsigned l2) {
+    return (unsigned long long)l0 + ((unsigned long long)l1 << 16) + ((unsigned long long)l2 << 32);
 }
 __device__ __forceinline__ unsigned long long px_take(unsigned* a) {
-    const unsigned lo = atomicExch(&a[0], 0u), hi = atomicExch(&a[1], 0u);
-    return ((unsigned long long)hi << 32) + lo;
+    const unsigned l0 = atomicExch(&a[0], 0u), l1 = atomicExch(&a[1], 0u), l2 = atomicExch(&a[2], 0u);
+    return px_combine(l0, l1, l2);
 }
 
 // Walk all windows the warp obtains in this round.  Software pipeline over the
@@ -817,7 +902,7 @@ __device__ __forceinline__ unsigned long long px_take(unsigned* a) {
 // Reading a master one window early is a read slightly before the walk
 // reaches it -- the same asynchronous semantics as any concurrent push.
 template <bool ADS>
-__device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigned long long pol_stream,
+__device__ void walk_accum(const KParams& P, const Queue& ticket, Acc& acc, unsigned long long pol_stream,
                            unsigned long long pol_keep, const Proxies& px, uint4* gbuf, int* s_done) {
     const int lane = threadIdx.x & 31;
     const unsigned long long eps = P.eps_fx;
@@ -878,7 +963,7 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
                 c = __shfl_sync(0xffffffffu, c, 0);
                 if (c % P.px_refresh == 0) {
                     for (int64_t i = lane; i < px.H; i += 32) {
-                        const unsigned long long a = px_take(&px.acc[2 * i]);
+                        const unsigned long long a = px_take(&px.acc[kPxLimbs * i]);
                         if (a) atomicAdd(&P.vs_t[i], a);
                     }
                     __syncwarp();
@@ -910,7 +995,7 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
             T[k] = 0ull;
             if (valid[k]) {
                 if (vtx[k] < px.H) {
-                    T[k] = px.T[vtx[k]] + px_read(&px.acc[2 * vtx[k]]);
+                    T[k] = px.T[vtx[k]];
                 } else {
                     const uint4 q = gbuf[slot * 128 + k * 32 + lane];
                     T[k] = (vtx[k] & 1u) ? ((unsigned long long)q.w << 32 | q.z) : ((unsigned long long)q.y << 32 | q.x);
@@ -962,7 +1047,7 @@ __device__ void walk_accum(const KParams& P, unsigned* ticket, Acc& acc, unsigne
                 if (!hd[k]) acc.edges++;
                 const unsigned long long p = fx_from(pin[k]);
                 if (p) {
-                    if (vtx[k] < px.H) px_add(&px.acc[2 * vtx[k]], p);  // proxy: shared-memory atomics
+                    if (vtx[k] < px.H) px_push(&px.acc[kPxLimbs * vtx[k]], p, &P.vs_t[vtx[k]]);  // proxy: shared REDs
                     else red_add_u64_h(&P.vs_t[vtx[k]], p, pol_keep);   // master: REDG (no return)
                     acc.upd++;
                 }
@@ -1322,9 +1407,14 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
     constexpr bool multi = MR;
     int r = 0, since = 0;
     unsigned long long ex = 0;
+    __shared__ unsigned s_queue[2];
     for (; r < P.max_rounds; r++) {
         const int round = P.ctr->round + r;  // ctr->round only changes after the loop
         const int cur = round & 1, nxt = cur ^ 1;
+        // this round's partition queues (per CTA, with stealing; or the global ticket)
+        if (threadIdx.x == 0) { s_queue[0] = 1u; s_queue[1] = 0u; }
+        __syncthreads();
+        const Queue dq{P.qtick ? P.qtick + (size_t)cur * kQStride * gridDim.x : nullptr, &P.ctr->ticket[cur], s_queue};
         // a rank of a fused multi-rank run keeps going without local work: it
         // idles through rounds to the next exchange (mr_exchange)
         const bool idle = *((volatile unsigned*)&P.ctr->active[cur]) == 0;
@@ -1346,16 +1436,19 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             if (px.H) {  // round-start snapshot of the proxied masters
                 for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) {
                     px.T[i] = __ldcg(&P.vs_t[i]);
-                    px.acc[2 * i] = px.acc[2 * i + 1] = 0u;
+#pragma unroll
+                    for (int l = 0; l < kPxLimbs; l++) px.acc[kPxLimbs * i + l] = 0u;
                 }
                 if (threadIdx.x == 0) s_done = 0;
                 __syncthreads();
             }
-            walk_accum<ALGO == DG_ADSORPTION>(P, &P.ctr->ticket[cur], acc, pol_stream, pol_keep, px, gbuf, &s_done);
+            walk_accum<ALGO == DG_ADSORPTION>(P, dq, acc, pol_stream, pol_keep, px, gbuf, &s_done);
             if (px.H) {  // send the proxies' accumulated pushes to their masters
                 __syncthreads();
-                for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x)
-                    if (const unsigned long long a = px_read(&px.acc[2 * i])) atomicAdd(&P.vs_t[i], a);
+                for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) {
+                    const unsigned* l = &px.acc[kPxLimbs * i];
+                    if (const unsigned long long a = px_combine(l[0], l[1], l[2])) atomicAdd(&P.vs_t[i], a);
+                }
             }
             }
             grid.sync();  // all pushes of the round landed
@@ -1375,8 +1468,8 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
                 if (ALGO == DG_SSSP) walk_sparse<0>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
                 else if (ALGO == DG_BFS) walk_sparse<1>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
                 else walk_sparse<3>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
-            } else if (ALGO == DG_SSSP) walk_minplus<0>(P, ticket, bcur, bnxt, theta, acc);
-            else if (ALGO == DG_BFS) walk_minplus<1>(P, ticket, bcur, bnxt, theta, acc);
+            } else if (ALGO == DG_SSSP) walk_minplus<0>(P, dq, bcur, bnxt, theta, acc);
+            else if (ALGO == DG_BFS) walk_minplus<1>(P, dq, bcur, bnxt, theta, acc);
             else if (ALGO == DG_WCC) {
                 // sparse WCC round: labels go forward along the out-edges, then
                 // backward along the in-edges of the signalled vertices
@@ -1400,20 +1493,18 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
                     walk_sparse_bwd<true>(P, P.iocc_off, P.iocc, P.occ_items, *((volatile unsigned*)&P.ctr->qn_in[cur]),
                                           &P.ctr->ticket_in[cur], bnxt, acc);
                 } else {
-                    walk_minplus<2>(P, ticket, bcur, bnxt, INF, acc);
+                    walk_minplus<2>(P, dq, bcur, bnxt, INF, acc);
                 }
             }
-            else if (ALGO == 100) walk_minplus<3>(P, ticket, bcur, bnxt, INF, acc);
+            else if (ALGO == 100) walk_minplus<3>(P, dq, bcur, bnxt, INF, acc);
             else if (ALGO == 101 && sparse_round(P, grid, cur, bcur)) {
                 // sparse backward round (same decision as the forward rounds)
                 dense = false;
                 walk_sparse_bwd<false>(P, P.occ_off, P.occ, P.occ_items, *((volatile unsigned*)&P.ctr->qcur[cur]), ticket, bnxt, acc);
             } else if (ALGO == 101) {
                 while (true) {
-                    unsigned t = 0;
-                    if (lane == 0) t = atomicAdd(ticket, 1u);
-                    t = __shfl_sync(0xffffffffu, t, 0);
-                    if (t >= (unsigned)P.n_part) break;
+                    const unsigned t = next_partition(P, dq);
+                    if (t == kNoPart) break;
                     walk_scc_bwd(P, P.part_off[t], P.part_off[t + 1], bcur, bnxt, acc);
                 }
             }
@@ -1433,6 +1524,7 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             acc.vmin = INF;
         }
         grid.sync();
+        if (P.qtick && threadIdx.x == 0) P.qtick[((size_t)cur * gridDim.x + blockIdx.x) * kQStride] = 0u;
         if (!kAccum) {  // retire this round's bitmap for reuse two rounds later
             uint32_t* bc = P.bits + (int64_t)cur * P.nw;
             for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.nw;
@@ -1440,6 +1532,14 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
                 bc[i] = 0u;
         }
         if (blockIdx.x == 0 && threadIdx.x == 0) {
+            if (P.trace && r < P.trace_cap) {  // developer trace (DG_TRACE)
+                unsigned long long t;
+                asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+                P.trace[4 * r] = t;
+                P.trace[4 * r + 1] = P.ctr->active[cur];
+                P.trace[4 * r + 2] = dense;
+                P.trace[4 * r + 3] = P.ctr->osum[cur];
+            }
             // a round whose pending relaxations were all beyond the bucket keeps the
             // bucket base; otherwise the next bucket starts at the smallest new distance
             if ((ALGO == DG_SSSP || ALGO == DG_BFS) && P.ctr->minval[nxt] == INF)
@@ -1987,6 +2087,8 @@ KParams make_params(const DevLayout& D, DevWork* W) {
     P.ctr = W->ctr;
     P.mark = W->scc_mark; P.scc_label = W->scc_label;
     P.orig = D.orig; P.n_proxy = D.n_proxy;
+    const char* dd = std::getenv("DG_DISPATCH");  // developer knob: 0 = one global ticket
+    P.qtick = (dd && std::atoi(dd) == 0) ? nullptr : W->qtick;
     return P;
 }
 
@@ -2008,6 +2110,7 @@ int ensure_work(DevWork*& W, const DevLayout& D, std::string& err) {
     if ((rc = dalloc(&W->vlist[1], D.n + 1, bytes, err))) return rc;
     if ((rc = dalloc(&W->ctr, 1, bytes, err))) return rc;
     if ((rc = dalloc(&W->dsum, 1, bytes, err))) return rc;
+    if ((rc = dalloc(&W->qtick, 2 * kMaxGrid * kQStride, bytes, err))) return rc;
     CK(cudaMemset(W->s_val, 0, sizeof(unsigned long long) * (D.M + kPad)));
     CK(cudaEventCreate(&W->ev0));
     CK(cudaEventCreate(&W->ev1));
@@ -2031,7 +2134,8 @@ int coop_launch(DevWork* W, void* fn, KParams& P, RunState& S, std::string& err,
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
     if (smem) CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, kBlock, smem));
-    const int grid = sms * std::max(1, per);
+    const int grid = std::min(sms * std::max(1, per), kMaxGrid);
+    if (P.qtick) CK(cudaMemsetAsync(P.qtick, 0, sizeof(unsigned) * 2 * kMaxGrid * kQStride));
     void* args[] = {&P};
     CK(cudaEventRecord(W->kev0));
     CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kBlock), args, smem, 0));
@@ -2169,11 +2273,31 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
     // (developer knob)
     if (const char* np = std::getenv("DG_N_PROXY")) P.n_proxy = std::min<int64_t>(P.n_proxy, std::max(0, std::atoi(np)));
     if (!accum) P.n_proxy = 0;
-    const size_t smem = accum ? kGbufBytes + (size_t)P.n_proxy * 16 : 0;
-    if (accum) P.e_coef = algo_k == DG_ADSORPTION ? W->e_coef : W->pr_coef;
+    // proxies need a flush at least every 2^16 pushes per hub and CTA (px_push):
+    // bound the refresh interval by the largest partition, else no proxies
     {
         const char* e = std::getenv("DG_PROXY_REFRESH");  // developer knob
-        P.px_refresh = e ? std::atoi(e) : DG_PROXY_REFRESH;
+        const int want = e ? std::atoi(e) : DG_PROXY_REFRESH;
+        const int64_t allowed = 65535 / std::max<int64_t>(1, D.max_part) - 2 * kWarps;
+        if (allowed < 1) P.n_proxy = 0;
+        P.px_refresh = (want <= 0 || want > allowed) ? (int)std::max<int64_t>(1, allowed) : want;
+    }
+    if (accum && P.n_proxy) {
+        // as many proxies as fit acc_minb() CTAs per SM (the top ids are the
+        // highest-degree vertices, so a smaller H' is still the hubs)
+        int dev = 0, sm_bytes = 0, reserved = 0;
+        cudaFuncAttributes fa{};
+        CK(cudaGetDevice(&dev));
+        CK(cudaDeviceGetAttribute(&sm_bytes, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
+        CK(cudaDeviceGetAttribute(&reserved, cudaDevAttrReservedSharedMemoryPerBlock, dev));
+        CK(cudaFuncGetAttributes(&fa, fn));
+        const int64_t per_cta = sm_bytes / std::max(1, acc_minb()) - reserved - (int64_t)fa.sharedSizeBytes -
+                                (int64_t)kGbufBytes;
+        P.n_proxy = std::max<int64_t>(0, std::min<int64_t>(P.n_proxy, per_cta / (8 + 4 * kPxLimbs)));
+    }
+    const size_t smem = accum ? kGbufBytes + (size_t)P.n_proxy * (8 + 4 * kPxLimbs) : 0;
+    if (accum) P.e_coef = algo_k == DG_ADSORPTION ? W->e_coef : W->pr_coef;
+    {
         const char* dl = std::getenv("DG_DELTA");  // bucket width knob; default: reading R-DELTA
         // clamped to INF: sat_add and the bucket advance assume operands <= INF
         const long long dv = dl ? std::atoll(dl) : (long long)S.delta;
@@ -2206,7 +2330,27 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
             while (gcd(P.part_order, D.n_part) != 1) P.part_order++;
         }
     }
-    return coop_launch(W, fn, P, S, err, smem);
+    // developer trace (DG_TRACE): per-round timing and activity on stderr
+    unsigned long long* trace = nullptr;
+    constexpr int kTraceCap = 1 << 16;
+    if (std::getenv("DG_TRACE") && cudaMalloc(&trace, sizeof(unsigned long long) * 4 * kTraceCap) == cudaSuccess) {
+        cudaMemset(trace, 0, sizeof(unsigned long long) * 4 * kTraceCap);
+        P.trace = trace;
+        P.trace_cap = kTraceCap;
+    }
+    int rc = coop_launch(W, fn, P, S, err, smem);
+    if (trace) {
+        std::vector<unsigned long long> h(4 * (size_t)kTraceCap);
+        cudaMemcpy(h.data(), trace, sizeof(unsigned long long) * h.size(), cudaMemcpyDeviceToHost);
+        cudaFree(trace);
+        for (int r = 0; r < kTraceCap && h[4 * r]; r++) {
+            const unsigned long long prev = r ? h[4 * (r - 1)] : 0ull;  // round 0: no reference
+            fprintf(stderr, "[trace] algo %d round %d: %.1f us, signalled-in %llu, %s, out-edges %llu\n", algo_k, r,
+                    prev ? (h[4 * r] - prev) / 1e3 : 0.0, h[4 * r + 1], h[4 * r + 2] ? "dense" : "sparse",
+                    h[4 * r + 3]);
+        }
+    }
+    return rc;
 }
 
 int launch_vertex(DevWork* W, const DevLayout& D, int algo, int rounds, RunState& S, std::string& err) {
@@ -2456,6 +2600,8 @@ int dev_upload_layout(DevLayout& D, const HostLayout& L, std::string& err) {
         return DG_EINVAL;
     }
     D.n_part = (int64_t)L.part_off.size() - 1;
+    D.max_part = 0;
+    for (int64_t q = 0; q < D.n_part; q++) D.max_part = std::max(D.max_part, L.part_off[q + 1] - L.part_off[q]);
     D.n_bnd = (int64_t)L.boundary.size();
     if ((rc = dalloc_once(&D.e_idx, D.M + kPad, D.bytes, err))) return rc;
     if ((rc = dalloc_once(&D.part_off, D.n_part + 1, D.bytes, err))) return rc;
@@ -2492,7 +2638,7 @@ void dev_free_work(DevWork*& W) {
     if (!W) return;
     dfree(W->vs_u); dfree(W->vstamp); dfree(W->vs_f); dfree(W->vs_t); dfree(W->sigma); dfree(W->s_val); dfree(W->bnd_base);
     dfree(W->e_coef); dfree(W->pr_coef); dfree(W->ads_base); dfree(W->bits); dfree(W->vlist[0]); dfree(W->vlist[1]);
-    dfree(W->ctr); dfree(W->dsum); dfree(W->scc_label); dfree(W->scc_mark); dfree(W->remaining); dfree(W->out_stage);
+    dfree(W->ctr); dfree(W->dsum); dfree(W->qtick); dfree(W->scc_label); dfree(W->scc_mark); dfree(W->remaining); dfree(W->out_stage);
     dfree(W->occ_off); dfree(W->occ); dfree(W->occ_items); dfree(W->iocc_off); dfree(W->iocc); dfree(W->occ_cur);
     if (W->cub_tmp) cudaFree(W->cub_tmp);
     if (W->ev0) cudaEventDestroy(W->ev0);

@@ -208,8 +208,10 @@ def test_accumulative_in_sparse_and_dense_rounds(graph, sparse_div, gname):
     got = dg.get_states().astype(np.float64)
     exp, _ = OA.adsorption_jacobi(g.n, src, dst, w, p_inj, p_cont, inj, tol=1e-12)
     assert np.abs(got - exp).sum() / np.abs(exp).sum() <= 1e-4
-    big = exp > 1e-3 * exp.mean()
-    assert (np.abs(got - exp)[big] / exp[big]).max() <= 1e-3
+    # every vertex: relative 1e-3 plus an absolute floor of 100 * eps (a
+    # vertex stops at a pending delta < eps; states near 0 -- p_inj ~ 0 --
+    # have no meaningful relative error)
+    assert np.all(np.abs(got - exp) <= 1e-3 * exp + 100 * 1e-7), (np.abs(got - exp) - 1e-3 * exp).max()
 
 
 def test_edge_cases_in_sparse_rounds(sparse_div):

@@ -40,6 +40,8 @@ def _worker(rank, world, port, algo, q, sparse=False, exchange="fused"):
     g = _graph()
     dg = DiGraph(device=0)
     dg.load_graph(g).build_paths(part_entries=256, rank=rank, world=world)
+    if algo == "adsorption":
+        dg.set_vertex_params(*inputs.adsorption_params(g.n, seed=3))
     dev = torch.device("cuda", 0)
     stats, info = parallel.run_distributed(dg, algo, source=0, epsilon=1e-7, device=dev, exchange=exchange)
     out = parallel.gather_states(dg, algo, g.n, device=dev)
@@ -51,7 +53,7 @@ def _worker(rank, world, port, algo, q, sparse=False, exchange="fused"):
 
 @pytest.mark.parametrize("exchange", ["fused", "p2p", "collective"])
 @pytest.mark.parametrize("sparse", [False, True])
-@pytest.mark.parametrize("algo", ["sssp", "wcc", "pagerank"])
+@pytest.mark.parametrize("algo", ["sssp", "wcc", "pagerank", "adsorption"])
 def test_two_ranks_on_one_gpu_match_oracle(algo, sparse, exchange, cuda_required):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -72,6 +74,12 @@ def test_two_ranks_on_one_gpu_match_oracle(algo, sparse, exchange, cuda_required
     elif algo == "wcc":
         exp, _ = OA.wcc_label_propagation(g.n, src, dst)
         assert np.array_equal(got.astype(np.int64), exp)
+    elif algo == "adsorption":
+        p_inj, p_cont, inj = inputs.adsorption_params(g.n, seed=3)
+        exp, _ = OA.adsorption_jacobi(g.n, src, dst, w, p_inj, p_cont, inj, tol=1e-12)
+        got = got.astype(np.float64)
+        assert np.abs(got - exp).sum() / np.abs(exp).sum() <= 1e-4
+        assert np.all(np.abs(got - exp) <= 1e-3 * exp + 100 * 1e-7)
     else:
         exp, _ = OA.pagerank_power(g.n, src, dst)
         assert np.abs(got.astype(np.float64) - exp).sum() <= 1e-4

@@ -140,8 +140,10 @@ def test_adsorption_within_tolerance(name):
     exp, _ = OA.adsorption_jacobi(g.n, src, dst, w, p_inj, p_cont, inj, tol=1e-12)
     scale = np.abs(exp).sum()
     assert np.abs(got - exp).sum() / scale <= PR_L1
-    big = exp > 1e-3 * exp.mean()
-    assert (np.abs(got - exp)[big] / exp[big]).max() <= PR_REL
+    # every vertex: relative 1e-3 plus an absolute floor of 100 * eps (a
+    # vertex stops at a pending delta < eps; states near 0 -- p_inj ~ 0 --
+    # have no meaningful relative error)
+    assert np.all(np.abs(got - exp) <= 1e-3 * exp + 100 * 1e-7), (np.abs(got - exp) - 1e-3 * exp).max()
 
 
 def test_edge_cases():

@@ -52,6 +52,10 @@ class CpuPathEngine:
     def boundary_vertices(self):
         return self.bnd
 
+    def set_vertex_params(self, p_inj, p_cont, inj):
+        """Adsorption inputs (DESIGN.md R-ADS), as dg_set_vertex_params."""
+        self.ads = (np.asarray(p_inj, np.float64), np.asarray(p_cont, np.float64), np.asarray(inj, np.float64))
+
     def run_begin(self, algo, source=0, epsilon=1e-7, damping=0.85):
         self.algo = algo
         if algo in ("sssp", "wcc"):
@@ -62,8 +66,20 @@ class CpuPathEngine:
                 self.x = np.arange(self.n, dtype=np.int64)
         else:
             self.eps = int(epsilon * FX)
-            self.T = np.full(self.n, int((1 - damping) * FX), np.int64)
-            self.coef = np.where(self.outdeg > 0, damping / np.maximum(self.outdeg, 1), 0.0)
+            if algo == "adsorption":
+                # x_v = p_inj I + sum_u p_cont(u) w(u,v)/W(u) x_u: path edge t of a
+                # path carries p_cont(p[t]) * w / W(p[t])
+                p_inj, p_cont, inj = self.ads
+                self.T = np.array([int(x * FX) for x in (p_inj * inj)], np.int64)
+                W = np.zeros(self.n)
+                for (a, _), ws in self.wmap.items():
+                    W[a] += sum(ws)
+                self.ecoef = [[p_cont[u] * wt / W[u] for u, wt in zip(p[:-1].tolist(), ws)]
+                              for p, ws in zip(self.paths, self.pw)]
+            else:
+                self.T = np.full(self.n, int((1 - damping) * FX), np.int64)
+                coef = np.where(self.outdeg > 0, damping / np.maximum(self.outdeg, 1), 0.0)
+                self.ecoef = [[coef[u] for u in p[:-1].tolist()] for p in self.paths]
             self.S = [np.zeros(len(p), np.int64) for p in self.paths]
             self.base = self.T[self.bnd].copy()
 
@@ -93,7 +109,7 @@ class CpuPathEngine:
 
     def _walk_accum(self):
         pushed = 0
-        for p, S in zip(self.paths, self.S):
+        for p, S, ec in zip(self.paths, self.S, self.ecoef):
             carry = 0.0
             for t, v in enumerate(p.tolist()):
                 pin = carry if t > 0 else 0.0
@@ -104,7 +120,7 @@ class CpuPathEngine:
                 if t < len(p) - 1:
                     pend = (self.T[v] - pfx) - S[t]      # the total before this walk's push
                     pend = pend if pend >= self.eps else 0
-                    carry = self.coef[v] * ((pend / FX) + pin)
+                    carry = ec[t] * ((pend / FX) + pin)
                     S[t] += pend + pfx
                 else:
                     carry = 0.0
@@ -216,6 +232,8 @@ def _worker(rank, world, port, algo, q, exchange=None):
     from paper_conf_asplos_zhangl0hlg19_b200 import parallel
     g = inputs.rmat(10, 1024, 6000, seed=21, weights=(1, 20))
     eng = {"p2p": NoPeerEngine, "fused": FusedModelEngine}.get(exchange, CpuPathEngine)(g, rank, world)
+    if algo == "adsorption":
+        eng.set_vertex_params(*inputs.adsorption_params(g.n, seed=3))
     stats, info = parallel.run_distributed(eng, algo, source=0, epsilon=1e-7, device=torch.device("cpu"),
                                            exchange=exchange)
     out = parallel.gather_states(eng, algo, g.n, device=torch.device("cpu"))
@@ -225,8 +243,9 @@ def _worker(rank, world, port, algo, q, exchange=None):
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("algo,exchange", [("sssp", None), ("wcc", None), ("pagerank", None), ("sssp", "p2p"),
-                                           ("sssp", "fused"), ("wcc", "fused"), ("pagerank", "fused")])
+@pytest.mark.parametrize("algo,exchange", [("sssp", None), ("wcc", None), ("pagerank", None), ("adsorption", None),
+                                           ("sssp", "p2p"), ("sssp", "fused"), ("wcc", "fused"),
+                                           ("pagerank", "fused"), ("adsorption", "fused")])
 def test_two_rank_protocol_matches_oracle(algo, exchange):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -249,6 +268,11 @@ def test_two_rank_protocol_matches_oracle(algo, exchange):
     elif algo == "wcc":
         exp, _ = OA.wcc_label_propagation(g.n, src, dst)
         assert np.array_equal(got.astype(np.int64), exp)
+    elif algo == "adsorption":
+        p_inj, p_cont, inj = inputs.adsorption_params(g.n, seed=3)
+        exp, _ = OA.adsorption_jacobi(g.n, src, dst, w, p_inj, p_cont, inj, tol=1e-12)
+        assert np.abs(got - exp).sum() / np.abs(exp).sum() <= 1e-4
+        assert np.all(np.abs(got - exp) <= 1e-3 * exp + 100 * 1e-7)
     else:
         exp, _ = OA.pagerank_power(g.n, src, dst)
         assert np.abs(got - exp).sum() <= 1e-4
