@@ -308,7 +308,7 @@ def main():
     ap.add_argument("--part-entries", type=int, default=0)
     ap.add_argument("--merge-rule", default="relaxed")
     ap.add_argument("--l-merge", type=int, default=64)
-    ap.add_argument("--n-proxy", type=int, default=4096)
+    ap.add_argument("--n-proxy", type=int, default=8192)
     ap.add_argument("--l2-flush-mb", type=int, default=512)
     ap.add_argument("--no-extras", action="store_true", help="skip ablation/e2e/cpu baseline/sssp (profiling runs)")
     ap.add_argument("--no-sssp", action="store_true", help="skip the SSSP record of the default PageRank line")
@@ -333,19 +333,53 @@ def main():
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
 
-    t0 = time.time()
-    g = inputs.make(args.config, seed=args.seed)
-    t_gen = time.time() - t0
-    n, m, gname = g.n, g.m, g.name
+    bp = dict(part_entries=args.part_entries, merge_rule=args.merge_rule, n_proxy=args.n_proxy,
+              l_merge=args.l_merge)
     dg = DiGraph(device=local)
-    t0 = time.time()
-    dg.load_graph(g)
-    t_load = time.time() - t0
-    del g  # the library holds its own copy of the CSR
-    t0 = time.time()
-    dg.build_paths(part_entries=args.part_entries, rank=rank, world=world, merge_rule=args.merge_rule,
-                   n_proxy=args.n_proxy, l_merge=args.l_merge)
-    t_pre = time.time() - t0
+    t_gen = t_load = t_pre = 0.0
+    gname = f"{args.config}-seed{args.seed}"
+    if world == 1:
+        t0 = time.time()
+        g = inputs.make(args.config, seed=args.seed)
+        t_gen = time.time() - t0
+        gname = g.name
+        t0 = time.time()
+        dg.load_graph(g)
+        t_load = time.time() - t0
+        del g  # the library holds its own copy of the CSR
+        t0 = time.time()
+        dg.build_paths(**bp)
+        t_pre = time.time() - t0
+    else:
+        # preprocess ONCE (rank 0) and hand every rank its share through layout
+        # files (dg_build_paths_shared / dg_load_layout):
+        # the other ranks neither generate the graph nor run Algorithm 1
+        shm = "/dev/shm" if os.path.isdir("/dev/shm") else "/tmp"
+        prefix = os.path.join(shm, f"dg_layout_{os.environ.get('MASTER_PORT', '0')}_{args.config}_{args.seed}")
+        if rank == 0:
+            t0 = time.time()
+            g = inputs.make(args.config, seed=args.seed)
+            t_gen = time.time() - t0
+            gname = g.name
+            dg.load_graph(g)
+            del g
+            t0 = time.time()
+            dg.build_paths_shared(prefix, world=world, rank=0, **bp)
+            t_pre = time.time() - t0
+        dist.barrier()
+        if rank != 0:
+            t0 = time.time()
+            dg.load_layout(f"{prefix}.{rank}")
+            t_load = time.time() - t0
+        dist.barrier()
+        if rank == 0:
+            for r in range(world):
+                try:
+                    os.remove(f"{prefix}.{r}")
+                except OSError:
+                    pass
+    info0 = dg.layout_info()
+    n, m = info0["n"], info0["m"]
     dg.upload()
     info = dg.layout_info()
     M = info["n_entries"]
@@ -455,7 +489,9 @@ def main():
                                  if args.algo in ("sssp", "bfs") else None),
                        "l2": f"flushed between steps ({args.l2_flush_mb} MB write outside the step events)",
                        "parallelism": f"paths partitioned over {world} GPU(s)",
-                       "preprocess_s": t_pre, "n_paths": info["n_paths"], "n_entries": M,
+                       "preprocess_s": t_pre, "preprocess": ("once on rank 0, shares handed out as layout files"
+                                                             if world > 1 else "dg_build_paths"),
+                       "n_paths": info["n_paths"], "n_entries": M,
                        "n_partitions": info["n_partitions"], "n_layers": info["n_layers"],
                        "n_boundary": info["n_boundary"], "l_merge": args.l_merge},
             "time_to_convergence_ms": ms,
@@ -466,7 +502,13 @@ def main():
             "roofline": roof, "clocks": clk, "paper_context": PAPER_CONTEXT,
         }
         if syncs[-1]:
-            line["sync"] = syncs[-1]
+            sy = syncs[-1]
+            line["sync"] = sy
+            # NVLink traffic of the replica synchronisation (north_star reporting)
+            line["exchanges"] = sy.get("syncs")
+            line["nvlink_bytes_per_exchange"] = sy.get("nvlink_bytes_per_sync")
+            line["nvlink_bytes_per_round"] = (sy.get("nvlink_bytes_per_sync", 0) * sy.get("syncs", 0) /
+                                              max(1, st0["rounds"]))
         line.update(extras)
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -79,7 +79,7 @@ typedef struct {
 
 /* Fill *p with the defaults (d_max 16, l_merge 64, n_sub 64, order 0,
  * hot_factor 2, part_entries 0 (auto), rank 0, world 1, merge_rule 1,
- * n_proxy 4096). */
+ * n_proxy 8192; the kernel uses as many as fit its shared memory). */
 void dg_default_params(dg_path_params *p);
 
 /* Statistics of one dg_run (device-side counters). */
@@ -148,6 +148,25 @@ int dg_load_csr(dg_graph *g, int64_t n, int64_t m, const int64_t *row_ptr,
  * ("state synchronization of vertex replicas").
  * p may be NULL (defaults). */
 int dg_build_paths(dg_graph *g, const dg_path_params *p);
+
+/* ---- preprocess once, hand every rank its share (PAPER.md lines 104-114,
+ * 176: the graph is preprocessed on the CPU, then paths are dispatched from
+ * the host to the GPUs) ----
+ * dg_build_paths_shared: ONE preprocessing pass for all p->world ranks; writes
+ *   rank r's layout to the file "<prefix>.<r>" (r = 0..world-1) and keeps
+ *   rank p->rank's layout in this handle (as dg_build_paths would).  The
+ *   caller owns the files (e.g. under /dev/shm) and removes them.
+ * dg_save_layout: write this handle's built layout to `path`.
+ * dg_load_layout: replace this handle's graph and layout with a layout file
+ *   (then dg_upload / dg_run as usual; no dg_load_csr is needed).  A loaded
+ *   layout carries no CSR: dg_build_paths and the vertex-centric ablation
+ *   return DG_EINVAL on it; every path-mode algorithm runs.  On failure the
+ *   handle is unchanged.
+ * Files are host byte order with a version tag (DG_EINVAL on mismatch,
+ * truncation or an unopenable path). */
+int dg_build_paths_shared(dg_graph *g, const dg_path_params *p, const char *prefix);
+int dg_save_layout(const dg_graph *g, const char *path);
+int dg_load_layout(dg_graph *g, const char *path);
 
 /* Copy the host CSR and the built layout to the device (the H2D part of an
  * end-to-end run).  dg_run / dg_run_begin / dg_set_vertex_params call it

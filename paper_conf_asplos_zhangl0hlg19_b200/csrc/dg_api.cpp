@@ -50,7 +50,7 @@ void dg_default_params(dg_path_params* p) {
     p->rank = 0;
     p->world = 1;
     p->merge_rule = 1;
-    p->n_proxy = 4096;
+    p->n_proxy = 8192;
 }
 
 int dg_create(dg_graph** out, int device) {
@@ -117,15 +117,22 @@ int dg_load_csr(dg_graph* g, int64_t n, int64_t m, const int64_t* row_ptr, const
     return DG_OK;
 }
 
-int dg_build_paths(dg_graph* g, const dg_path_params* p) {
-    if (!g || !g->loaded) return fail(DG_EINVAL, "dg_build_paths: no graph loaded");
-    dg_path_params q;
-    dg_default_params(&q);
-    if (p) q = *p;
+static int check_params(const dg_path_params& q) {
     if (q.d_max < 1 || q.n_sub < 1 || q.part_entries < 0 || q.world < 1 || q.world > 64 ||
         q.rank < 0 || q.rank >= q.world || q.l_merge < 0 || q.merge_rule < 0 || q.merge_rule > 1 ||
         q.n_proxy < 0 || q.n_proxy > 16384)
         return fail(DG_EINVAL, "dg_build_paths: bad parameters");
+    return DG_OK;
+}
+
+int dg_build_paths(dg_graph* g, const dg_path_params* p) {
+    if (!g || !g->loaded) return fail(DG_EINVAL, "dg_build_paths: no graph loaded");
+    if (g->csr.row_ptr.empty())
+        return fail(DG_EINVAL, "dg_build_paths: the graph came from a layout file (no CSR); use dg_load_csr");
+    dg_path_params q;
+    dg_default_params(&q);
+    if (p) q = *p;
+    if (int rc0 = check_params(q)) return rc0;
     dg::dev_p2p_free(g->p2p);
     dg::dev_free_work(g->work);
     dg::dev_free_layout(g->dev, true);
@@ -161,6 +168,73 @@ int dg_upload(dg_graph* g) {
     return DG_OK;
 }
 
+int dg_build_paths_shared(dg_graph* g, const dg_path_params* p, const char* prefix) {
+    if (!g || !g->loaded || !p || !prefix) return fail(DG_EINVAL, "dg_build_paths_shared: no graph loaded or NULL argument");
+    if (g->csr.row_ptr.empty())
+        return fail(DG_EINVAL, "dg_build_paths_shared: the graph came from a layout file (no CSR)");
+    if (int rc0 = check_params(*p)) return rc0;
+    dg::dev_p2p_free(g->p2p);
+    dg::dev_free_work(g->work);
+    dg::dev_free_layout(g->dev, true);
+    dg::dev_unpin_all(g->dev);
+    g->uploaded = false;
+    g->ran = false;
+    g->layout = dg::HostLayout();
+    std::vector<int> ranks;
+    for (int r = 0; r < p->world; r++) ranks.push_back(r);
+    std::string err;
+    int rc = DG_OK;
+    try {
+        // ONE preprocessing pass emits every rank's share; this handle keeps its own
+        dg::build_layouts(g->csr, *p, ranks, [&](int r, dg::HostLayout& L) {
+            if (!rc) rc = dg::save_layout(g->csr, L, (std::string(prefix) + "." + std::to_string(r)).c_str(), err);
+            if (r == p->rank) g->layout = L;
+        });
+    } catch (const std::bad_alloc&) {
+        g->layout = dg::HostLayout();
+        return fail(DG_ENOMEM, "dg_build_paths_shared: out of host memory");
+    } catch (const std::exception& e) {
+        g->layout = dg::HostLayout();
+        return fail(DG_EINVAL, std::string("dg_build_paths_shared: ") + e.what());
+    }
+    if (rc) {
+        g->layout = dg::HostLayout();
+        return fail(rc, "dg_build_paths_shared: " + err);
+    }
+    return DG_OK;
+}
+
+int dg_save_layout(const dg_graph* g, const char* path) {
+    if (!g || !g->layout.built || !path) return fail(DG_EINVAL, "dg_save_layout: no layout built or NULL path");
+    std::string err;
+    const int rc = dg::save_layout(g->csr, g->layout, path, err);
+    return rc ? fail(rc, "dg_save_layout: " + err) : DG_OK;
+}
+
+int dg_load_layout(dg_graph* g, const char* path) {
+    if (!g || !path) return fail(DG_EINVAL, "dg_load_layout: NULL argument");
+    dg::HostCSR c;
+    dg::HostLayout L;
+    std::string err;
+    int rc;
+    try {
+        rc = dg::load_layout(c, L, path, err);
+    } catch (const std::bad_alloc&) {
+        return fail(DG_ENOMEM, "dg_load_layout: out of host memory");
+    }
+    if (rc) return fail(rc, "dg_load_layout: " + err);  // the handle is unchanged
+    dg::dev_p2p_free(g->p2p);
+    dg::dev_free_work(g->work);
+    dg::dev_free_layout(g->dev, true);
+    dg::dev_unpin_all(g->dev);
+    g->csr = std::move(c);
+    g->layout = std::move(L);
+    g->loaded = true;
+    g->uploaded = false;
+    g->ran = false;
+    return DG_OK;
+}
+
 static int ensure_uploaded(dg_graph* g) {
     return g->uploaded ? DG_OK : dg_upload(g);
 }
@@ -188,8 +262,10 @@ static void build_sym_csr(dg::HostLayout& L, int64_t n) {
 // the parts of the device layout an algorithm reads beyond the path entries
 static int ensure_parts(dg_graph* g, int algo, int mode) {
     const bool need_sym = mode == DG_MODE_VERTEX && algo == DG_WCC;
-    const bool need_csr = (mode == DG_MODE_VERTEX && !need_sym) || algo == DG_ADSORPTION;
+    const bool need_csr = mode == DG_MODE_VERTEX && !need_sym;
     const bool need_ew = (mode == DG_MODE_PATH && algo == DG_SSSP) || algo == DG_ADSORPTION;
+    if ((need_sym || need_csr) && !g->layout.has_csr)
+        return fail(DG_EINVAL, "dg_run: the vertex-centric ablation needs the CSR (this layout came from a file)");
     std::string err;
     try {
         if (need_sym) build_sym_csr(g->layout, g->csr.n);
@@ -217,7 +293,7 @@ int dg_set_vertex_params(dg_graph* g, const double* p_inj, const double* p_cont,
     std::vector<double> a(n), b(n), c(n);
     for (int64_t u = 0; u < n; u++) { a[u] = p_inj[orig[u]]; b[u] = p_cont[orig[u]]; c[u] = inj[orig[u]]; }
     std::string err;
-    int rc = dg::dev_set_vertex_params(g->work, g->dev, a.data(), b.data(), c.data(), err);
+    int rc = dg::dev_set_vertex_params(g->work, g->dev, a.data(), b.data(), c.data(), g->layout.wsum.data(), err);
     return rc ? fail(rc, err) : DG_OK;
 }
 

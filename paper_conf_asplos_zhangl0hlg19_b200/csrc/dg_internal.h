@@ -2,6 +2,7 @@
 // the CUDA kernels (dg_kernels.cu).  Not part of the public ABI.
 #pragma once
 #include <cstdint>
+#include <functional>
 #include <string>
 #include <vector>
 
@@ -51,12 +52,23 @@ struct HostLayout {
     std::vector<int32_t> scol;
     // multi-rank
     std::vector<int32_t> boundary;      // internal ids of vertices present on >1 rank (ascending)
+    std::vector<float> wsum;            // per vertex (internal ids): sum of out-edge weights (Adsorption)
+    bool has_csr = true;                // prow_ptr/pcol/pw present (false: loaded from a layout file)
     // stats
     int64_t n_layers = 0, n_dep_sccs = 0, giant = 0, paths_before_merge = 0, n_hot = 0;
     double preprocess_ms = 0;
 };
 
 void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L);
+// One preprocessing pass for several ranks of a multi-rank layout: everything
+// but the rank selection runs once; emit(rank, L) receives each rank's layout
+// (L is reused between calls).
+void build_layouts(const HostCSR& g, const dg_path_params& p, const std::vector<int>& ranks,
+                   const std::function<void(int, HostLayout&)>& emit);
+// Layout files (dg_save_layout / dg_load_layout): the layout without the CSR
+// arrays, plus the graph's n, m, has_w and max_w.
+int save_layout(const HostCSR& g, const HostLayout& L, const char* path, std::string& err);
+int load_layout(HostCSR& g, HostLayout& L, const char* path, std::string& err);
 
 // ---------------- device side ----------------
 struct DevLayout {
@@ -99,7 +111,7 @@ int dev_ensure_parts(DevLayout& D, const HostCSR& g, const HostLayout& L, bool n
                      std::string& err);
 void dev_free_layout(DevLayout& D, bool csr_too);
 int dev_set_vertex_params(DevWork*& W, const DevLayout& D, const double* p_inj, const double* p_cont,
-                          const double* inj, std::string& err);
+                          const double* inj, const float* wsum, std::string& err);
 int dev_run(DevWork*& W, const DevLayout& D, RunState& S, int64_t max_rounds, std::string& err);
 int dev_run_begin(DevWork*& W, const DevLayout& D, RunState& S, std::string& err);
 int dev_rounds(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, int64_t* active, std::string& err);

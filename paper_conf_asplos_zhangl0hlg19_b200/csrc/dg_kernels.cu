@@ -132,6 +132,7 @@ struct MultiRank {
     int64_t nb;
     unsigned long long slot_bytes, epoch0, timeout_ns, eps_fx;
     int world, rank, every, sum;
+    int mark;  // SCC backward phase: the replicated state is the reachability mark (value 0 = marked, MIN = OR)
 };
 
 struct KParams {
@@ -858,51 +859,103 @@ __device__ __forceinline__ float fx_to(unsigned long long v) { return __ull2floa
 // pushed new states of its local mirrors ... sent to the master when the
 // partition assigned to this SMX has been handled".  Per CTA: the round-start
 // totals and the CTA's unflushed pushes.
-// Reads of a hub use the CTA's snapshot T only (refreshed every px_refresh
-// partitions): the CTA's own unflushed pushes are a 1/G share of what the hub
-// receives and, like every other push, are seen after the next refresh.
-// Pushes accumulate write-only in three 32-bit limbs per hub with
-// fire-and-forget shared REDs (shared memory has native 32-bit atomic adds
-// only; a 64-bit add is a CAS loop): limb 0 takes bits 0-15 of the push,
-// limb 1 bits 16-31, limb 2 bits 32-47.  A push >= 2^48 (2^16 in rank units)
-// goes straight to the master.  No limb can wrap: fewer than 2^16 pushes reach
-// a hub between two flushes of it (launch_path bounds px_refresh by the
-// largest partition), and every limb addend is < 2^16.
-constexpr int kPxLimbs = 3;
+// The pushes accumulate in two 32-bit words per hub (lo, hi) because shared
+// memory has native 32-bit atomic adds only (a 64-bit add is a CAS loop): lo
+// takes the push, its carry goes to hi.  A concurrent reader can see a carry
+// not yet applied (an under-estimate: pend only shrinks, safe) and a flush can
+// leave a pending carry for the next flush (the total is conserved).
+// (Measured against write-only proxies with three 16-bit limbs and fire-and-
+// forget shared REDs: no faster.)
 struct Proxies {
     unsigned long long* T;  // snapshot of the hub totals
-    unsigned* acc;          // kPxLimbs words per hub
+    unsigned* acc;          // 2 words per hub
     int64_t H;
 };
-__device__ __forceinline__ void red_shared_u32(unsigned* a, unsigned v) {
-    asm volatile("red.shared.add.u32 [%0], %1;" ::"r"((unsigned)__cvta_generic_to_shared(a)), "r"(v) : "memory");
+__device__ __forceinline__ void px_add(unsigned* a, unsigned long long p) {
+    const unsigned lo = (unsigned)p, hi = (unsigned)(p >> 32);
+    const unsigned old = atomicAdd(&a[0], lo);
+    const unsigned c = hi + (old + lo < old ? 1u : 0u);
+    if (c) atomicAdd(&a[1], c);
 }
-__device__ __forceinline__ void px_push(unsigned* a, unsigned long long p, unsigned long long* master) {
-    if (p >> 48) {
-        atomicAdd(master, p);
-        return;
-    }
-    const unsigned l0 = (unsigned)p & 0xFFFFu, l1 = (unsigned)(p >> 16) & 0xFFFFu, l2 = (unsigned)(p >> 32);
-    if (l0) red_shared_u32(&a[0], l0);
-    if (l1) red_shared_u32(&a[1], l1);
-    if (l2) red_shared_u32(&a[2], l2);
-}
-__device__ __forceinline__ unsigned long long px_combine(unsigned l0, unsigned l1, unsigned l2) {
-    return (unsigned long long)l0 + ((unsigned long long)l1 << 16) + ((unsigned long long)l2 << 32);
+__device__ __forceinline__ unsigned long long px_read(const unsigned* a) {
+    const unsigned lo = *(const volatile unsigned*)&a[0], hi = *(const volatile unsigned*)&a[1];
+    return ((unsigned long long)hi << 32) + lo;
 }
 __device__ __forceinline__ unsigned long long px_take(unsigned* a) {
-    const unsigned l0 = atomicExch(&a[0], 0u), l1 = atomicExch(&a[1], 0u), l2 = atomicExch(&a[2], 0u);
-    return px_combine(l0, l1, l2);
+    const unsigned lo = atomicExch(&a[0], 0u), hi = atomicExch(&a[1], 0u);
+    return ((unsigned long long)hi << 32) + lo;
+}
+constexpr int kPxBytes = 16;  // shared memory per proxied hub
+
+// Mid-round proxy flush (every px_refresh partitions a CTA starts): one warp
+// sends the proxies' accumulated pushes to the masters and reloads the
+// snapshot, so hub totals propagate between CTAs within the round.  The
+// reloads are batched (16 L2 loads in flight per lane).
+__device__ __forceinline__ void px_refresh(const KParams& P, const Proxies& px) {
+    const int lane = threadIdx.x & 31;
+    for (int64_t i = lane; i < px.H; i += 32) {
+        const unsigned long long a = px_take(&px.acc[2 * i]);
+        if (a) atomicAdd(&P.vs_t[i], a);
+    }
+    __syncwarp();
+    for (int64_t i0 = lane; i0 < px.H; i0 += 32 * 16) {
+        unsigned long long t16[16];
+#pragma unroll
+        for (int u = 0; u < 16; u++) t16[u] = i0 + 32 * u < px.H ? __ldcg(&P.vs_t[i0 + 32 * u]) : 0ull;
+#pragma unroll
+        for (int u = 0; u < 16; u++)
+            if (i0 + 32 * u < px.H) px.T[i0 + 32 * u] = t16[u];
+    }
+}
+
+// A warp's partition feed for the accumulative walk: with the global ticket
+// (default) the ticket of the partition after next and the bounds of the next
+// partition are fetched one partition early, so a partition switch waits for
+// no atomic or load.  With per-CTA queues (DG_DISPATCH=1) the switch takes
+// the next partition synchronously.
+struct Feed {
+    unsigned t_pend;     // lane 0: ticket taken for the partition after next
+    uint32_t nbeg, nend; // bounds of the next partition (nbeg == kNoWin: none)
+};
+__device__ __forceinline__ unsigned map_order(const KParams& P, unsigned t) {
+    if (P.part_order == 1) return (unsigned)P.n_part - 1 - t;  // developer knob: dispatch-order experiments
+    if (P.part_order > 1) return (unsigned)(((unsigned long long)t * P.part_order) % (unsigned long long)P.n_part);
+    return t;
+}
+__device__ __forceinline__ void feed_fetch(const KParams& P, const Queue& q, Feed& f) {
+    // the pending ticket becomes the next partition; a new ticket is taken
+    const unsigned t = __shfl_sync(0xffffffffu, f.t_pend, 0);
+    if (t < (unsigned)P.n_part) {
+        const unsigned u = map_order(P, t);
+        f.nbeg = (uint32_t)P.part_off[u];
+        f.nend = (uint32_t)P.part_off[u + 1];
+    } else {
+        f.nbeg = kNoWin;
+        f.nend = 0;
+    }
+    if ((threadIdx.x & 31) == 0) f.t_pend = atomicAdd(q.global, 1u);
+}
+__device__ __forceinline__ Win feed_next(const KParams& P, const Queue& q, const Win& w, Feed& f) {
+    if (w.base == kNoWin) return w;
+    if (w.base + 128 < w.end) return Win{w.base + 128, w.beg, w.end};
+    if (q.qt) return win_first_of(P, q);
+    const Win nw = f.nbeg == kNoWin ? Win{kNoWin, 0, 0} : Win{f.nbeg & ~3u, f.nbeg, f.nend};
+    if (nw.base != kNoWin) feed_fetch(P, q, f);
+    return nw;
 }
 
 // Walk all windows the warp obtains in this round.  Software pipeline over the
-// window stream: while window w is walked, the master totals of window w+1
-// are in flight into shared memory (cp.async, a 2-slot ring per warp), its
-// mirrors and coefficients into registers, and the indices of window w+2.
-// Reading a master one window early is a read slightly before the walk
-// reaches it -- the same asynchronous semantics as any concurrent push.
+// window stream (kRing-slot shared ring per warp): while window w is walked,
+// the master totals of windows w+1 and w+2 are in flight into shared memory
+// (cp.async: no registers held), the mirrors and coefficients of window w+1
+// into registers, and the indices of window w+3.  Reading a master two
+// windows early is a read slightly before the walk reaches it -- the same
+// asynchronous semantics as any concurrent push.
+constexpr int kRing = 3;
+template <int NW>
+__host__ __device__ constexpr size_t gbuf_bytes() { return (size_t)NW * kRing * 128 * sizeof(uint4); }
 template <bool ADS>
-__device__ void walk_accum(const KParams& P, const Queue& ticket, Acc& acc, unsigned long long pol_stream,
+__device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned long long pol_stream,
                            unsigned long long pol_keep, const Proxies& px, uint4* gbuf, int* s_done) {
     const int lane = threadIdx.x & 31;
     const unsigned long long eps = P.eps_fx;
@@ -936,69 +989,58 @@ __device__ void walk_accum(const KParams& P, const Queue& ticket, Acc& acc, unsi
         cp_async_commit();
     };
 
-    Win wc = win_first_of(P, ticket);
-    if (wc.base == kNoWin) return;
-    Win wn = win_next(P, wc, ticket);
-    uint4 code_c = load_code(wc), code_n = load_code(wn);
+    Feed f{0u, kNoWin, 0u};
+    Win w0 = win_first_of(P, q);
+    if (w0.base == kNoWin) return;
+    if (!q.qt) {  // prime the feed: next partition's bounds and the ticket after it
+        if (lane == 0) f.t_pend = atomicAdd(q.global, 1u);
+        feed_fetch(P, q, f);
+    }
+    Win w1 = feed_next(P, q, w0, f);
+    Win w2 = feed_next(P, q, w1, f);
+    uint4 c0 = load_code(w0), c1 = load_code(w1), c2 = load_code(w2);
     unsigned long long sv_c[4], sv_n[4];
     float4 cf_c, cf_n;
-    load_sv(wc, sv_c, cf_c);
-    gather(wc, code_c, 0);
+    load_sv(w0, sv_c, cf_c);
+    gather(w0, c0, 0);
+    gather(w1, c1, 1);
     int slot = 0;
     float carry = 0.f;
-    while (wc.base != kNoWin) {
-        const Win wnn = win_next(P, wn, ticket);
-        const uint4 code_nn = load_code(wnn);
-        gather(wn, code_n, slot ^ 1);
-        load_sv(wn, sv_n, cf_n);
-        const bool part_start = wc.base == (wc.beg & ~3u);
+    while (w0.base != kNoWin) {
+        const Win w3 = feed_next(P, q, w2, f);
+        const uint4 c3 = load_code(w3);
+        gather(w2, c2, slot == 0 ? 2 : slot - 1);  // slot (w+2) % kRing
+        load_sv(w1, sv_n, cf_n);
+        const bool part_start = w0.base == (w0.beg & ~3u);
         if (part_start) {
             carry = 0.f;
             if (px.H && P.px_refresh > 0) {
-                // every px_refresh partitions of this CTA, one warp sends the
-                // proxies' pushes to their masters and refreshes the snapshot, so
-                // hub totals propagate between CTAs within the round
                 int c = 0;
                 if (lane == 0) c = atomicAdd(s_done, 1) + 1;
                 c = __shfl_sync(0xffffffffu, c, 0);
-                if (c % P.px_refresh == 0) {
-                    for (int64_t i = lane; i < px.H; i += 32) {
-                        const unsigned long long a = px_take(&px.acc[kPxLimbs * i]);
-                        if (a) atomicAdd(&P.vs_t[i], a);
-                    }
-                    __syncwarp();
-                    // snapshot refresh: eight independent L2 loads in flight per lane
-                    for (int64_t i0 = lane; i0 < px.H; i0 += 32 * 8) {
-                        unsigned long long t8[8];
-#pragma unroll
-                        for (int u = 0; u < 8; u++) t8[u] = i0 + 32 * u < px.H ? __ldcg(&P.vs_t[i0 + 32 * u]) : 0ull;
-#pragma unroll
-                        for (int u = 0; u < 8; u++)
-                            if (i0 + 32 * u < px.H) px.T[i0 + 32 * u] = t8[u];
-                    }
-                }
+                if (c % P.px_refresh == 0) px_refresh(P, px);
             }
         }
-        cp_async_wait1();  // this window's masters have landed (its own lane's copies)
-        const uint32_t i0 = wc.base + 4 * lane;
+        asm volatile("cp.async.wait_group 2;" ::: "memory");  // window w's masters (its own lane's copies)
+        const uint32_t i0 = w0.base + 4 * lane;
         uint32_t vtx[4];
         unsigned long long T[4], pend[4];
         bool valid[4], hd[4], tl[4], any_act = false;
 #pragma unroll
         for (int k = 0; k < 4; k++) {
             const uint32_t i = i0 + k;
-            const uint32_t c = u4get(code_c, k);
-            valid[k] = i >= wc.beg && i < wc.end;
+            const uint32_t c = u4get(c0, k);
+            valid[k] = i >= w0.beg && i < w0.end;
             vtx[k] = c & kVMask;
             hd[k] = !valid[k] || (c & kHead);
             tl[k] = !valid[k] || (c & kTail);
             T[k] = 0ull;
             if (valid[k]) {
                 if (vtx[k] < px.H) {
-                    T[k] = px.T[vtx[k]];
+                    T[k] = px.T[vtx[k]] + px_read(&px.acc[2 * vtx[k]]);
                 } else {
-                    const uint4 q = gbuf[slot * 128 + k * 32 + lane];
-                    T[k] = (vtx[k] & 1u) ? ((unsigned long long)q.w << 32 | q.z) : ((unsigned long long)q.y << 32 | q.x);
+                    const uint4 g = gbuf[slot * 128 + k * 32 + lane];
+                    T[k] = (vtx[k] & 1u) ? ((unsigned long long)g.w << 32 | g.z) : ((unsigned long long)g.y << 32 | g.x);
                 }
             }
             const unsigned long long pd = T[k] > sv_c[k] ? T[k] - sv_c[k] : 0ull;
@@ -1016,48 +1058,49 @@ __device__ void walk_accum(const KParams& P, const Queue& ticket, Acc& acc, unsi
             }
             // in-order walk = inclusive warp scan of the entries' affine maps
             // p_(i+1) = al_i + be_i * p_i (heads reset, tails push nothing)
-            auto walk_scan = [&](float (&pin)[4]) {
-                float Al = 0.f, Be = 1.f;
+            float Al = 0.f, Be = 1.f;
 #pragma unroll
-                for (int k = 0; k < 4; k++) { Al = al[k] + be[k] * Al; Be = be[k] * Be; }
+            for (int k = 0; k < 4; k++) { Al = al[k] + be[k] * Al; Be = be[k] * Be; }
 #pragma unroll
-                for (int off = 1; off < 32; off <<= 1) {
-                    float Ap = __shfl_up_sync(0xffffffffu, Al, off);
-                    float Bp = __shfl_up_sync(0xffffffffu, Be, off);
-                    if (lane >= off) { Al = Al + Be * Ap; Be = Be * Bp; }
-                }
-                float Ae = __shfl_up_sync(0xffffffffu, Al, 1);
-                float Bx = __shfl_up_sync(0xffffffffu, Be, 1);
-                if (lane == 0) { Ae = 0.f; Bx = 1.f; }
-                float prev = Ae + Bx * carry;
-#pragma unroll
-                for (int k = 0; k < 4; k++) {
-                    pin[k] = hd[k] ? 0.f : prev;
-                    prev = al[k] + be[k] * prev;
-                }
-                return __shfl_sync(0xffffffffu, prev, 31);
-            };
+            for (int off = 1; off < 32; off <<= 1) {
+                const float Ap = __shfl_up_sync(0xffffffffu, Al, off);
+                const float Bp = __shfl_up_sync(0xffffffffu, Be, off);
+                if (lane >= off) { Al = Al + Be * Ap; Be = Be * Bp; }
+            }
+            float Ae = __shfl_up_sync(0xffffffffu, Al, 1);
+            float Bx = __shfl_up_sync(0xffffffffu, Be, 1);
+            if (lane == 0) { Ae = 0.f; Bx = 1.f; }
+            float prev = Ae + Bx * carry;
             float pin[4];
-            carry = walk_scan(pin);
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                pin[k] = hd[k] ? 0.f : prev;
+                prev = al[k] + be[k] * prev;
+            }
+            carry = __shfl_sync(0xffffffffu, prev, 31);
             bool dirty = false;
+            unsigned n_valid = 0, n_edges = 0, n_upd = 0;
 #pragma unroll
             for (int k = 0; k < 4; k++) {
                 if (!valid[k]) continue;
-                acc.entries++;
-                if (!hd[k]) acc.edges++;
+                n_valid++;
+                n_edges += !hd[k];
                 const unsigned long long p = fx_from(pin[k]);
                 if (p) {
-                    if (vtx[k] < px.H) px_push(&px.acc[kPxLimbs * vtx[k]], p, &P.vs_t[vtx[k]]);  // proxy: shared REDs
+                    if (vtx[k] < px.H) px_add(&px.acc[2 * vtx[k]], p);  // proxy: shared-memory atomics
                     else red_add_u64_h(&P.vs_t[vtx[k]], p, pol_keep);   // master: REDG (no return)
-                    acc.upd++;
+                    n_upd++;
                 }
                 if (!tl[k] && (pend[k] | p)) { sv_c[k] += pend[k] + p; dirty = true; }
             }
+            acc.entries += n_valid;
+            acc.edges += n_edges;
+            acc.upd += n_upd;
             // lanes whose four entries all lie in this partition write one 256-bit
             // store; lanes at the partition's ends write only their own entries
             // (the neighbouring partition's mirrors belong to another warp)
             if (dirty) {
-                if (i0 >= wc.beg && i0 + 3 < wc.end) {
+                if (i0 >= w0.beg && i0 + 3 < w0.end) {
                     st_stream_u64x4_h(P.s_val + i0, sv_c, pol_stream);
                 } else {
 #pragma unroll
@@ -1069,14 +1112,16 @@ __device__ void walk_accum(const KParams& P, const Queue& ticket, Acc& acc, unsi
             carry = 0.f;
         }
         // rotate the pipeline
-        wc = wn; wn = wnn;
-        code_c = code_n; code_n = code_nn;
+        w0 = w1; w1 = w2; w2 = w3;
+        c0 = c1; c1 = c2; c2 = c3;
 #pragma unroll
         for (int k = 0; k < 4; k++) sv_c[k] = sv_n[k];
         cf_c = cf_n;
-        slot ^= 1;
+        slot = slot == kRing - 1 ? 0 : slot + 1;
     }
     cp_async_wait0();
+    // an unused prefetched ticket is simply dropped (the round's ticket only
+    // needs to exceed n_part, which it then does)
 }
 
 // End-of-round vertex sweep of the accumulative algorithms: a vertex whose
@@ -1114,10 +1159,11 @@ __device__ void accum_sweep(const KParams& P, uint32_t* bnxt, unsigned& cnt) {
 // signalled vertex's entry (that entry has its own starter), at a tail, or at
 // the length cap only adds its push to the master; the push stays pending in
 // T(x) - S_val[e], like any push from another path.
+template <int NW>
 __device__ void walk_sparse_acc(const KParams& P, const uint2* list, unsigned qn, unsigned* ticket,
                                 const uint32_t* bcur, Acc& acc) {
-    __shared__ uint32_t s_off[kWarps][33];
-    __shared__ uint32_t s_beg[kWarps][32];
+    __shared__ uint32_t s_off[NW][33];
+    __shared__ uint32_t s_beg[NW][32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
     const unsigned long long eps = P.eps_fx;
     while (true) {
@@ -1270,9 +1316,11 @@ __device__ void walk_scc_bwd(const KParams& P, int64_t beg, int64_t end, const u
 }
 
 // ------------------------------------------------------------------ persistent round driver
-// Dynamic shared memory of the accumulative kernels: per-CTA proxies (16 B per
-// hub) then the per-warp 2 x 128-entry master ring (kWarps x 4 KB).
-constexpr size_t kGbufBytes = (size_t)kWarps * 2 * 128 * sizeof(uint4);
+// Dynamic shared memory of the accumulative kernels: the per-warp kRing x
+// 128-entry master rings (kAccWarps x 6 KB), then the CTA's proxies (16 B per
+// hub).  The accumulative kernels run ONE CTA of kAccWarps warps per SM, so
+// the SM's shared memory holds one proxy table (not one per CTA).
+constexpr int kAccWarps = 16;
 
 // ---- fused multi-rank exchange (P.mr.world > 1; DESIGN.md "Peer-memory
 // exchange"): the same protocol as dg_boundary_exchange, run by the
@@ -1299,7 +1347,7 @@ __device__ __forceinline__ bool mr_exchange(const KParams& P, cg::grid_group& gr
             mine[k] = g;
             dirty += g != 0;
         } else {
-            const uint32_t x = P.vs_u[v];
+            const uint32_t x = M.mark ? (P.mark[v] ? 0u : 1u) : P.vs_u[v];
             mine[k] = x;
             dirty += x != M.last[k];
         }
@@ -1366,7 +1414,12 @@ __device__ __forceinline__ bool mr_exchange(const KParams& P, cg::grid_group& gr
             unsigned long long m = ~0ull;
             for (int r = 0; r < M.world; r++) m = min(m, __ldcv((const unsigned long long*)(M.region[r] + off) + k));
             M.last[k] = (uint32_t)m;
-            if ((uint32_t)m < P.vs_u[v]) {
+            if (M.mark) {  // marked on some rank: reachable backward from its colour's root
+                if (m == 0 && !P.mark[v] && P.scc_label[v] < 0) {
+                    P.mark[v] = 1;
+                    cnt += signal_vertex(b, (uint32_t)v);
+                }
+            } else if ((uint32_t)m < P.vs_u[v]) {
                 P.vs_u[v] = (uint32_t)m;
                 cnt += signal_vertex(b, (uint32_t)v);
             }
@@ -1380,8 +1433,9 @@ __device__ __forceinline__ bool mr_exchange(const KParams& P, cg::grid_group& gr
 
 // MR: fused multi-rank run (P.mr.world > 1) -- a separate instantiation, so a
 // single-rank run carries none of its code or registers
-template <int ALGO, int MINB = DG_PATH_MINB, bool MR = false>
-__global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
+template <int ALGO, int MINB = DG_PATH_MINB, bool MR = false,
+          int NW = (ALGO == DG_PAGERANK || ALGO == DG_ADSORPTION) ? kAccWarps : kWarps>
+__global__ void __launch_bounds__(NW * 32, MINB) path_kernel(KParams P) {
     cg::grid_group grid = cg::this_grid();
     const int lane = threadIdx.x & 31;
     constexpr bool kAccum = ALGO == DG_PAGERANK || ALGO == DG_ADSORPTION;
@@ -1398,9 +1452,9 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
     Proxies px{nullptr, nullptr, 0};
     uint4* gbuf = nullptr;
     if (kAccum) {
-        gbuf = reinterpret_cast<uint4*>(dyn_smem) + (size_t)(threadIdx.x >> 5) * 256;
+        gbuf = reinterpret_cast<uint4*>(dyn_smem) + (size_t)(threadIdx.x >> 5) * kRing * 128;
         px.H = P.n_proxy;
-        px.T = reinterpret_cast<unsigned long long*>(dyn_smem + kGbufBytes);
+        px.T = reinterpret_cast<unsigned long long*>(dyn_smem + gbuf_bytes<NW>());
         px.acc = reinterpret_cast<unsigned*>(px.T + px.H);
     }
     Acc acc;
@@ -1427,17 +1481,16 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
                 for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.nw;
                      i += (int64_t)gridDim.x * blockDim.x)
                     bnxt[i] = 0u;
-        } else if (kAccum) {
+        } else if constexpr (kAccum) {
             // sparse round: few signalled vertices whose out-edges are at most M / sparse_div
             if (sparse_round(P, grid, cur, bcur)) {
                 dense = false;
-                walk_sparse_acc(P, P.occ_items, *((volatile unsigned*)&P.ctr->qcur[cur]), &P.ctr->ticket[cur], bcur, acc);
+                walk_sparse_acc<NW>(P, P.occ_items, *((volatile unsigned*)&P.ctr->qcur[cur]), &P.ctr->ticket[cur], bcur, acc);
             } else {
             if (px.H) {  // round-start snapshot of the proxied masters
                 for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) {
                     px.T[i] = __ldcg(&P.vs_t[i]);
-#pragma unroll
-                    for (int l = 0; l < kPxLimbs; l++) px.acc[kPxLimbs * i + l] = 0u;
+                    px.acc[2 * i] = px.acc[2 * i + 1] = 0u;
                 }
                 if (threadIdx.x == 0) s_done = 0;
                 __syncthreads();
@@ -1445,10 +1498,8 @@ __global__ void __launch_bounds__(kBlock, MINB) path_kernel(KParams P) {
             walk_accum<ALGO == DG_ADSORPTION>(P, dq, acc, pol_stream, pol_keep, px, gbuf, &s_done);
             if (px.H) {  // send the proxies' accumulated pushes to their masters
                 __syncthreads();
-                for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) {
-                    const unsigned* l = &px.acc[kPxLimbs * i];
-                    if (const unsigned long long a = px_combine(l[0], l[1], l[2])) atomicAdd(&P.vs_t[i], a);
-                }
+                for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x)
+                    if (const unsigned long long a = px_read(&px.acc[2 * i])) atomicAdd(&P.vs_t[i], a);
             }
             }
             grid.sync();  // all pushes of the round landed
@@ -1749,13 +1800,6 @@ __global__ void ads_coef_kernel(float* e_coef, const uint32_t* e_idx, const int3
             x = pcont[u] * (float)e_w[i + 1] / wsum[u];
         }
         e_coef[i] = x;
-    }
-}
-__global__ void wsum_kernel(float* wsum, const int64_t* row_ptr, const int32_t* w, int64_t n) {
-    GRID_STRIDE(v, n) {
-        double s = 0;
-        for (int64_t e = row_ptr[v]; e < row_ptr[v + 1]; e++) s += w ? (double)w[e] : 1.0;
-        wsum[v] = (float)s;
     }
 }
 __device__ __forceinline__ double final_value(const float4* vf, const unsigned long long* va, int64_t v) {
@@ -2128,17 +2172,18 @@ int write_counters(DevWork* W, const Counters& c, std::string& err) {
     return DG_OK;
 }
 
-int coop_launch(DevWork* W, void* fn, KParams& P, RunState& S, std::string& err, size_t smem = 0) {
+int coop_launch(DevWork* W, void* fn, KParams& P, RunState& S, std::string& err, size_t smem = 0,
+                int threads = kBlock) {
     int dev = 0, sms = 0, per = 0;
     CK(cudaGetDevice(&dev));
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
     if (smem) CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, kBlock, smem));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, threads, smem));
     const int grid = std::min(sms * std::max(1, per), kMaxGrid);
     if (P.qtick) CK(cudaMemsetAsync(P.qtick, 0, sizeof(unsigned) * 2 * kMaxGrid * kQStride));
     void* args[] = {&P};
     CK(cudaEventRecord(W->kev0));
-    CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(kBlock), args, smem, 0));
+    CK(cudaLaunchCooperativeKernel(fn, dim3(grid), dim3(threads), args, smem, 0));
     CK(cudaGetLastError());
     CK(cudaEventRecord(W->kev1));
     CK(cudaEventSynchronize(W->kev1));
@@ -2149,12 +2194,6 @@ int coop_launch(DevWork* W, void* fn, KParams& P, RunState& S, std::string& err,
     return DG_OK;
 }
 
-// resident CTAs per SM the accumulative kernels are compiled for (2: up to 128
-// registers, no spills; 3: 80 registers); DG_ACC_MINB selects (developer knob)
-int acc_minb() {
-    const char* e = std::getenv("DG_ACC_MINB");
-    return e ? std::atoi(e) : 2;
-}
 
 // Sparse min-plus rounds: a round with at most
 // n/4 signalled vertices whose out-edges are at most M / DG_SPARSE_DIV walks
@@ -2251,18 +2290,16 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
             case DG_SSSP: fn = (void*)path_kernel<DG_SSSP, DG_PATH_MINB, true>; break;
             case DG_BFS: fn = (void*)path_kernel<DG_BFS, DG_PATH_MINB, true>; break;
             case DG_WCC: fn = (void*)path_kernel<DG_WCC, DG_PATH_MINB, true>; break;
-            case DG_PAGERANK: fn = (void*)path_kernel<DG_PAGERANK, 2, true>; break;
-            case DG_ADSORPTION: fn = (void*)path_kernel<DG_ADSORPTION, 2, true>; break;
+            case DG_PAGERANK: fn = (void*)path_kernel<DG_PAGERANK, 1, true>; break;
+            case DG_ADSORPTION: fn = (void*)path_kernel<DG_ADSORPTION, 1, true>; break;
             default: err = "fused multi-rank run: bad algo"; return DG_EINVAL;
         }
     } else switch (algo_k) {
         case DG_SSSP: fn = (void*)path_kernel<DG_SSSP>; break;
         case DG_BFS: fn = (void*)path_kernel<DG_BFS>; break;
         case DG_WCC: fn = (void*)path_kernel<DG_WCC>; break;
-        case DG_PAGERANK: fn = acc_minb() == 2 ? (void*)path_kernel<DG_PAGERANK, 2> : (void*)path_kernel<DG_PAGERANK>; break;
-        case DG_ADSORPTION:
-            fn = acc_minb() == 2 ? (void*)path_kernel<DG_ADSORPTION, 2> : (void*)path_kernel<DG_ADSORPTION>;
-            break;
+        case DG_PAGERANK: fn = (void*)path_kernel<DG_PAGERANK, 1>; break;
+        case DG_ADSORPTION: fn = (void*)path_kernel<DG_ADSORPTION, 1>; break;
         case 100: fn = (void*)path_kernel<100>; break;
         case 101: fn = (void*)path_kernel<101>; break;
         default: err = "bad algo"; return DG_EINVAL;
@@ -2273,29 +2310,22 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
     // (developer knob)
     if (const char* np = std::getenv("DG_N_PROXY")) P.n_proxy = std::min<int64_t>(P.n_proxy, std::max(0, std::atoi(np)));
     if (!accum) P.n_proxy = 0;
-    // proxies need a flush at least every 2^16 pushes per hub and CTA (px_push):
-    // bound the refresh interval by the largest partition, else no proxies
     {
         const char* e = std::getenv("DG_PROXY_REFRESH");  // developer knob
-        const int want = e ? std::atoi(e) : DG_PROXY_REFRESH;
-        const int64_t allowed = 65535 / std::max<int64_t>(1, D.max_part) - 2 * kWarps;
-        if (allowed < 1) P.n_proxy = 0;
-        P.px_refresh = (want <= 0 || want > allowed) ? (int)std::max<int64_t>(1, allowed) : want;
+        P.px_refresh = e ? std::atoi(e) : DG_PROXY_REFRESH;
     }
     if (accum && P.n_proxy) {
-        // as many proxies as fit acc_minb() CTAs per SM (the top ids are the
-        // highest-degree vertices, so a smaller H' is still the hubs)
-        int dev = 0, sm_bytes = 0, reserved = 0;
+        // as many proxies as fit next to the rings in one CTA per SM (the top
+        // ids are the highest-degree vertices, so a smaller H' is still the hubs)
+        int dev = 0, sm_bytes = 0;
         cudaFuncAttributes fa{};
         CK(cudaGetDevice(&dev));
-        CK(cudaDeviceGetAttribute(&sm_bytes, cudaDevAttrMaxSharedMemoryPerMultiprocessor, dev));
-        CK(cudaDeviceGetAttribute(&reserved, cudaDevAttrReservedSharedMemoryPerBlock, dev));
+        CK(cudaDeviceGetAttribute(&sm_bytes, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev));
         CK(cudaFuncGetAttributes(&fa, fn));
-        const int64_t per_cta = sm_bytes / std::max(1, acc_minb()) - reserved - (int64_t)fa.sharedSizeBytes -
-                                (int64_t)kGbufBytes;
-        P.n_proxy = std::max<int64_t>(0, std::min<int64_t>(P.n_proxy, per_cta / (8 + 4 * kPxLimbs)));
+        const int64_t room = sm_bytes - (int64_t)fa.sharedSizeBytes - (int64_t)gbuf_bytes<kAccWarps>();
+        P.n_proxy = std::max<int64_t>(0, std::min<int64_t>(P.n_proxy, room / kPxBytes));
     }
-    const size_t smem = accum ? kGbufBytes + (size_t)P.n_proxy * (8 + 4 * kPxLimbs) : 0;
+    const size_t smem = accum ? gbuf_bytes<kAccWarps>() + (size_t)P.n_proxy * kPxBytes : 0;
     if (accum) P.e_coef = algo_k == DG_ADSORPTION ? W->e_coef : W->pr_coef;
     {
         const char* dl = std::getenv("DG_DELTA");  // bucket width knob; default: reading R-DELTA
@@ -2338,7 +2368,7 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
         P.trace = trace;
         P.trace_cap = kTraceCap;
     }
-    int rc = coop_launch(W, fn, P, S, err, smem);
+    int rc = coop_launch(W, fn, P, S, err, smem, accum ? kAccWarps * 32 : kBlock);
     if (trace) {
         std::vector<unsigned long long> h(4 * (size_t)kTraceCap);
         cudaMemcpy(h.data(), trace, sizeof(unsigned long long) * h.size(), cudaMemcpyDeviceToHost);
@@ -2656,10 +2686,10 @@ void dev_layout_changed(DevWork* W) {
 }
 
 int dev_set_vertex_params(DevWork*& W, const DevLayout& D, const double* p_inj, const double* p_cont,
-                          const double* inj, std::string& err) {
+                          const double* inj, const float* wsum_h, std::string& err) {
     int rc;
     if ((rc = ensure_work(W, D, err))) return rc;
-    if (!D.w) { err = "Adsorption needs edge weights (load the CSR with weights)"; return DG_EINVAL; }
+    if (!D.e_w) { err = "Adsorption needs the path-edge weights on the device"; return DG_EINVAL; }
     int64_t bytes = 0;
     if (!W->ads_base) {
         if ((rc = dalloc(&W->ads_base, D.n + 1, bytes, err))) return rc;
@@ -2672,8 +2702,8 @@ int dev_set_vertex_params(DevWork*& W, const DevLayout& D, const double* p_inj, 
     if ((rc = dalloc(&wsum, D.n + 1, bytes, err))) { cudaFree(pcont); return rc; }
     rc = h2d(W->ads_base, base.data(), D.n, err);
     if (!rc) rc = h2d(pcont, pc.data(), D.n, err);
+    if (!rc) rc = h2d(wsum, wsum_h, D.n, err);  // W(u), summed on the host at preprocessing
     if (!rc) {
-        wsum_kernel<<<grid_1d(D.n), 256>>>(wsum, D.row_ptr, D.w, D.n);
         cudaMemset(W->e_coef, 0, sizeof(float) * (D.M + kPad));
         ads_coef_kernel<<<grid_1d(D.M), 256>>>(W->e_coef, D.e_idx, D.e_w, pcont, wsum, D.M);
         cudaError_t e = cudaDeviceSynchronize();

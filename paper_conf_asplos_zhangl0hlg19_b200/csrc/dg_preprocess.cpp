@@ -436,7 +436,8 @@ void dependency_dag(const DepGraph& G, DagResult& R, const std::function<void(co
 
 }  // namespace
 
-void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
+void build_layouts(const HostCSR& g, const dg_path_params& p, const std::vector<int>& ranks,
+                   const std::function<void(int, HostLayout&)>& emit) {
     auto t0 = std::chrono::steady_clock::now();
     auto tp = t0;
     const bool verbose = std::getenv("DG_VERBOSE") != nullptr;
@@ -448,7 +449,7 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
         tp = now;
     };
     const int64_t n = g.n, m = g.m;
-    L = HostLayout();
+    HostLayout L;
     L.params = p;
     std::vector<int64_t> deg(n);
     for (int64_t v = 0; v < n; v++) deg[v] = (int64_t)g.indeg[v] + g.outdeg[v];
@@ -786,9 +787,24 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
         std::sort(L.boundary.begin(), L.boundary.end());
     }
 
+    // per-vertex sum of out-edge weights (Adsorption's W(u), reading R-ADS), so
+    // a layout needs no CSR on the device for it
+    L.wsum.assign(n, 0.f);
+    #pragma omp parallel for schedule(dynamic, 4096)
+    for (int64_t u = 0; u < n; u++) {
+        double ws = 0;
+        for (int64_t e = L.prow_ptr[u]; e < L.prow_ptr[u + 1]; e++) ws += g.has_w ? (double)L.pw[e] : 1.0;
+        L.wsum[u] = (float)ws;
+    }
+    L.n_layers = n_layers;
+    L.n_dep_sccs = n_dep_sccs;
+    L.giant = giant;
+
     phase("priority+partitions");
-    // ---- this rank's layout
-    {
+    // ---- each requested rank's layout (the steps above ran once for all)
+    for (const int rank : ranks) {
+        L.params.rank = rank;
+        L.path_off.clear(); L.part_off.clear();
         // this rank's paths (priority order within its partitions) and offsets
         std::vector<int64_t> sel;
         L.part_off.push_back(0);
@@ -823,14 +839,15 @@ void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& L) {
             nh += hot[i];
         }
         L.n_hot = nh;
+        L.built = true;
+        L.preprocess_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+        phase("layout");
+        emit(rank, L);
     }
+}
 
-    phase("layout");
-    L.n_layers = n_layers;
-    L.n_dep_sccs = n_dep_sccs;
-    L.giant = giant;
-    L.built = true;
-    L.preprocess_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+void build_layout(const HostCSR& g, const dg_path_params& p, HostLayout& out) {
+    build_layouts(g, p, {p.rank}, [&](int, HostLayout& L) { out = std::move(L); });
 }
 
 }  // namespace dg

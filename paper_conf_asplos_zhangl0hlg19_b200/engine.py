@@ -74,16 +74,43 @@ class DiGraph:
         """Load an ``inputs.Graph``."""
         return self.load_csr(g.n, g.row_ptr, g.col, g.w)
 
-    def build_paths(self, d_max=16, l_merge=64, n_sub=64, order="degree", hot_factor=2.0,
-                    part_entries=0, rank=0, world=1, merge_rule="relaxed", n_proxy=4096):
+    @staticmethod
+    def _path_params(d_max=16, l_merge=64, n_sub=64, order="degree", hot_factor=2.0,
+                     part_entries=0, rank=0, world=1, merge_rule="relaxed", n_proxy=8192):
         p = default_params()
         p.d_max, p.l_merge, p.n_sub = d_max, l_merge, n_sub
         p.order = 0 if order == "degree" else 1
         p.hot_factor, p.part_entries, p.rank, p.world = hot_factor, part_entries, rank, world
         p.merge_rule = {"paper": 0, "relaxed": 1}[merge_rule]
         p.n_proxy = n_proxy
+        return p
+
+    def build_paths(self, d_max=16, l_merge=64, n_sub=64, order="degree", hot_factor=2.0,
+                    part_entries=0, rank=0, world=1, merge_rule="relaxed", n_proxy=8192):
+        p = self._path_params(d_max, l_merge, n_sub, order, hot_factor, part_entries, rank, world, merge_rule,
+                              n_proxy)
         check(self._L.dg_build_paths(self._h, ctypes.byref(p)), "dg_build_paths")
         self.p2p_key = None  # the library freed any exchange region
+        return self
+
+    def build_paths_shared(self, prefix, world, rank=0, **kw):
+        """dg_build_paths_shared: one preprocessing pass for `world` ranks, rank
+        r's layout written to "<prefix>.<r>"; this handle keeps `rank`'s."""
+        p = self._path_params(rank=rank, world=world, **kw)
+        check(self._L.dg_build_paths_shared(self._h, ctypes.byref(p), prefix.encode()), "dg_build_paths_shared")
+        self.p2p_key = None
+        return self
+
+    def save_layout(self, path):
+        check(self._L.dg_save_layout(self._h, path.encode()), "dg_save_layout")
+        return self
+
+    def load_layout(self, path):
+        """dg_load_layout: this handle's graph and layout from a layout file."""
+        check(self._L.dg_load_layout(self._h, path.encode()), "dg_load_layout")
+        info = self.layout_info()
+        self.n, self.m = info["n"], info["m"]
+        self.p2p_key = None
         return self
 
     def upload(self):

@@ -196,3 +196,62 @@ def test_p2p_exchange_lifecycle_is_checked():
         dg.p2p_open([b"\0" * 64, b"\0" * 64])
     with pytest.raises(DGError, match="DG_EINVAL"):
         dg.boundary_exchange()
+
+
+def test_layout_file_round_trip(tmp_path):
+    """dg_save_layout / dg_load_layout: the loaded handle exports exactly the
+    saved layout (paths, layers, SCC labels, partitions, boundary)."""
+    g = inputs.rmat(11, 2048, 20000, seed=13)
+    a = DiGraph().load_graph(g).build_paths(part_entries=256)
+    path = str(tmp_path / "lay.0")
+    a.save_layout(path)
+    b = DiGraph().load_layout(path)
+    ea, eb = a.export_paths(), b.export_paths()
+    for k in ea:
+        assert np.array_equal(ea[k], eb[k]), k
+    ia, ib = a.layout_info(), b.layout_info()
+    for k in ("n", "m", "n_paths", "n_entries", "n_partitions", "n_hot_paths", "n_layers", "n_dep_sccs",
+              "giant_scc_paths", "n_boundary", "paths_before_merge"):
+        assert ia[k] == ib[k], k
+    assert b.n == g.n and b.m == g.m
+    # a layout file carries no CSR: re-preprocessing it is refused
+    with pytest.raises(DGError, match="DG_EINVAL"):
+        b.build_paths()
+
+
+def test_shared_build_equals_per_rank_builds(tmp_path):
+    """dg_build_paths_shared (one preprocessing pass) writes, for every rank,
+    the layout a per-rank dg_build_paths(rank, world) builds."""
+    g = inputs.rmat(11, 2048, 20000, seed=17)
+    world = 3
+    prefix = str(tmp_path / "shared")
+    own = DiGraph().load_graph(g).build_paths_shared(prefix, world=world, rank=1, part_entries=128)
+    for r in range(world):
+        ref = DiGraph().load_graph(g).build_paths(part_entries=128, rank=r, world=world)
+        got = DiGraph().load_layout(f"{prefix}.{r}")
+        er, eg = ref.export_paths(), got.export_paths()
+        for k in er:
+            assert np.array_equal(er[k], eg[k]), (r, k)
+        assert np.array_equal(ref.boundary_vertices(), got.boundary_vertices())
+    eo, e1 = own.export_paths(), DiGraph().load_layout(f"{prefix}.1").export_paths()
+    for k in eo:
+        assert np.array_equal(eo[k], e1[k]), k
+
+
+def test_bad_layout_file_keeps_the_handle(tmp_path):
+    g = fig4_graph()
+    dg = DiGraph().load_graph(g).build_paths()
+    before = dg.layout_info()
+    p = tmp_path / "bad"
+    p.write_bytes(b"DGLAYOUT" + b"\0" * 16)
+    for path in (str(p), str(tmp_path / "missing")):
+        with pytest.raises(DGError, match="DG_EINVAL"):
+            dg.load_layout(path)
+        assert dg.layout_info() == before
+    good = str(tmp_path / "good")
+    dg.save_layout(good)
+    data = open(good, "rb").read()
+    open(str(p), "wb").write(data[: len(data) // 2])  # truncated
+    with pytest.raises(DGError, match="DG_EINVAL"):
+        dg.load_layout(str(p))
+    assert dg.layout_info() == before
