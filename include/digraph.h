@@ -269,6 +269,24 @@ int dg_boundary_pack(dg_graph *g, void *buf);
  * (an upper bound on the signalled vertices, as for dg_rounds). */
 int dg_boundary_unpack(dg_graph *g, const void *buf, int64_t *active);
 
+/* Multi-rank SCC (DG_SCC in dg_run_begin; the paths of an
+ * SCC-vertex run "over SMXs of multiple GPUs"): the colouring iterations of
+ * the single-rank dg_run(DG_SCC) with every phase a multi-rank run.  The
+ * caller repeats { dg_scc_phase(0): forward min-colour propagation -- then
+ * rounds and exchanges as for MIN algorithms (dg_rounds + dg_boundary_*,
+ * dg_boundary_exchange or dg_run_fused) until the global activity is 0;
+ * dg_scc_phase(1): the roots (vertices keeping their own id) start backward
+ * reachability inside their colour -- rounds and exchanges again (the
+ * replicated state is now the mark, packed as 0 = marked / 1 = not, so the
+ * MIN exchange is an OR); dg_scc_assign: marked vertices take their colour
+ * as label, *remaining = this rank's unassigned vertices } until the sum of
+ * `remaining` over ranks is 0; then dg_run_end.  *active = vertices the phase
+ * signalled on this rank.  dg_get_states then returns this rank's labels; a
+ * vertex on none of its paths carries its own id, so the MIN over ranks is
+ * every vertex's label (smallest vertex id of its SCC). */
+int dg_scc_phase(dg_graph *g, int phase, int64_t *active);
+int dg_scc_assign(dg_graph *g, int64_t *remaining);
+
 /* Finish the run: normalisation (PageRank) and statistics. */
 int dg_run_end(dg_graph *g, dg_run_stats *stats);
 

@@ -25,7 +25,7 @@ EXPORTS = [
     "dg_get_layout_info", "dg_export_paths", "dg_boundary_size", "dg_boundary_vertices",
     "dg_run_begin", "dg_rounds", "dg_boundary_pack", "dg_boundary_unpack", "dg_run_end",
     "dg_normalize_states", "dg_p2p_alloc", "dg_p2p_open", "dg_boundary_exchange", "dg_run_fused",
-    "dg_build_paths_shared", "dg_save_layout", "dg_load_layout",
+    "dg_build_paths_shared", "dg_save_layout", "dg_load_layout", "dg_scc_phase", "dg_scc_assign",
 ]
 
 
@@ -105,6 +105,8 @@ def lib():
         "dg_build_paths_shared": (i32, [P, pp(dg_path_params), ctypes.c_char_p]),
         "dg_save_layout": (i32, [P, ctypes.c_char_p]),
         "dg_load_layout": (i32, [P, ctypes.c_char_p]),
+        "dg_scc_phase": (i32, [P, i32, pp(i64)]),
+        "dg_scc_assign": (i32, [P, pp(i64)]),
     }
     for name, (res, args) in sig.items():
         f = getattr(L, name)

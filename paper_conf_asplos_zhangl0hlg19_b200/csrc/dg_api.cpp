@@ -414,7 +414,6 @@ int dg_boundary_vertices(const dg_graph* g, int32_t* out) {
 int dg_run_begin(dg_graph* g, int algo, int64_t source, double epsilon, double param) {
     int rc = check_run_args(g, algo, source, epsilon, param, DG_MODE_PATH);
     if (rc) return rc;
-    if (algo == DG_SCC) return fail(DG_EINVAL, "dg_run_begin: SCC is single-rank only");
     if ((rc = select_dev(g))) return rc;
     if ((rc = ensure_uploaded(g))) return rc;
     if ((rc = ensure_parts(g, algo, DG_MODE_PATH))) return rc;
@@ -429,6 +428,24 @@ int dg_run_begin(dg_graph* g, int algo, int64_t source, double epsilon, double p
     if (rc) return fail(rc, err);
     g->multi_active = true;
     return DG_OK;
+}
+
+int dg_scc_phase(dg_graph* g, int phase, int64_t* active) {
+    if (!g || !g->multi_active || g->run.algo != DG_SCC || !active || (phase != 0 && phase != 1))
+        return fail(DG_EINVAL, "dg_scc_phase: no multi-rank SCC run in progress, or phase not 0/1");
+    if (int rc0 = select_dev(g)) return rc0;
+    std::string err;
+    int rc = dg::dev_scc_phase(g->work, g->dev, g->run, phase, active, err);
+    return rc ? fail(rc, err) : DG_OK;
+}
+
+int dg_scc_assign(dg_graph* g, int64_t* remaining) {
+    if (!g || !g->multi_active || g->run.algo != DG_SCC || !remaining)
+        return fail(DG_EINVAL, "dg_scc_assign: no multi-rank SCC run in progress");
+    if (int rc0 = select_dev(g)) return rc0;
+    std::string err;
+    int rc = dg::dev_scc_assign(g->work, g->dev, g->run, remaining, err);
+    return rc ? fail(rc, err) : DG_OK;
 }
 
 int dg_rounds(dg_graph* g, int64_t max_rounds, int64_t* active) {

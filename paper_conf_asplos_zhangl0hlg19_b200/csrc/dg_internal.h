@@ -100,6 +100,7 @@ struct RunState {
     int64_t delta = 0;  // SSSP/BFS bucket width (reading R-DELTA), 0 = unbounded
     int64_t round = 0;
     bool raw_states = false;  // multi-rank: per-rank additive contributions, not normalised
+    int scc_phase = -1;       // multi-rank SCC: 0 forward colouring, 1 backward marks, -1 between
     dg_run_stats stats{};
 };
 
@@ -118,6 +119,8 @@ int dev_rounds(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, 
 int dev_boundary_pack(DevWork* W, const DevLayout& D, RunState& S, void* buf, std::string& err);
 int dev_boundary_unpack(DevWork* W, const DevLayout& D, RunState& S, const void* buf, int64_t* active, std::string& err);
 int dev_run_end(DevWork* W, const DevLayout& D, RunState& S, std::string& err);
+int dev_scc_phase(DevWork* W, const DevLayout& D, RunState& S, int phase, int64_t* active, std::string& err);
+int dev_scc_assign(DevWork* W, const DevLayout& D, RunState& S, int64_t* remaining, std::string& err);
 struct P2P;  // peer-memory boundary exchange (dg_kernels.cu)
 int dev_p2p_alloc(P2P*& X, const DevLayout& D, int world, int rank, void* handle, std::string& err);
 int dev_p2p_open(P2P* X, const void* handles, std::string& err);

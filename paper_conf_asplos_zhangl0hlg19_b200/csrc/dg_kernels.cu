@@ -1948,18 +1948,30 @@ __global__ void scc_assign_kernel(const uint32_t* vs, int32_t* label, const uint
 
 // ---- multi-GPU boundary exchange ("each mirror always
 // sends its new state to its master"; line 96: synchronisation in batches)
-__global__ void pack_min_kernel(const uint32_t* vs, const int32_t* bnd, int64_t nb, uint32_t* buf) {
-    GRID_STRIDE(k, nb) buf[k] = vs[bnd[k]];
+// MIN exchanges; with `mark` set (SCC backward phase) the replicated state is
+// the reachability mark, encoded 0 = marked / 1 = not, so MIN is OR.
+__device__ __forceinline__ uint32_t min_value(const uint32_t* vs, const uint8_t* mark, int v) {
+    return mark ? (mark[v] ? 0u : 1u) : vs[v];
 }
-__global__ void unpack_min_kernel(uint32_t* vs, const int32_t* bnd, int64_t nb, const uint32_t* buf, uint32_t* b,
-                                  Counters* ctr, int slot) {
+__device__ __forceinline__ bool min_apply(uint32_t* vs, uint8_t* mark, const int32_t* label, int v, uint32_t m) {
+    if (mark) {
+        if (m != 0u || mark[v] || label[v] >= 0) return false;
+        mark[v] = 1;
+        return true;
+    }
+    if (m >= vs[v]) return false;
+    vs[v] = m;
+    return true;
+}
+__global__ void pack_min_kernel(const uint32_t* vs, const uint8_t* mark, const int32_t* bnd, int64_t nb, uint32_t* buf) {
+    GRID_STRIDE(k, nb) buf[k] = min_value(vs, mark, bnd[k]);
+}
+__global__ void unpack_min_kernel(uint32_t* vs, uint8_t* mark, const int32_t* label, const int32_t* bnd, int64_t nb,
+                                  const uint32_t* buf, uint32_t* b, Counters* ctr, int slot) {
     unsigned cnt = 0;
     GRID_STRIDE(k, nb) {
         const int v = bnd[k];
-        if (buf[k] < vs[v]) {
-            vs[v] = buf[k];
-            cnt += signal_vertex(b, (uint32_t)v);
-        }
+        if (min_apply(vs, mark, label, v, buf[k])) cnt += signal_vertex(b, (uint32_t)v);
     }
     for (int off = 16; off; off >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, off);
     if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(&ctr->active[slot], cnt);
@@ -2007,8 +2019,9 @@ __global__ void unpack_sum_kernel(unsigned long long* vs, unsigned long long* si
 struct PeerSlots {
     const void* p[kP2PMaxRanks];
 };
-__global__ void p2p_pack_min_kernel(const uint32_t* vs, const int32_t* bnd, int64_t nb, unsigned long long* slot) {
-    GRID_STRIDE(k, nb) slot[k] = vs[bnd[k]];
+__global__ void p2p_pack_min_kernel(const uint32_t* vs, const uint8_t* mark, const int32_t* bnd, int64_t nb,
+                                    unsigned long long* slot) {
+    GRID_STRIDE(k, nb) slot[k] = min_value(vs, mark, bnd[k]);
 }
 __global__ void p2p_pack_sum_kernel(const unsigned long long* vs, const int32_t* bnd, int64_t nb,
                                     const unsigned long long* base, unsigned long long* slot) {
@@ -2038,17 +2051,14 @@ __global__ void p2p_signal_wait_kernel(PeerSlots flags, int world, int rank, uns
         }
     }
 }
-__global__ void p2p_reduce_min_kernel(PeerSlots slots, int world, uint32_t* vs, const int32_t* bnd, int64_t nb,
-                                      uint32_t* b, Counters* ctr, int slot) {
+__global__ void p2p_reduce_min_kernel(PeerSlots slots, int world, uint32_t* vs, uint8_t* mark, const int32_t* label,
+                                      const int32_t* bnd, int64_t nb, uint32_t* b, Counters* ctr, int slot) {
     unsigned cnt = 0;
     GRID_STRIDE(k, nb) {
         unsigned long long m = ~0ull;
         for (int r = 0; r < world; r++) m = min(m, __ldcv((const unsigned long long*)slots.p[r] + k));
         const int v = bnd[k];
-        if ((uint32_t)m < vs[v]) {
-            vs[v] = (uint32_t)m;
-            cnt += signal_vertex(b, (uint32_t)v);
-        }
+        if (min_apply(vs, mark, label, v, (uint32_t)m)) cnt += signal_vertex(b, (uint32_t)v);
     }
     for (int off = 16; off; off >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, off);
     if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(&ctr->active[slot], cnt);
@@ -2292,6 +2302,8 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
             case DG_WCC: fn = (void*)path_kernel<DG_WCC, DG_PATH_MINB, true>; break;
             case DG_PAGERANK: fn = (void*)path_kernel<DG_PAGERANK, 1, true>; break;
             case DG_ADSORPTION: fn = (void*)path_kernel<DG_ADSORPTION, 1, true>; break;
+            case 100: fn = (void*)path_kernel<100, DG_PATH_MINB, true>; break;
+            case 101: fn = (void*)path_kernel<101, DG_PATH_MINB, true>; break;
             default: err = "fused multi-rank run: bad algo"; return DG_EINVAL;
         }
     } else switch (algo_k) {
@@ -2749,7 +2761,116 @@ int dev_run(DevWork*& W, const DevLayout& D, RunState& S, int64_t max_rounds, st
     return DG_OK;
 }
 
+// ---- multi-rank SCC (dg_run_begin(DG_SCC) / dg_scc_phase / dg_scc_assign):
+// the colouring iterations of run_scc with every phase a multi-rank run --
+// forward colouring exchanges colours with MIN, backward reachability
+// exchanges marks (MIN of 0 = marked / 1 = not, i.e. OR).  A vertex on none
+// of this rank's paths is assigned its own original id at the start: the
+// owning ranks' labels are <= it, so a MIN over ranks gives every vertex its
+// SCC label, and a vertex on no rank's paths (no edges) is its own SCC.
+namespace {
+__global__ void scc_present_kernel(const uint32_t* e_idx, int64_t M, uint8_t* mark) {
+    GRID_STRIDE(i, M) mark[e_idx[i] & kVMask] = 1;
+}
+__global__ void scc_label_init_kernel(int32_t* label, uint8_t* mark, const int32_t* orig, int64_t n) {
+    GRID_STRIDE(v, n) {
+        label[v] = mark[v] ? -1 : orig[v];
+        mark[v] = 0;
+    }
+}
+__global__ void scc_count_kernel(const int32_t* label, int64_t n, int32_t* remaining) {
+    int cnt = 0;
+    GRID_STRIDE(v, n) cnt += label[v] < 0;
+    for (int off = 16; off; off >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, off);
+    if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(remaining, cnt);
+}
+// the device counters of the phase that just ran, added to the run's statistics
+int fold_counters(DevWork* W, RunState& S, std::string& err) {
+    Counters c;
+    int rc;
+    if ((rc = read_counters(W, c, err))) return rc;
+    S.stats.rounds += c.round;
+    S.stats.vertex_updates += (int64_t)c.updates;
+    S.stats.edges_processed += (int64_t)c.edges;
+    S.stats.units_processed += (int64_t)c.units;
+    S.stats.entries_processed += (int64_t)c.entries;
+    S.stats.dense_rounds += (int64_t)c.dense_rounds;
+    return write_counters(W, Counters{}, err);
+}
+}  // namespace
+
+// the kernel algorithm of a run (SCC phases: 100 forward colouring, 101 backward marks)
+int launch_algo(const RunState& S) { return S.algo == DG_SCC ? (S.scc_phase == 1 ? 101 : 100) : S.algo; }
+// the replicated mark array of an SCC backward phase (else null: MIN over vs_u)
+uint8_t* scc_marks(DevWork* W, const RunState& S) { return S.algo == DG_SCC && S.scc_phase == 1 ? W->scc_mark : nullptr; }
+
+int dev_scc_begin(DevWork*& W, const DevLayout& D, RunState& S, std::string& err) {
+    int rc;
+    if ((rc = ensure_work(W, D, err))) return rc;
+    int64_t bytes = 0;
+    if (!W->scc_label) {
+        if ((rc = dalloc(&W->scc_label, D.n + 1, bytes, err))) return rc;
+        if ((rc = dalloc(&W->scc_mark, D.n + 1, bytes, err))) return rc;
+        if ((rc = dalloc(&W->remaining, 1, bytes, err))) return rc;
+    }
+    CK(cudaMemset(W->scc_mark, 0, D.n + 1));
+    if (D.M) scc_present_kernel<<<grid_1d(D.M), 256>>>(D.e_idx, D.M, W->scc_mark);
+    scc_label_init_kernel<<<grid_1d(D.n), 256>>>(W->scc_label, W->scc_mark, D.orig, D.n);
+    CK(cudaGetLastError());
+    S.scc_phase = -1;
+    S.stats.kernel_launches += 2;
+    if ((rc = write_counters(W, Counters{}, err))) return rc;
+    CK(cudaEventRecord(W->ev0));
+    return DG_OK;
+}
+
+int dev_scc_phase(DevWork* W, const DevLayout& D, RunState& S, int phase, int64_t* active, std::string& err) {
+    if (!W || !W->scc_label) { err = "dg_scc_phase: no SCC run in progress"; return DG_EINVAL; }
+    int rc;
+    if ((rc = fold_counters(W, S, err))) return rc;
+    CK(cudaMemsetAsync(W->bits, 0, sizeof(uint32_t) * 2 * W->nw));
+    const int g = grid_1d(D.n);
+    Counters c{};
+    if (phase == 0) {  // forward colouring: unassigned vertices start with their own id, all signalled
+        scc_init_kernel<<<g, 256>>>(W->vs_u, W->scc_label, D.orig, W->scc_mark, D.n);
+        scc_bits_kernel<<<grid_1d(W->nw), 256>>>(W->scc_label, D.n, W->bits, W->nw);
+        CK(cudaMemset(W->remaining, 0, sizeof(int32_t)));
+        scc_count_kernel<<<g, 256>>>(W->scc_label, D.n, W->remaining);
+        int32_t rem = 0;
+        CK(cudaMemcpy(&rem, W->remaining, sizeof(int32_t), cudaMemcpyDeviceToHost));
+        c.active[0] = (unsigned)rem;
+        if ((rc = write_counters(W, c, err))) return rc;
+        *active = rem;
+        S.stats.kernel_launches += 3;
+    } else {  // backward reachability from the roots (vertices keeping their own id)
+        scc_roots_kernel<<<g, 256>>>(W->vs_u, W->scc_label, D.orig, W->scc_mark, D.n, W->bits, W->ctr);
+        S.stats.kernel_launches += 1;
+        if ((rc = read_counters(W, c, err))) return rc;
+        *active = c.active[0];
+    }
+    CK(cudaGetLastError());
+    S.scc_phase = phase;
+    S.round = 0;
+    return DG_OK;
+}
+
+int dev_scc_assign(DevWork* W, const DevLayout& D, RunState& S, int64_t* remaining, std::string& err) {
+    if (!W || !W->scc_label || S.scc_phase != 1) { err = "dg_scc_assign: after a backward phase only"; return DG_EINVAL; }
+    int rc;
+    if ((rc = fold_counters(W, S, err))) return rc;
+    CK(cudaMemset(W->remaining, 0, sizeof(int32_t)));
+    scc_assign_kernel<<<grid_1d(D.n), 256>>>(W->vs_u, W->scc_label, W->scc_mark, D.n, W->remaining);
+    int32_t rem = 0;
+    CK(cudaMemcpy(&rem, W->remaining, sizeof(int32_t), cudaMemcpyDeviceToHost));
+    *remaining = rem;
+    S.stats.kernel_launches += 1;
+    S.stats.outer_iterations++;
+    S.scc_phase = -1;
+    return DG_OK;
+}
+
 int dev_run_begin(DevWork*& W, const DevLayout& D, RunState& S, std::string& err) {
+    if (S.algo == DG_SCC) return dev_scc_begin(W, D, S, err);
     int rc;
     if ((rc = ensure_work(W, D, err))) return rc;
     if (S.algo == DG_ADSORPTION && !W->have_params) { err = "Adsorption needs dg_set_vertex_params first"; return DG_EINVAL; }
@@ -2763,7 +2884,8 @@ int dev_run_begin(DevWork*& W, const DevLayout& D, RunState& S, std::string& err
 
 int dev_rounds(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, int64_t* active, std::string& err) {
     int rc;
-    if ((rc = launch_path(W, D, S.algo, (int)std::min<int64_t>(max_rounds, 1 << 30), S, err))) return rc;
+    if (S.algo == DG_SCC && S.scc_phase < 0) { err = "dg_rounds: SCC run without a phase (dg_scc_phase)"; return DG_EINVAL; }
+    if ((rc = launch_path(W, D, launch_algo(S), (int)std::min<int64_t>(max_rounds, 1 << 30), S, err))) return rc;
     Counters c;
     if ((rc = read_counters(W, c, err))) return rc;
     *active = c.active[c.round & 1];
@@ -2775,7 +2897,7 @@ int dev_boundary_pack(DevWork* W, const DevLayout& D, RunState& S, void* buf, st
     if (S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION)
         pack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_t, D.bnd, D.n_bnd, W->bnd_base, (unsigned long long*)buf);
     else
-        pack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, D.bnd, D.n_bnd, (uint32_t*)buf);
+        pack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, scc_marks(W, S), D.bnd, D.n_bnd, (uint32_t*)buf);
     S.stats.kernel_launches++;
     CK(cudaGetLastError());
     CK(cudaDeviceSynchronize());
@@ -2796,8 +2918,8 @@ int dev_boundary_unpack(DevWork* W, const DevLayout& D, RunState& S, const void*
                                                          (unsigned long long)(S.eps * 4294967296.0), b, W->ctr,
                                                          slot);
         else
-            unpack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, D.bnd, D.n_bnd, (const uint32_t*)buf, b, W->ctr,
-                                                         slot);
+            unpack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, scc_marks(W, S), W->scc_label, D.bnd, D.n_bnd,
+                                                         (const uint32_t*)buf, b, W->ctr, slot);
         S.stats.kernel_launches++;
         CK(cudaGetLastError());
     }
@@ -2879,7 +3001,7 @@ int dev_boundary_exchange(DevWork* W, const DevLayout& D, RunState& S, P2P* X, i
     unsigned long long* mine = (unsigned long long*)(X->own + off);
     if (D.n_bnd) {
         if (sum) p2p_pack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_t, D.bnd, D.n_bnd, W->bnd_base, mine);
-        else p2p_pack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, D.bnd, D.n_bnd, mine);
+        else p2p_pack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, scc_marks(W, S), D.bnd, D.n_bnd, mine);
     }
     unsigned long long* own_flags = (unsigned long long*)X->own;
     p2p_signal_wait_kernel<<<1, 32>>>(flags, X->world, X->rank, e, own_flags, 60ull * 1000000000ull);
@@ -2890,8 +3012,8 @@ int dev_boundary_exchange(DevWork* W, const DevLayout& D, RunState& S, P2P* X, i
                                                              W->bnd_base, (unsigned long long)(S.eps * 4294967296.0),
                                                              b, W->ctr, slot);
         else
-            p2p_reduce_min_kernel<<<grid_1d(D.n_bnd), 256>>>(slots, X->world, W->vs_u, D.bnd, D.n_bnd, b, W->ctr,
-                                                             slot);
+            p2p_reduce_min_kernel<<<grid_1d(D.n_bnd), 256>>>(slots, X->world, W->vs_u, scc_marks(W, S), W->scc_label,
+                                                             D.bnd, D.n_bnd, b, W->ctr, slot);
     }
     S.stats.kernel_launches += D.n_bnd ? 3 : 1;
     CK(cudaGetLastError());
@@ -2910,11 +3032,7 @@ int dev_run_fused(DevWork* W, const DevLayout& D, RunState& S, P2P* X, int64_t l
                   int64_t* exchanges, int64_t* converged, std::string& err) {
     if (!X || !X->opened) { err = "dg_run_fused: peers not opened (dg_p2p_open)"; return DG_EINVAL; }
     if (X->nb != D.n_bnd) { err = "dg_run_fused: layout changed since dg_p2p_alloc"; return DG_EINVAL; }
-    if (S.algo != DG_SSSP && S.algo != DG_BFS && S.algo != DG_WCC && S.algo != DG_PAGERANK &&
-        S.algo != DG_ADSORPTION) {
-        err = "dg_run_fused: SSSP, BFS, WCC, PageRank or Adsorption";
-        return DG_EINVAL;
-    }
+    if (S.algo == DG_SCC && S.scc_phase < 0) { err = "dg_run_fused: SCC run without a phase (dg_scc_phase)"; return DG_EINVAL; }
     const size_t nbs = (size_t)std::max<int64_t>(D.n_bnd, 1);
     if (!X->last) CK(cudaMalloc(&X->last, sizeof(uint32_t) * nbs));
     CK(cudaMemset(X->last, 0xFF, sizeof(uint32_t) * nbs));  // differs from every state: the first exchange is dirty
@@ -2933,8 +3051,9 @@ int dev_run_fused(DevWork* W, const DevLayout& D, RunState& S, P2P* X, int64_t l
     M.rank = X->rank;
     M.every = (int)std::max<int64_t>(1, local_rounds);
     M.sum = S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION;
+    M.mark = scc_marks(W, S) != nullptr;
     int rc;
-    if ((rc = launch_path(W, D, S.algo, (int)std::min<int64_t>(max_rounds, 1 << 30), S, err, &M))) return rc;
+    if ((rc = launch_path(W, D, launch_algo(S), (int)std::min<int64_t>(max_rounds, 1 << 30), S, err, &M))) return rc;
     Counters c;
     if ((rc = read_counters(W, c, err))) return rc;
     X->epoch += c.mr_ex;
@@ -2950,7 +3069,7 @@ int dev_run_end(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
     float ms = 0;
     CK(cudaEventElapsedTime(&ms, W->ev0, W->ev1));
     int rc;
-    if ((rc = collect_stats(W, S, err))) return rc;
+    if ((rc = S.algo == DG_SCC ? fold_counters(W, S, err) : collect_stats(W, S, err))) return rc;
     S.stats.time_ms = ms;
     return DG_OK;
 }

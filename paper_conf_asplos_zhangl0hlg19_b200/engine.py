@@ -219,6 +219,19 @@ class DiGraph:
         check(self._L.dg_boundary_exchange(self._h, ctypes.byref(a)), "dg_boundary_exchange")
         return a.value
 
+    def scc_phase(self, phase):
+        """dg_scc_phase: 0 forward colouring, 1 backward marks; returns the
+        vertices this rank signalled."""
+        a = ctypes.c_int64()
+        check(self._L.dg_scc_phase(self._h, int(phase), ctypes.byref(a)), "dg_scc_phase")
+        return a.value
+
+    def scc_assign(self):
+        """dg_scc_assign: returns this rank's unassigned vertices."""
+        a = ctypes.c_int64()
+        check(self._L.dg_scc_assign(self._h, ctypes.byref(a)), "dg_scc_assign")
+        return a.value
+
     def run_fused(self, local_rounds=4, max_rounds=0):
         """The whole multi-rank run in one launch (dg_run_fused); returns
         (exchanges, converged)."""

@@ -33,7 +33,7 @@ import torch
 import torch.distributed as dist
 
 SUM_ALGOS = ("pagerank", "adsorption")
-MIN_ALGOS = ("sssp", "bfs", "wcc")
+MIN_ALGOS = ("sssp", "bfs", "wcc", "scc")  # SCC phases exchange colours / marks with MIN
 
 
 def boundary_buffer(n_boundary, algo, device):
@@ -75,12 +75,41 @@ def p2p_setup(engine, group=None, device=None):
     return first
 
 
+def _converge(engine, exchange, nb, buf, op, local_rounds, max_outer, group, device):
+    """One multi-rank run (or SCC phase) to global convergence; returns the
+    number of boundary exchanges."""
+    if exchange == "fused":
+        syncs, converged = engine.run_fused(local_rounds)
+        if not converged:
+            raise RuntimeError("multi-rank run did not converge")
+        return syncs
+    active = torch.zeros(1, dtype=torch.int64, device=device)
+    for syncs in range(1, max_outer + 1):
+        engine.rounds(local_rounds)
+        if exchange == "p2p":
+            act = engine.boundary_exchange()
+        else:
+            if nb:
+                engine.boundary_pack(buf)
+            dist.all_reduce(buf, op=op, group=group)
+            act = engine.boundary_unpack(buf)
+        active.fill_(int(act))
+        dist.all_reduce(active, op=dist.ReduceOp.SUM, group=group)
+        if int(active.item()) == 0:
+            return syncs
+    raise RuntimeError("multi-rank run did not converge")
+
+
 def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_rounds=4,
                     max_outer=1_000_000, device=None, group=None, exchange=None):
     """Run ``algo`` to global convergence.  Returns (stats, sync_info).
-    ``exchange``: "fused" (default on CUDA devices), "p2p" or "collective"."""
+    ``exchange``: "fused" (default on CUDA devices), "p2p" or "collective".
+    SCC runs its colouring iterations (include/digraph.h dg_scc_phase): per
+    iteration a forward-colouring phase and a backward-marking phase, each a
+    multi-rank run with MIN exchanges, then dg_scc_assign; the iterations stop
+    when no rank has an unassigned vertex."""
     if algo not in SUM_ALGOS + MIN_ALGOS:
-        raise ValueError(f"{algo}: no multi-rank protocol (SCC is single-rank)")
+        raise ValueError(f"{algo}: no multi-rank protocol")
     device = device if device is not None else (torch.device("cuda", torch.cuda.current_device())
                                                 if torch.cuda.is_available() else torch.device("cpu"))
     if exchange is None:
@@ -90,7 +119,6 @@ def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_ro
     nb = len(engine.boundary_vertices())
     buf = boundary_buffer(nb, algo, device)
     op = dist.ReduceOp.SUM if algo in SUM_ALGOS else dist.ReduceOp.MIN
-    active = torch.zeros(1, dtype=torch.int64, device=device)
     engine.run_begin(algo, source=source, epsilon=epsilon, damping=damping)
     p2p_error = None
     if exchange in ("fused", "p2p"):
@@ -100,33 +128,28 @@ def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_ro
             print(f"[parallel] peer-memory exchange unavailable ({p2p_error}); using the collective",
                   file=sys.stderr, flush=True)
             exchange = "collective"
-    syncs, bytes_per_sync = 0, buf.numel() * buf.element_size()
-    if exchange == "fused":
-        syncs, converged = engine.run_fused(local_rounds)
-        if not converged:
-            raise RuntimeError("multi-rank run did not converge")
-        max_outer = 0
-    for _ in range(max_outer):
-        engine.rounds(local_rounds)
-        if exchange == "p2p":
-            act = engine.boundary_exchange()
-        else:
-            if nb:
-                engine.boundary_pack(buf)
-            dist.all_reduce(buf, op=op, group=group)
-            act = engine.boundary_unpack(buf)
-        syncs += 1
-        active.fill_(int(act))
-        dist.all_reduce(active, op=dist.ReduceOp.SUM, group=group)
-        if int(active.item()) == 0:
-            break
+    args = (exchange, nb, buf, op, local_rounds, max_outer, group, device)
+    syncs, iterations = 0, 0
+    if algo == "scc":
+        rem = torch.zeros(1, dtype=torch.int64, device=device)
+        while True:
+            for phase in (0, 1):
+                engine.scc_phase(phase)
+                syncs += _converge(engine, *args)
+            rem.fill_(int(engine.scc_assign()))
+            dist.all_reduce(rem, op=dist.ReduceOp.SUM, group=group)
+            iterations += 1
+            if int(rem.item()) == 0:
+                break
     else:
-        if exchange != "fused":
-            raise RuntimeError("multi-rank run did not converge")
+        syncs = _converge(engine, *args)
     stats = engine.run_end()
+    bytes_per_sync = buf.numel() * buf.element_size()
     if exchange in ("fused", "p2p"):  # every rank reads each peer's 8-byte slot per boundary vertex
         bytes_per_sync = 8 * nb * (dist.get_world_size(group) - 1)
     info = {"syncs": syncs, "boundary": nb, "nvlink_bytes_per_sync": bytes_per_sync, "exchange": exchange}
+    if algo == "scc":
+        info["scc_iterations"] = iterations
     if p2p_error:
         info["p2p_error"] = p2p_error
     return stats, info

@@ -53,7 +53,7 @@ def _worker(rank, world, port, algo, q, sparse=False, exchange="fused"):
 
 @pytest.mark.parametrize("exchange", ["fused", "p2p", "collective"])
 @pytest.mark.parametrize("sparse", [False, True])
-@pytest.mark.parametrize("algo", ["sssp", "wcc", "pagerank", "adsorption"])
+@pytest.mark.parametrize("algo", ["sssp", "wcc", "pagerank", "adsorption", "scc"])
 def test_two_ranks_on_one_gpu_match_oracle(algo, sparse, exchange, cuda_required):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -74,6 +74,10 @@ def test_two_ranks_on_one_gpu_match_oracle(algo, sparse, exchange, cuda_required
     elif algo == "wcc":
         exp, _ = OA.wcc_label_propagation(g.n, src, dst)
         assert np.array_equal(got.astype(np.int64), exp)
+    elif algo == "scc":
+        exp = OA.scc_tarjan(g.n, src, dst)
+        assert np.array_equal(got.astype(np.int64), exp)
+        assert info["scc_iterations"] >= 1
     elif algo == "adsorption":
         p_inj, p_cont, inj = inputs.adsorption_params(g.n, seed=3)
         exp, _ = OA.adsorption_jacobi(g.n, src, dst, w, p_inj, p_cont, inj, tol=1e-12)

@@ -58,6 +58,16 @@ class CpuPathEngine:
 
     def run_begin(self, algo, source=0, epsilon=1e-7, damping=0.85):
         self.algo = algo
+        if algo == "scc":
+            # vertices on none of this rank's paths carry their own id (MIN-gathered)
+            present = np.zeros(self.n, bool)
+            for p in self.paths:
+                present[p] = True
+            self.label = np.where(present, -1, np.arange(self.n)).astype(np.int64)
+            self.x = np.full(self.n, OA.UNREACHED, np.int64)
+            self.mark = np.zeros(self.n, bool)
+            self.phase = -1
+            return
         if algo in ("sssp", "wcc"):
             self.x = np.full(self.n, OA.UNREACHED, np.int64)
             if algo == "sssp":
@@ -126,14 +136,57 @@ class CpuPathEngine:
                     carry = 0.0
         return pushed
 
+    # ---- SCC colouring phases (include/digraph.h dg_scc_phase / dg_scc_assign)
+    def scc_phase(self, phase):
+        self.phase = phase
+        un = self.label < 0
+        if phase == 0:
+            self.x = np.where(un, np.arange(self.n), OA.UNREACHED).astype(np.int64)
+            self.mark[:] = False
+            return int(un.sum())
+        self.mark = un & (self.x == np.arange(self.n))
+        return int(self.mark.sum())
+
+    def scc_assign(self):
+        sel = self.mark & (self.label < 0)
+        self.label[sel] = self.x[sel]
+        self.phase = -1
+        return int((self.label < 0).sum())
+
+    def _walk_scc(self):
+        changed = 0
+        for p in self.paths:
+            vs = p.tolist()
+            if self.phase == 0:  # forward min colour; assigned vertices break the path
+                cur = None
+                for v in vs:
+                    if self.label[v] >= 0:
+                        cur = None
+                        continue
+                    if cur is not None and cur < self.x[v]:
+                        self.x[v] = cur
+                        changed += 1
+                    cur = self.x[v]
+            else:  # backward marks inside a colour
+                for a, b in zip(vs[-2::-1], vs[:0:-1]):
+                    if (self.mark[b] and not self.mark[a] and self.label[a] < 0 and self.label[b] < 0
+                            and self.x[a] == self.x[b]):
+                        self.mark[a] = True
+                        changed += 1
+        return changed
+
     def rounds(self, k):
+        walk = (self._walk_scc if self.algo == "scc" else
+                self._walk_min if self.algo in ("sssp", "wcc") else self._walk_accum)
         for _ in range(100000):
-            if (self._walk_min() if self.algo in ("sssp", "wcc") else self._walk_accum()) == 0:
+            if walk() == 0:
                 return 0
         raise RuntimeError("local rounds did not converge")
 
     def boundary_pack(self, buf):
-        if self.algo in ("sssp", "wcc"):
+        if self.algo == "scc" and self.phase == 1:  # marks: 0 = marked, MIN = OR
+            buf.copy_(torch.from_numpy(np.where(self.mark[self.bnd], 0, 1).astype(np.int32)))
+        elif self.algo in ("sssp", "wcc", "scc"):
             buf.copy_(torch.from_numpy(self.x[self.bnd].astype(np.int32)))
         else:
             buf.copy_(torch.from_numpy(self.T[self.bnd] - self.base))
@@ -142,7 +195,11 @@ class CpuPathEngine:
         if len(self.bnd) == 0:
             return 0
         b = buf.numpy().astype(np.int64)
-        if self.algo in ("sssp", "wcc"):
+        if self.algo == "scc" and self.phase == 1:
+            new = (b == 0) & ~self.mark[self.bnd] & (self.label[self.bnd] < 0)
+            self.mark[self.bnd[new]] = True
+            return int(new.sum())
+        if self.algo in ("sssp", "wcc", "scc"):
             new = np.minimum(self.x[self.bnd], b)
             act = int((new < self.x[self.bnd]).sum())
             self.x[self.bnd] = new
@@ -157,7 +214,9 @@ class CpuPathEngine:
         return {}
 
     def get_states(self, out):
-        if self.algo in ("sssp", "wcc"):
+        if self.algo == "scc":
+            out.copy_(torch.from_numpy(self.label.astype(np.int32)))
+        elif self.algo in ("sssp", "wcc"):
             out.copy_(torch.from_numpy(self.x.astype(np.int32)))
         else:
             out.copy_(torch.from_numpy((self.T / FX).astype(np.float32)))
@@ -205,7 +264,7 @@ class FusedModelEngine(CpuPathEngine):
 
     def run_fused(self, local_rounds=4, max_rounds=0):
         nb = len(self.bnd)
-        minalgo = self.algo in ("sssp", "wcc")
+        minalgo = self.algo in ("sssp", "wcc", "scc")
         last = None
         for ex in range(1, 100000):
             act = self.rounds(local_rounds)
@@ -245,7 +304,8 @@ def _worker(rank, world, port, algo, q, exchange=None):
 
 @pytest.mark.parametrize("algo,exchange", [("sssp", None), ("wcc", None), ("pagerank", None), ("adsorption", None),
                                            ("sssp", "p2p"), ("sssp", "fused"), ("wcc", "fused"),
-                                           ("pagerank", "fused"), ("adsorption", "fused")])
+                                           ("pagerank", "fused"), ("adsorption", "fused"), ("scc", None),
+                                           ("scc", "fused")])
 def test_two_rank_protocol_matches_oracle(algo, exchange):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
@@ -268,6 +328,10 @@ def test_two_rank_protocol_matches_oracle(algo, exchange):
     elif algo == "wcc":
         exp, _ = OA.wcc_label_propagation(g.n, src, dst)
         assert np.array_equal(got.astype(np.int64), exp)
+    elif algo == "scc":
+        exp = OA.scc_tarjan(g.n, src, dst)
+        assert np.array_equal(got.astype(np.int64), exp)
+        assert info["scc_iterations"] >= 1
     elif algo == "adsorption":
         p_inj, p_cont, inj = inputs.adsorption_params(g.n, seed=3)
         exp, _ = OA.adsorption_jacobi(g.n, src, dst, w, p_inj, p_cont, inj, tol=1e-12)
