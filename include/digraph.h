@@ -75,11 +75,16 @@ typedef struct {
                               l_merge; reading R-MERGE) */
     int32_t n_proxy;       /* highest-degree vertices kept as shared-memory proxies by the
                               PageRank/Adsorption walk; 0 = none */
+    int32_t placement;     /* world > 1: partition -> rank placement; 0: round-robin over the
+                              priority order; 1: locality (each partition to the rank already
+                              holding most of its vertices, entry loads within 2 %; PAPER.md
+                              line 178; reading R-PLACE) */
 } dg_path_params;
 
 /* Fill *p with the defaults (d_max 16, l_merge 64, n_sub 64, order 0,
  * hot_factor 2, part_entries 0 (auto), rank 0, world 1, merge_rule 1,
- * n_proxy 8192; the kernel uses as many as fit its shared memory). */
+ * n_proxy 8192 (the kernel uses as many as fit its shared memory),
+ * placement 1). */
 void dg_default_params(dg_path_params *p);
 
 /* Statistics of one dg_run (device-side counters). */

@@ -33,7 +33,7 @@ class dg_path_params(ctypes.Structure):
     _fields_ = [("d_max", ctypes.c_int32), ("l_merge", ctypes.c_int32), ("n_sub", ctypes.c_int32),
                 ("order", ctypes.c_int32), ("hot_factor", ctypes.c_float),
                 ("part_entries", ctypes.c_int32), ("rank", ctypes.c_int32), ("world", ctypes.c_int32),
-                ("merge_rule", ctypes.c_int32), ("n_proxy", ctypes.c_int32)]
+                ("merge_rule", ctypes.c_int32), ("n_proxy", ctypes.c_int32), ("placement", ctypes.c_int32)]
 
 
 class dg_run_stats(ctypes.Structure):

@@ -51,6 +51,7 @@ void dg_default_params(dg_path_params* p) {
     p->world = 1;
     p->merge_rule = 1;
     p->n_proxy = 8192;
+    p->placement = 1;
 }
 
 int dg_create(dg_graph** out, int device) {
@@ -120,7 +121,7 @@ int dg_load_csr(dg_graph* g, int64_t n, int64_t m, const int64_t* row_ptr, const
 static int check_params(const dg_path_params& q) {
     if (q.d_max < 1 || q.n_sub < 1 || q.part_entries < 0 || q.world < 1 || q.world > 64 ||
         q.rank < 0 || q.rank >= q.world || q.l_merge < 0 || q.merge_rule < 0 || q.merge_rule > 1 ||
-        q.n_proxy < 0 || q.n_proxy > 16384)
+        q.n_proxy < 0 || q.n_proxy > 16384 || q.placement < 0 || q.placement > 1)
         return fail(DG_EINVAL, "dg_build_paths: bad parameters");
     return DG_OK;
 }

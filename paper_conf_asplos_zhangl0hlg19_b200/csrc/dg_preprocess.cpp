@@ -721,18 +721,73 @@ void build_layouts(const HostCSR& g, const dg_path_params& p, const std::vector<
         for (int64_t i = 0; i < P; i++) tot += nvert[i];
         target = std::min<int64_t>(2048, std::max<int64_t>(128, tot / 16384));
     }
-    std::vector<int64_t> gpart_first{0};  // global partition -> first index in `order`
-    {
-        int64_t acc = 0;
+    const int world = std::max(1, p.world), rank = p.rank;
+    // ---- path -> rank placement (world > 1, placement 1; reading R-PLACE,
+    // a dispatch unit goes to "the GPU with the most number
+    // of its direct precursors"): paths in priority order, each to the rank
+    // already holding most of its vertices among the ranks whose entry load
+    // stays within 2 % of an even share (ties: the least loaded) -- a greedy
+    // vertex-cut that keeps replicas (the boundary) few.  The order is then
+    // regrouped rank by rank (priority order inside a rank) so a partition
+    // never spans two ranks.  placement 0: partitions round-robin (below).
+    std::vector<int32_t> grp_owner;  // owner rank of each group of `order` (placement 1)
+    std::vector<int64_t> grp_first{0, P};
+    if (world > 1 && p.placement == 1) {
+        int64_t tot = 0;
+        for (int64_t i = 0; i < P; i++) tot += nvert[i];
+        const double cap = 1.02 * (double)tot / world;
+        std::vector<uint64_t> pres(n, 0);
+        std::vector<int64_t> load(world, 0), cnt(world);
+        std::vector<int32_t> path_owner(P);
         for (int64_t r = 0; r < P; r++) {
-            if (acc >= target) { gpart_first.push_back(r); acc = 0; }
+            const int64_t i = order[r];
+            std::fill(cnt.begin(), cnt.end(), 0);
+            for (int64_t k = moff[i]; k < moff[i + 1]; k++)
+                for (uint64_t b = pres[mv[k]]; b; b &= b - 1) cnt[__builtin_ctzll(b)]++;
+            int best = -1;
+            for (int w = 0; w < world; w++) {
+                if ((double)(load[w] + nvert[i]) > cap) continue;
+                if (best < 0 || cnt[w] > cnt[best] || (cnt[w] == cnt[best] && load[w] < load[best])) best = w;
+            }
+            if (best < 0) best = (int)(std::min_element(load.begin(), load.end()) - load.begin());
+            path_owner[i] = best;
+            load[best] += nvert[i];
+            const uint64_t bit = 1ull << best;
+            for (int64_t k = moff[i]; k < moff[i + 1]; k++) pres[mv[k]] |= bit;
+        }
+        std::vector<int64_t> grouped;
+        grouped.reserve(P);
+        grp_first.assign(1, 0);
+        for (int w = 0; w < world; w++) {
+            for (int64_t r = 0; r < P; r++)
+                if (path_owner[order[r]] == w) grouped.push_back(order[r]);
+            grp_first.push_back((int64_t)grouped.size());
+            grp_owner.push_back(w);
+        }
+        order.swap(grouped);
+    }
+    // ---- partitions over the (grouped) priority order (greedy, whole paths)
+    std::vector<int64_t> gpart_first{0};  // global partition -> first index in `order`
+    std::vector<int32_t> owner;           // global partition -> rank
+    for (size_t grp = 0; grp + 1 < grp_first.size(); grp++) {
+        int64_t acc = 0;
+        for (int64_t r = grp_first[grp]; r < grp_first[grp + 1]; r++) {
+            if (acc >= target && r > gpart_first.back()) {
+                gpart_first.push_back(r);
+                owner.push_back(grp_owner.empty() ? 0 : grp_owner[grp]);
+                acc = 0;
+            }
             acc += nvert[order[r]];
         }
-        gpart_first.push_back(P);
-        if (P == 0) gpart_first.assign(1, 0);
+        if (grp_first[grp + 1] > gpart_first.back()) {
+            gpart_first.push_back(grp_first[grp + 1]);
+            owner.push_back(grp_owner.empty() ? 0 : grp_owner[grp]);
+        }
     }
+    if (P == 0) { gpart_first.assign(1, 0); owner.clear(); }
     const int64_t G = (int64_t)gpart_first.size() - 1;
-    const int world = std::max(1, p.world), rank = p.rank;
+    if (grp_owner.empty())  // placement 0 (or one rank): round-robin over the priority order
+        for (int64_t q = 0; q < G; q++) owner[q] = (int32_t)(q % world);
 
     // ---- internal numbering: vertices in degree-descending order (ties by id).
     // The H highest-degree vertices get ids [0, H) so the path kernel keeps them
@@ -772,13 +827,13 @@ void build_layouts(const HostCSR& g, const dg_path_params& p, const std::vector<
         }
     }
 
-    // ---- boundary vertices: present in partitions of >1 rank (round-robin owner q % world)
+    // ---- the boundary: vertices present in partitions of more than one rank
     if (world > 1) {
         std::vector<uint64_t> present(n, 0);  // ranks whose partitions hold v
         for (int64_t q = 0; q < G; q++) {
-            uint64_t bit = 1ull << ((q % world) & 63);
+            const uint64_t bit = 1ull << owner[q];
             for (int64_t r = gpart_first[q]; r < gpart_first[q + 1]; r++) {
-                int64_t i = order[r];
+                const int64_t i = order[r];
                 for (int64_t k = moff[i]; k < moff[i + 1]; k++) present[mv[k]] |= bit;
             }
         }
@@ -809,7 +864,8 @@ void build_layouts(const HostCSR& g, const dg_path_params& p, const std::vector<
         std::vector<int64_t> sel;
         L.part_off.push_back(0);
         std::vector<int64_t> part_paths{0};
-        for (int64_t q = rank; q < G; q += world) {
+        for (int64_t q = 0; q < G; q++) {
+            if (owner[q] != rank) continue;
             for (int64_t r = gpart_first[q]; r < gpart_first[q + 1]; r++) sel.push_back(order[r]);
             part_paths.push_back((int64_t)sel.size());
         }

@@ -76,19 +76,20 @@ class DiGraph:
 
     @staticmethod
     def _path_params(d_max=16, l_merge=64, n_sub=64, order="degree", hot_factor=2.0,
-                     part_entries=0, rank=0, world=1, merge_rule="relaxed", n_proxy=8192):
+                     part_entries=0, rank=0, world=1, merge_rule="relaxed", n_proxy=8192, placement="locality"):
         p = default_params()
         p.d_max, p.l_merge, p.n_sub = d_max, l_merge, n_sub
         p.order = 0 if order == "degree" else 1
         p.hot_factor, p.part_entries, p.rank, p.world = hot_factor, part_entries, rank, world
         p.merge_rule = {"paper": 0, "relaxed": 1}[merge_rule]
         p.n_proxy = n_proxy
+        p.placement = {"round_robin": 0, "locality": 1}[placement]
         return p
 
     def build_paths(self, d_max=16, l_merge=64, n_sub=64, order="degree", hot_factor=2.0,
-                    part_entries=0, rank=0, world=1, merge_rule="relaxed", n_proxy=8192):
+                    part_entries=0, rank=0, world=1, merge_rule="relaxed", n_proxy=8192, placement="locality"):
         p = self._path_params(d_max, l_merge, n_sub, order, hot_factor, part_entries, rank, world, merge_rule,
-                              n_proxy)
+                              n_proxy, placement)
         check(self._L.dg_build_paths(self._h, ctypes.byref(p)), "dg_build_paths")
         self.p2p_key = None  # the library freed any exchange region
         return self

@@ -114,14 +114,16 @@ def test_edge_weights_follow_paths():
     assert sorted(cover) == sorted(zip(src.tolist(), dst.tolist()))
 
 
-def test_multirank_partitioning_is_a_disjoint_cover():
+@pytest.mark.parametrize("placement", ["locality", "round_robin"])
+def test_multirank_partitioning_is_a_disjoint_cover(placement):
     g = inputs.rmat(10, 1000, 8000, seed=3)
     world = 3
-    covers, bnd_sets, presence = [], [], []
+    covers, bnd_sets, presence, entries = [], [], [], []
     for r in range(world):
         dg = DiGraph()
         dg.load_graph(g)
-        dg.build_paths(part_entries=128, rank=r, world=world)
+        dg.build_paths(part_entries=128, rank=r, world=world, placement=placement)
+        entries.append(dg.layout_info()["n_entries"])
         ex = dg.export_paths()
         cov = []
         for p in split(ex):
@@ -135,8 +137,22 @@ def test_multirank_partitioning_is_a_disjoint_cover():
     # boundary = vertices replicated on more than one rank's paths
     multi = sorted(v for v in range(g.n) if sum(v in s_ for s_ in presence) > 1)
     assert bnd_sets[0] == multi
-    sizes = [len(c) for c in covers]
-    assert max(sizes) - min(sizes) <= 0.2 * max(sizes)       # balanced
+    # balanced in path entries (what a rank's kernel walks): within 2 % of an
+    # even share plus one partition for the locality placement
+    assert max(entries) - min(entries) <= 0.1 * max(entries), entries
+
+
+def test_locality_placement_shrinks_the_boundary():
+    """Reading R-PLACE: paths go to the rank already holding most of their
+    vertices, so fewer vertices are replicated than with round-robin
+    partitions (same graph, same world)."""
+    for g, gain in ((inputs.chains(40000, 60000, chain_len=512, seed=5), 0.6),
+                    (inputs.rmat(13, 8192, 80000, seed=31), 1.0)):
+        nb = {}
+        for pl in ("round_robin", "locality"):
+            dg = DiGraph().load_graph(g).build_paths(part_entries=256, rank=0, world=2, placement=pl)
+            nb[pl] = dg.layout_info()["n_boundary"]
+        assert nb["locality"] < gain * nb["round_robin"], nb
 
 
 def test_run_without_cuda_fails_loudly():
