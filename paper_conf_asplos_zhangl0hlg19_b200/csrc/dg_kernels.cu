@@ -174,6 +174,7 @@ struct KParams {
     uint32_t sparse_occ;      // ... and are walked sparse if their out-edges are at most this many
     int sparse_walk;          // path edges a sparse walk follows at most
     MultiRank mr;             // world > 1: fused multi-rank run
+    int acc_skip;               // accumulative walk: gather only the masters of signalled vertices (DG_ACC_SKIP)
     unsigned* qtick;            // per-CTA partition queue counters, 2 x grid x kQStride (null: global ticket)
     unsigned long long* trace;  // DG_TRACE: per round {end time ns, vertices signalled into it, dense, out-edges}
     int trace_cap;
@@ -956,7 +957,8 @@ template <int NW>
 __host__ __device__ constexpr size_t gbuf_bytes() { return (size_t)NW * kRing * 128 * sizeof(uint4); }
 template <bool ADS>
 __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned long long pol_stream,
-                           unsigned long long pol_keep, const Proxies& px, uint4* gbuf, int* s_done) {
+                           unsigned long long pol_keep, const Proxies& px, uint4* gbuf, int* s_done,
+                           const uint32_t* bcur) {
     const int lane = threadIdx.x & 31;
     const unsigned long long eps = P.eps_fx;
     const uint4 kFill = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
@@ -974,15 +976,36 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
             cf = make_float4(0.f, 0.f, 0.f, 0.f);
         }
     };
+    // signal-bitmap words of a window's four entries (L1-cached: the bitmap is
+    // read-only during the walk); with P.acc_skip only the entries of
+    // signalled vertices (T grew by >= eps since their last signal) gather
+    // their master -- an entry of a vertex not signalled has pend < 2 eps
+    // (reading R-ACT) and is walked with pend = 0
+    auto probe = [&](const Win& w, const uint4& code, uint4& words) {
+        words = make_uint4(0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu);
+        if (!P.acc_skip || w.base == kNoWin) return;
+#pragma unroll
+        for (int k = 0; k < 4; k++) {
+            const uint32_t wd = __ldg(&bcur[(u4get(code, k) & kVMask) >> 5]);
+            if (k == 0) words.x = wd; else if (k == 1) words.y = wd; else if (k == 2) words.z = wd; else words.w = wd;
+        }
+    };
+    auto sigmask = [&](const uint4& code, const uint4& words) {
+        unsigned m = 0;
+#pragma unroll
+        for (int k = 0; k < 4; k++) m |= ((u4get(words, k) >> (u4get(code, k) & 31)) & 1u) << k;
+        return m;
+    };
     // masters of a window into ring slot s: entry 4*lane+k -> gbuf[s*128 + k*32 + lane]
-    // (16-byte aligned pair {T[v & ~1], T[v | 1]}); proxies and invalid entries skip
-    auto gather = [&](const Win& w, const uint4& code, int s) {
+    // (16-byte aligned pair {T[v & ~1], T[v | 1]}); proxies, invalid and
+    // unsignalled entries skip
+    auto gather = [&](const Win& w, const uint4& code, unsigned sm, int s) {
         if (w.base != kNoWin) {
 #pragma unroll
             for (int k = 0; k < 4; k++) {
                 const uint32_t i = w.base + 4 * lane + k;
                 const uint32_t v = u4get(code, k) & kVMask;
-                if (i >= w.beg && i < w.end && v >= px.H)
+                if (i >= w.beg && i < w.end && v >= px.H && ((sm >> k) & 1u))
                     cp_async16(&gbuf[s * 128 + k * 32 + lane], P.vs_t + (v & ~1u), pol_keep);
             }
         }
@@ -1002,14 +1025,20 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
     unsigned long long sv_c[4], sv_n[4];
     float4 cf_c, cf_n;
     load_sv(w0, sv_c, cf_c);
-    gather(w0, c0, 0);
-    gather(w1, c1, 1);
+    uint4 pw;
+    probe(w0, c0, pw);
+    unsigned sm0 = sigmask(c0, pw);
+    probe(w1, c1, pw);
+    unsigned sm1 = sigmask(c1, pw);
+    gather(w0, c0, sm0, 0);
+    gather(w1, c1, sm1, 1);
     int slot = 0;
     float carry = 0.f;
     while (w0.base != kNoWin) {
         const Win w3 = feed_next(P, q, w2, f);
         const uint4 c3 = load_code(w3);
-        gather(w2, c2, slot == 0 ? 2 : slot - 1);  // slot (w+2) % kRing
+        uint4 pw2;
+        probe(w2, c2, pw2);  // consumed after this window's walk (gathers of w+2)
         load_sv(w1, sv_n, cf_n);
         const bool part_start = w0.base == (w0.beg & ~3u);
         if (part_start) {
@@ -1021,7 +1050,7 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
                 if (c % P.px_refresh == 0) px_refresh(P, px);
             }
         }
-        asm volatile("cp.async.wait_group 2;" ::: "memory");  // window w's masters (its own lane's copies)
+        asm volatile("cp.async.wait_group 1;" ::: "memory");  // window w's masters (its own lane's copies)
         const uint32_t i0 = w0.base + 4 * lane;
         uint32_t vtx[4];
         unsigned long long T[4], pend[4];
@@ -1035,7 +1064,7 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
             hd[k] = !valid[k] || (c & kHead);
             tl[k] = !valid[k] || (c & kTail);
             T[k] = 0ull;
-            if (valid[k]) {
+            if (valid[k] && ((sm0 >> k) & 1u)) {
                 if (vtx[k] < px.H) {
                     T[k] = px.T[vtx[k]] + px_read(&px.acc[2 * vtx[k]]);
                 } else {
@@ -1044,7 +1073,7 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
                 }
             }
             const unsigned long long pd = T[k] > sv_c[k] ? T[k] - sv_c[k] : 0ull;
-            pend[k] = (!tl[k] && pd >= eps) ? pd : 0ull;
+            pend[k] = (!tl[k] && ((sm0 >> k) & 1u) && pd >= eps) ? pd : 0ull;
             any_act |= pend[k] != 0ull;
         }
         if (__any_sync(0xffffffffu, any_act) || carry != 0.f) {
@@ -1111,9 +1140,13 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
         } else {
             carry = 0.f;
         }
+        // masters of window w+2 (its signal bits arrived during the walk)
+        const unsigned sm2 = sigmask(c2, pw2);
+        gather(w2, c2, sm2, slot == 0 ? 2 : slot - 1);  // slot (w+2) % kRing
         // rotate the pipeline
         w0 = w1; w1 = w2; w2 = w3;
         c0 = c1; c1 = c2; c2 = c3;
+        sm0 = sm1; sm1 = sm2;
 #pragma unroll
         for (int k = 0; k < 4; k++) sv_c[k] = sv_n[k];
         cf_c = cf_n;
@@ -1495,7 +1528,7 @@ __global__ void __launch_bounds__(NW * 32, MINB) path_kernel(KParams P) {
                 if (threadIdx.x == 0) s_done = 0;
                 __syncthreads();
             }
-            walk_accum<ALGO == DG_ADSORPTION>(P, dq, acc, pol_stream, pol_keep, px, gbuf, &s_done);
+            walk_accum<ALGO == DG_ADSORPTION>(P, dq, acc, pol_stream, pol_keep, px, gbuf, &s_done, bcur);
             if (px.H) {  // send the proxies' accumulated pushes to their masters
                 __syncthreads();
                 for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x)
@@ -2325,6 +2358,8 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
     {
         const char* e = std::getenv("DG_PROXY_REFRESH");  // developer knob
         P.px_refresh = e ? std::atoi(e) : DG_PROXY_REFRESH;
+        const char* sk = std::getenv("DG_ACC_SKIP");  // developer knob (default: skip)
+        P.acc_skip = sk ? std::atoi(sk) : 1;
     }
     if (accum && P.n_proxy) {
         // as many proxies as fit next to the rings in one CTA per SM (the top
