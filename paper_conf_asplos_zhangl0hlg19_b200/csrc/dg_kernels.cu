@@ -174,7 +174,6 @@ struct KParams {
     uint32_t sparse_occ;      // ... and are walked sparse if their out-edges are at most this many
     int sparse_walk;          // path edges a sparse walk follows at most
     MultiRank mr;             // world > 1: fused multi-rank run
-    int acc_skip;               // accumulative walk: gather only the masters of signalled vertices (DG_ACC_SKIP)
     unsigned* qtick;            // per-CTA partition queue counters, 2 x grid x kQStride (null: global ticket)
     unsigned long long* trace;  // DG_TRACE: per round {end time ns, vertices signalled into it, dense, out-edges}
     int trace_cap;
@@ -447,14 +446,31 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
     bool act_c[4], act_n[4];
     uint32_t a_c[4] = {INF, INF, INF, INF}, a_n[4] = {INF, INF, INF, INF};
     bool any_c = probe_finish(wc, code_c, words_c, act_c, a_c);
+    // SSSP: the path-edge weights of an active window are in flight one window ahead
+    auto load_w = [&](const Win& w, bool any) {
+        int4 wv = make_int4(0, 0, 0, 0);
+        if (MODE == 0 && any && w.base + 4 * lane < w.end) wv = ld_stream_i4(P.e_w + w.base + 4 * lane);
+        return wv;
+    };
+    int4 wv_c = load_w(wc, any_c);
     uint32_t carry = INF, carry_vtx = 0;
     bool carry_live = false;
+    // atomicMins in flight from the previous walked window (settled one window later)
+    uint32_t d_old[4] = {0u, 0u, 0u, 0u}, d_val[4] = {0u, 0u, 0u, 0u};
+    unsigned d_mask = 0;
+    auto settle = [&]() {
+#pragma unroll
+        for (int k = 0; k < 4; k++)
+            if (((d_mask >> k) & 1u) && d_val[k] < d_old[k]) acc.upd++;
+        d_mask = 0;
+    };
     while (wc.base != kNoWin) {
         const Win wn3 = win_next(P, wn2, ticket);
         const uint4 code_n3 = load_code(wn3);
         uint4 words_n2;
         probe_words(wn2, code_n2, words_n2);
         const bool any_n = probe_finish(wn, code_n, words_n, act_n, a_n);
+        const int4 wv_n = load_w(wn, any_n);
         if (wc.base == (wc.beg & ~3u)) { carry = INF; carry_live = false; }  // partition start
         const uint32_t i0 = wc.base + 4 * lane;
         // WCC looks one entry ahead: the path edge into the next window is walked backwards too
@@ -481,8 +497,8 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
                     a_c[k] = (i >= wc.beg && i < wc.end) ? P.vs_u[u4get(code_c, k) & kVMask] : INF;
                 }
             }
-            int4 wv = make_int4(0, 0, 0, 0);
-            if (MODE == 0 && i0 < wc.end) wv = ld_stream_i4(P.e_w + i0);
+            int4 wv = wv_c;
+            if (MODE == 0 && !any_c && i0 < wc.end) wv = ld_stream_i4(P.e_w + i0);  // walked for a carry only
             uint32_t vtx[4], a[4], wgt[4];
             bool hd[4], tl[4], live[4];
 #pragma unroll
@@ -548,37 +564,39 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
             // path predecessor of entry 0 (previous lane's last entry, or the carry's vertex)
             uint32_t pred0 = __shfl_up_sync(0xffffffffu, vtx[3], 1);
             if (lane == 0) pred0 = carry_vtx;
-            // the lane's (up to four) atomicMins are issued back to back and
-            // are in flight together; their results are consumed afterwards
-            uint32_t old[4];
-#pragma unroll
-            for (int k = 0; k < 4; k++) {
-                old[k] = 0u;
-                if (live[k] && val[k] < a[k] && val[k] <= theta) old[k] = atomicMin(&P.vs_u[vtx[k]], val[k]);
-            }
+            // the previous window's atomicMin results have had a whole window to
+            // arrive: count its successful updates now
+            settle();
+            // the lane's (up to four) atomicMins are issued back to back; their
+            // results are consumed one window later (settle), so no window waits
+            // for its atomics.  The signal of a lowered vertex is a fire-and-forget
+            // RED issued with the atomic: if another walk lowered the vertex
+            // further in the meantime, that walk signalled it too (a duplicate
+            // signal only re-walks the vertex), and the active counter is an
+            // upper bound, which is all its uses need (non-zero test, sparse
+            // threshold).  The bucket base (vmin) and the carry use the
+            // attempted value: the smallest attempt is the smallest commit.
 #pragma unroll
             for (int k = 0; k < 4; k++) {
                 if (!live[k]) continue;
                 acc.entries++;
                 if (!(u4get(code_c, k) & kHead)) acc.edges++;
-                if (val[k] < a[k]) {
-                    if (val[k] > theta) {
-                        // beyond this round's bucket: not committed; the path
-                        // predecessor stays active so the edge is relaxed again
-                        acc.sig += signal_vertex(bnxt, k ? vtx[k - 1] : pred0);
-                        continue;
-                    }
-                    if (val[k] < old[k]) {
-                        acc.upd++;
-                        if (k == 3) changed3 = true;
-                        // fire-and-forget signal (RED): the active counter may count a
-                        // vertex lowered twice in one round twice -- an upper bound,
-                        // which is all its uses need (non-zero test, sparse threshold)
-                        atomicOr(&bnxt[vtx[k] >> 5], 1u << (vtx[k] & 31));
-                        acc.sig++;
-                        acc.vmin = min(acc.vmin, val[k]);
-                    }
+                if (!(val[k] < a[k])) continue;
+                if (val[k] > theta) {
+                    // beyond this round's bucket: not committed; the path
+                    // predecessor stays active so the edge is relaxed again
+                    const uint32_t pv = k ? vtx[k - 1] : pred0;
+                    atomicOr(&bnxt[pv >> 5], 1u << (pv & 31));
+                    acc.sig++;
+                    continue;
                 }
+                d_old[k] = atomicMin(&P.vs_u[vtx[k]], val[k]);
+                d_val[k] = val[k];
+                d_mask |= 1u << k;
+                atomicOr(&bnxt[vtx[k] >> 5], 1u << (vtx[k] & 31));
+                acc.sig++;
+                acc.vmin = min(acc.vmin, val[k]);
+                if (k == 3) changed3 = true;
             }
             // the carry into the next window is live if the path continues and its
             // last vertex changed now or was signalled (its out-edge must be relaxed)
@@ -594,9 +612,11 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
         code_c = code_n; code_n = code_n2; code_n2 = code_n3;
         words_n = words_n2;
         any_c = any_n;
+        wv_c = wv_n;
 #pragma unroll
         for (int k = 0; k < 4; k++) { act_c[k] = act_n[k]; a_c[k] = a_n[k]; }
     }
+    settle();
 }
 
 // Sparse min-plus rounds (SSSP/BFS, the forward half of WCC, SCC's forward
@@ -957,8 +977,7 @@ template <int NW>
 __host__ __device__ constexpr size_t gbuf_bytes() { return (size_t)NW * kRing * 128 * sizeof(uint4); }
 template <bool ADS>
 __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned long long pol_stream,
-                           unsigned long long pol_keep, const Proxies& px, uint4* gbuf, int* s_done,
-                           const uint32_t* bcur) {
+                           unsigned long long pol_keep, const Proxies& px, uint4* gbuf, int* s_done) {
     const int lane = threadIdx.x & 31;
     const unsigned long long eps = P.eps_fx;
     const uint4 kFill = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
@@ -976,36 +995,15 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
             cf = make_float4(0.f, 0.f, 0.f, 0.f);
         }
     };
-    // signal-bitmap words of a window's four entries (L1-cached: the bitmap is
-    // read-only during the walk); with P.acc_skip only the entries of
-    // signalled vertices (T grew by >= eps since their last signal) gather
-    // their master -- an entry of a vertex not signalled has pend < 2 eps
-    // (reading R-ACT) and is walked with pend = 0
-    auto probe = [&](const Win& w, const uint4& code, uint4& words) {
-        words = make_uint4(0xffffffffu, 0xffffffffu, 0xffffffffu, 0xffffffffu);
-        if (!P.acc_skip || w.base == kNoWin) return;
-#pragma unroll
-        for (int k = 0; k < 4; k++) {
-            const uint32_t wd = __ldg(&bcur[(u4get(code, k) & kVMask) >> 5]);
-            if (k == 0) words.x = wd; else if (k == 1) words.y = wd; else if (k == 2) words.z = wd; else words.w = wd;
-        }
-    };
-    auto sigmask = [&](const uint4& code, const uint4& words) {
-        unsigned m = 0;
-#pragma unroll
-        for (int k = 0; k < 4; k++) m |= ((u4get(words, k) >> (u4get(code, k) & 31)) & 1u) << k;
-        return m;
-    };
     // masters of a window into ring slot s: entry 4*lane+k -> gbuf[s*128 + k*32 + lane]
-    // (16-byte aligned pair {T[v & ~1], T[v | 1]}); proxies, invalid and
-    // unsignalled entries skip
-    auto gather = [&](const Win& w, const uint4& code, unsigned sm, int s) {
+    // (16-byte aligned pair {T[v & ~1], T[v | 1]}); proxies and invalid entries skip
+    auto gather = [&](const Win& w, const uint4& code, int s) {
         if (w.base != kNoWin) {
 #pragma unroll
             for (int k = 0; k < 4; k++) {
                 const uint32_t i = w.base + 4 * lane + k;
                 const uint32_t v = u4get(code, k) & kVMask;
-                if (i >= w.beg && i < w.end && v >= px.H && ((sm >> k) & 1u))
+                if (i >= w.beg && i < w.end && v >= px.H)
                     cp_async16(&gbuf[s * 128 + k * 32 + lane], P.vs_t + (v & ~1u), pol_keep);
             }
         }
@@ -1025,20 +1023,14 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
     unsigned long long sv_c[4], sv_n[4];
     float4 cf_c, cf_n;
     load_sv(w0, sv_c, cf_c);
-    uint4 pw;
-    probe(w0, c0, pw);
-    unsigned sm0 = sigmask(c0, pw);
-    probe(w1, c1, pw);
-    unsigned sm1 = sigmask(c1, pw);
-    gather(w0, c0, sm0, 0);
-    gather(w1, c1, sm1, 1);
+    gather(w0, c0, 0);
+    gather(w1, c1, 1);
     int slot = 0;
     float carry = 0.f;
     while (w0.base != kNoWin) {
         const Win w3 = feed_next(P, q, w2, f);
         const uint4 c3 = load_code(w3);
-        uint4 pw2;
-        probe(w2, c2, pw2);  // consumed after this window's walk (gathers of w+2)
+        gather(w2, c2, slot == 0 ? 2 : slot - 1);  // slot (w+2) % kRing
         load_sv(w1, sv_n, cf_n);
         const bool part_start = w0.base == (w0.beg & ~3u);
         if (part_start) {
@@ -1050,7 +1042,7 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
                 if (c % P.px_refresh == 0) px_refresh(P, px);
             }
         }
-        asm volatile("cp.async.wait_group 1;" ::: "memory");  // window w's masters (its own lane's copies)
+        asm volatile("cp.async.wait_group 2;" ::: "memory");  // window w's masters (its own lane's copies)
         const uint32_t i0 = w0.base + 4 * lane;
         uint32_t vtx[4];
         unsigned long long T[4], pend[4];
@@ -1064,7 +1056,7 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
             hd[k] = !valid[k] || (c & kHead);
             tl[k] = !valid[k] || (c & kTail);
             T[k] = 0ull;
-            if (valid[k] && ((sm0 >> k) & 1u)) {
+            if (valid[k]) {
                 if (vtx[k] < px.H) {
                     T[k] = px.T[vtx[k]] + px_read(&px.acc[2 * vtx[k]]);
                 } else {
@@ -1073,7 +1065,7 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
                 }
             }
             const unsigned long long pd = T[k] > sv_c[k] ? T[k] - sv_c[k] : 0ull;
-            pend[k] = (!tl[k] && ((sm0 >> k) & 1u) && pd >= eps) ? pd : 0ull;
+            pend[k] = (!tl[k] && pd >= eps) ? pd : 0ull;
             any_act |= pend[k] != 0ull;
         }
         if (__any_sync(0xffffffffu, any_act) || carry != 0.f) {
@@ -1140,13 +1132,9 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
         } else {
             carry = 0.f;
         }
-        // masters of window w+2 (its signal bits arrived during the walk)
-        const unsigned sm2 = sigmask(c2, pw2);
-        gather(w2, c2, sm2, slot == 0 ? 2 : slot - 1);  // slot (w+2) % kRing
         // rotate the pipeline
         w0 = w1; w1 = w2; w2 = w3;
         c0 = c1; c1 = c2; c2 = c3;
-        sm0 = sm1; sm1 = sm2;
 #pragma unroll
         for (int k = 0; k < 4; k++) sv_c[k] = sv_n[k];
         cf_c = cf_n;
@@ -1528,7 +1516,7 @@ __global__ void __launch_bounds__(NW * 32, MINB) path_kernel(KParams P) {
                 if (threadIdx.x == 0) s_done = 0;
                 __syncthreads();
             }
-            walk_accum<ALGO == DG_ADSORPTION>(P, dq, acc, pol_stream, pol_keep, px, gbuf, &s_done, bcur);
+            walk_accum<ALGO == DG_ADSORPTION>(P, dq, acc, pol_stream, pol_keep, px, gbuf, &s_done);
             if (px.H) {  // send the proxies' accumulated pushes to their masters
                 __syncthreads();
                 for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x)
@@ -2358,8 +2346,6 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
     {
         const char* e = std::getenv("DG_PROXY_REFRESH");  // developer knob
         P.px_refresh = e ? std::atoi(e) : DG_PROXY_REFRESH;
-        const char* sk = std::getenv("DG_ACC_SKIP");  // developer knob (default: skip)
-        P.acc_skip = sk ? std::atoi(sk) : 1;
     }
     if (accum && P.n_proxy) {
         // as many proxies as fit next to the rings in one CTA per SM (the top
