@@ -119,6 +119,9 @@ typedef struct {
     double preprocess_ms;         /* host time of dg_build_paths                    */
     int64_t device_bytes;         /* device memory held by the layout               */
     int64_t h2d_bytes;            /* bytes the last dg_upload copied host -> device */
+    int64_t boundary_reads;       /* peer slots this rank reads per peer-memory exchange:
+                                     sum over the boundary vertices its paths hold of
+                                     (ranks holding the vertex - 1); x 8 B = NVLink bytes */
 } dg_layout_info;
 
 /* Create an empty graph bound to CUDA device `device` (cudaSetDevice is

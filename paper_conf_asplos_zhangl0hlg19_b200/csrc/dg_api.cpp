@@ -378,6 +378,9 @@ int dg_get_layout_info(const dg_graph* g, dg_layout_info* info) {
     info->preprocess_ms = L.preprocess_ms;
     info->device_bytes = g->dev.bytes;
     info->h2d_bytes = g->dev.h2d_bytes;
+    const int rk = L.params.rank;
+    for (const uint64_t h : L.bnd_hold)
+        if ((h >> rk) & 1ull) info->boundary_reads += __builtin_popcountll(h) - 1;
     return DG_OK;
 }
 

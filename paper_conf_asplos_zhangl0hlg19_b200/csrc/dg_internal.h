@@ -52,6 +52,7 @@ struct HostLayout {
     std::vector<int32_t> scol;
     // multi-rank
     std::vector<int32_t> boundary;      // internal ids of vertices present on >1 rank (ascending)
+    std::vector<uint64_t> bnd_hold;     // per boundary vertex: bit r set iff rank r's paths hold it
     std::vector<float> wsum;            // per vertex (internal ids): sum of out-edge weights (Adsorption)
     bool has_csr = true;                // prow_ptr/pcol/pw present (false: loaded from a layout file)
     // stats
@@ -77,6 +78,7 @@ struct DevLayout {
     int32_t* e_w = nullptr;
     int64_t* part_off = nullptr;
     int32_t* bnd = nullptr;
+    unsigned long long* bnd_hold = nullptr;  // holder ranks of each boundary vertex
     int32_t* new_id = nullptr;  // original -> internal
     int32_t* orig = nullptr;    // internal -> original
     int64_t n_proxy = 0;

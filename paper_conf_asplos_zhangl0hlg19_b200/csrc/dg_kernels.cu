@@ -54,9 +54,6 @@ constexpr int kPad = 256;  // zero entries after every per-entry array
 #ifndef DG_PATH_MINB
 #define DG_PATH_MINB 3  // resident CTAs per SM requested for the path kernel
 #endif
-#ifndef DG_PROXY_REFRESH
-#define DG_PROXY_REFRESH 8  // default: partitions a CTA walks between mid-round proxy flushes (0 = round end only)
-#endif
 
 // device counters of a run
 struct Counters {
@@ -127,6 +124,7 @@ struct MultiRank {
     const unsigned char* region[kP2PMaxRanks];  // every rank's region in this address space (own included)
     unsigned long long* own;                    // this rank's region
     const int32_t* bnd;                         // boundary vertices (internal ids), identical on every rank
+    const unsigned long long* hold;             // holder ranks of each boundary vertex (bit r: rank r)
     unsigned long long* base;                   // SUM: total after the last exchange
     uint32_t* last;                             // MIN: reduced value of the last exchange
     int64_t nb;
@@ -300,8 +298,9 @@ __device__ __forceinline__ void cp_async_wait0() { asm volatile("cp.async.wait_g
 // together.  A CTA's warps take partitions from its own queue (one atomic on
 // the CTA's own counter, on its own 32-byte line); once it is empty they steal
 // single partitions from the other CTAs' queues, starting at the next CTA, and
-// a per-CTA shared cursor skips victims found empty.  DG_DISPATCH=0 (developer
-// knob) restores one global ticket.
+// a per-CTA shared cursor skips victims found empty.  This is DG_DISPATCH=1
+// (developer knob); the default is one global ticket, which measured faster
+// (the accumulative walk also prefetches its tickets a partition ahead).
 struct Queue {
     unsigned* qt;        // per-CTA counters of this round (stride kQStride)
     unsigned* global;    // the single global ticket (DG_DISPATCH=0)
@@ -1361,7 +1360,11 @@ __device__ __forceinline__ bool mr_exchange(const KParams& P, cg::grid_group& gr
     const size_t off = kP2PHeader + (size_t)(e & 1) * M.slot_bytes;
     unsigned long long* mine = (unsigned long long*)((unsigned char*)M.own + off);
     unsigned dirty = 0;
+    // only the ranks holding a boundary vertex take part in its reduction: a
+    // rank packs and reduces the vertices its paths hold, reading the slots of
+    // their other holders only (DESIGN.md sec. 4 "Peer-memory exchange")
     for (int64_t k = t0; k < M.nb; k += T) {
+        if (!((M.hold[k] >> M.rank) & 1ull)) continue;
         const int v = M.bnd[k];
         if (M.sum) {
             const unsigned long long g = P.vs_t[v] - M.base[k];
@@ -1420,10 +1423,13 @@ __device__ __forceinline__ bool mr_exchange(const KParams& P, cg::grid_group& gr
     uint32_t* b = P.bits + (int64_t)ncur * P.nw;
     unsigned cnt = 0;
     for (int64_t k = t0; k < M.nb; k += T) {
+        const unsigned long long hm = M.hold[k];
+        if (!((hm >> M.rank) & 1ull)) continue;
         const int v = M.bnd[k];
         if (M.sum) {
             unsigned long long g = 0;
-            for (int r = 0; r < M.world; r++) g += __ldcv((const unsigned long long*)(M.region[r] + off) + k);
+            for (unsigned long long q = hm; q; q &= q - 1)
+                g += __ldcv((const unsigned long long*)(M.region[__ffsll((long long)q) - 1] + off) + k);
             const unsigned long long t = M.base[k] + g;
             M.base[k] = t;
             P.vs_t[v] = t;
@@ -1433,7 +1439,8 @@ __device__ __forceinline__ bool mr_exchange(const KParams& P, cg::grid_group& gr
             }
         } else {
             unsigned long long m = ~0ull;
-            for (int r = 0; r < M.world; r++) m = min(m, __ldcv((const unsigned long long*)(M.region[r] + off) + k));
+            for (unsigned long long q = hm; q; q &= q - 1)
+                m = min(m, __ldcv((const unsigned long long*)(M.region[__ffsll((long long)q) - 1] + off) + k));
             M.last[k] = (uint32_t)m;
             if (M.mark) {  // marked on some rank: reachable backward from its colour's root
                 if (m == 0 && !P.mark[v] && P.scc_label[v] < 0) {
@@ -2040,13 +2047,13 @@ __global__ void unpack_sum_kernel(unsigned long long* vs, unsigned long long* si
 struct PeerSlots {
     const void* p[kP2PMaxRanks];
 };
-__global__ void p2p_pack_min_kernel(const uint32_t* vs, const uint8_t* mark, const int32_t* bnd, int64_t nb,
-                                    unsigned long long* slot) {
-    GRID_STRIDE(k, nb) slot[k] = min_value(vs, mark, bnd[k]);
+__global__ void p2p_pack_min_kernel(const uint32_t* vs, const uint8_t* mark, const int32_t* bnd,
+                                    const unsigned long long* hold, int rank, int64_t nb, unsigned long long* slot) {
+    GRID_STRIDE(k, nb) if ((hold[k] >> rank) & 1ull) slot[k] = min_value(vs, mark, bnd[k]);
 }
-__global__ void p2p_pack_sum_kernel(const unsigned long long* vs, const int32_t* bnd, int64_t nb,
-                                    const unsigned long long* base, unsigned long long* slot) {
-    GRID_STRIDE(k, nb) slot[k] = vs[bnd[k]] - base[k];
+__global__ void p2p_pack_sum_kernel(const unsigned long long* vs, const int32_t* bnd, const unsigned long long* hold,
+                                    int rank, int64_t nb, const unsigned long long* base, unsigned long long* slot) {
+    GRID_STRIDE(k, nb) if ((hold[k] >> rank) & 1ull) slot[k] = vs[bnd[k]] - base[k];
 }
 __global__ void p2p_signal_wait_kernel(PeerSlots flags, int world, int rank, unsigned long long epoch,
                                        unsigned long long* own_flags, unsigned long long timeout_ns) {
@@ -2072,25 +2079,33 @@ __global__ void p2p_signal_wait_kernel(PeerSlots flags, int world, int rank, uns
         }
     }
 }
-__global__ void p2p_reduce_min_kernel(PeerSlots slots, int world, uint32_t* vs, uint8_t* mark, const int32_t* label,
-                                      const int32_t* bnd, int64_t nb, uint32_t* b, Counters* ctr, int slot) {
+__global__ void p2p_reduce_min_kernel(PeerSlots slots, int rank, uint32_t* vs, uint8_t* mark, const int32_t* label,
+                                      const int32_t* bnd, const unsigned long long* hold, int64_t nb, uint32_t* b,
+                                      Counters* ctr, int slot) {
     unsigned cnt = 0;
     GRID_STRIDE(k, nb) {
+        const unsigned long long hm = hold[k];
+        if (!((hm >> rank) & 1ull)) continue;
         unsigned long long m = ~0ull;
-        for (int r = 0; r < world; r++) m = min(m, __ldcv((const unsigned long long*)slots.p[r] + k));
+        for (unsigned long long q = hm; q; q &= q - 1)
+            m = min(m, __ldcv((const unsigned long long*)slots.p[__ffsll((long long)q) - 1] + k));
         const int v = bnd[k];
         if (min_apply(vs, mark, label, v, (uint32_t)m)) cnt += signal_vertex(b, (uint32_t)v);
     }
     for (int off = 16; off; off >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, off);
     if ((threadIdx.x & 31) == 0 && cnt) atomicAdd(&ctr->active[slot], cnt);
 }
-__global__ void p2p_reduce_sum_kernel(PeerSlots slots, int world, unsigned long long* vs, unsigned long long* sigma,
-                                      const int32_t* bnd, int64_t nb, unsigned long long* base, unsigned long long eps,
-                                      uint32_t* b, Counters* ctr, int slot) {
+__global__ void p2p_reduce_sum_kernel(PeerSlots slots, int rank, unsigned long long* vs, unsigned long long* sigma,
+                                      const int32_t* bnd, const unsigned long long* hold, int64_t nb,
+                                      unsigned long long* base, unsigned long long eps, uint32_t* b, Counters* ctr,
+                                      int slot) {
     unsigned cnt = 0;
     GRID_STRIDE(k, nb) {
+        const unsigned long long hm = hold[k];
+        if (!((hm >> rank) & 1ull)) continue;
         unsigned long long g = 0;
-        for (int r = 0; r < world; r++) g += __ldcv((const unsigned long long*)slots.p[r] + k);
+        for (unsigned long long q = hm; q; q &= q - 1)
+            g += __ldcv((const unsigned long long*)slots.p[__ffsll((long long)q) - 1] + k);
         const int v = bnd[k];
         const unsigned long long t = base[k] + g;
         base[k] = t;
@@ -2162,8 +2177,11 @@ KParams make_params(const DevLayout& D, DevWork* W) {
     P.ctr = W->ctr;
     P.mark = W->scc_mark; P.scc_label = W->scc_label;
     P.orig = D.orig; P.n_proxy = D.n_proxy;
-    const char* dd = std::getenv("DG_DISPATCH");  // developer knob: 0 = one global ticket
-    P.qtick = (dd && std::atoi(dd) == 0) ? nullptr : W->qtick;
+    // partition dispatch: one global ticket in priority order (default), or
+    // per-CTA queues with work stealing (DG_DISPATCH=1, developer knob;
+    // measured slower, DESIGN.md sec. 4 "Dispatch")
+    const char* dd = std::getenv("DG_DISPATCH");
+    P.qtick = (dd && std::atoi(dd) == 1) ? W->qtick : nullptr;
     return P;
 }
 
@@ -2344,8 +2362,15 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
     if (const char* np = std::getenv("DG_N_PROXY")) P.n_proxy = std::min<int64_t>(P.n_proxy, std::max(0, std::atoi(np)));
     if (!accum) P.n_proxy = 0;
     {
+        // refresh interval: about 16 mid-round flushes per CTA and round, at
+        // least every 8 and at most every 128 partitions (measured: LJ-shaped
+        // prefers 8-16, Twitter-shaped 64-128; DESIGN.md sec. 4 "Proxies")
         const char* e = std::getenv("DG_PROXY_REFRESH");  // developer knob
-        P.px_refresh = e ? std::atoi(e) : DG_PROXY_REFRESH;
+        int dev = 0, sms = 148;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        const int64_t autoint = std::min<int64_t>(128, std::max<int64_t>(8, D.n_part / ((int64_t)sms * 16)));
+        P.px_refresh = e ? std::atoi(e) : (int)autoint;
     }
     if (accum && P.n_proxy) {
         // as many proxies as fit next to the rings in one CTA per SM (the top
@@ -2669,10 +2694,12 @@ int dev_upload_layout(DevLayout& D, const HostLayout& L, std::string& err) {
     if ((rc = dalloc_once(&D.e_idx, D.M + kPad, D.bytes, err))) return rc;
     if ((rc = dalloc_once(&D.part_off, D.n_part + 1, D.bytes, err))) return rc;
     if ((rc = dalloc_once(&D.bnd, D.n_bnd + 1, D.bytes, err))) return rc;
+    if ((rc = dalloc_once(&D.bnd_hold, D.n_bnd + 1, D.bytes, err))) return rc;
     CK(cudaMemset(D.e_idx + D.M, 0, sizeof(uint32_t) * kPad));
     if ((rc = h2d(D.e_idx, L.e_idx.data(), D.M, err))) return rc;
     if ((rc = h2d(D.part_off, L.part_off.data(), D.n_part + 1, err))) return rc;
     if ((rc = h2d(D.bnd, L.boundary.data(), D.n_bnd, err))) return rc;
+    if ((rc = h2d(D.bnd_hold, (const unsigned long long*)L.bnd_hold.data(), D.n_bnd, err))) return rc;
     CK(cudaDeviceSynchronize());
     g_h2d_counter = nullptr;
     g_pin_list = nullptr;
@@ -2686,7 +2713,7 @@ void dev_unpin_all(DevLayout& D) {
 }
 
 void dev_free_layout(DevLayout& D, bool csr_too) {
-    dfree(D.e_idx); dfree(D.e_w); dfree(D.part_off); dfree(D.bnd);
+    dfree(D.e_idx); dfree(D.e_w); dfree(D.part_off); dfree(D.bnd); dfree(D.bnd_hold);
     if (csr_too) {
         dfree(D.row_ptr); dfree(D.col); dfree(D.w); dfree(D.outdeg); dfree(D.new_id); dfree(D.orig);
         dfree(D.srow_ptr); dfree(D.scol);
@@ -3021,20 +3048,23 @@ int dev_boundary_exchange(DevWork* W, const DevLayout& D, RunState& S, P2P* X, i
     const bool sum = S.algo == DG_PAGERANK || S.algo == DG_ADSORPTION;
     unsigned long long* mine = (unsigned long long*)(X->own + off);
     if (D.n_bnd) {
-        if (sum) p2p_pack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_t, D.bnd, D.n_bnd, W->bnd_base, mine);
-        else p2p_pack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, scc_marks(W, S), D.bnd, D.n_bnd, mine);
+        if (sum)
+            p2p_pack_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_t, D.bnd, D.bnd_hold, X->rank, D.n_bnd, W->bnd_base, mine);
+        else
+            p2p_pack_min_kernel<<<grid_1d(D.n_bnd), 256>>>(W->vs_u, scc_marks(W, S), D.bnd, D.bnd_hold, X->rank, D.n_bnd,
+                                                           mine);
     }
     unsigned long long* own_flags = (unsigned long long*)X->own;
     p2p_signal_wait_kernel<<<1, 32>>>(flags, X->world, X->rank, e, own_flags, 60ull * 1000000000ull);
     if (D.n_bnd) {
         uint32_t* b = W->bits + (int64_t)slot * W->nw;
         if (sum)
-            p2p_reduce_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(slots, X->world, W->vs_t, W->sigma, D.bnd, D.n_bnd,
-                                                             W->bnd_base, (unsigned long long)(S.eps * 4294967296.0),
-                                                             b, W->ctr, slot);
+            p2p_reduce_sum_kernel<<<grid_1d(D.n_bnd), 256>>>(slots, X->rank, W->vs_t, W->sigma, D.bnd, D.bnd_hold,
+                                                             D.n_bnd, W->bnd_base,
+                                                             (unsigned long long)(S.eps * 4294967296.0), b, W->ctr, slot);
         else
-            p2p_reduce_min_kernel<<<grid_1d(D.n_bnd), 256>>>(slots, X->world, W->vs_u, scc_marks(W, S), W->scc_label,
-                                                             D.bnd, D.n_bnd, b, W->ctr, slot);
+            p2p_reduce_min_kernel<<<grid_1d(D.n_bnd), 256>>>(slots, X->rank, W->vs_u, scc_marks(W, S), W->scc_label,
+                                                             D.bnd, D.bnd_hold, D.n_bnd, b, W->ctr, slot);
     }
     S.stats.kernel_launches += D.n_bnd ? 3 : 1;
     CK(cudaGetLastError());
@@ -3061,6 +3091,7 @@ int dev_run_fused(DevWork* W, const DevLayout& D, RunState& S, P2P* X, int64_t l
     for (int r = 0; r < X->world; r++) M.region[r] = X->peer[r];
     M.own = (unsigned long long*)X->own;
     M.bnd = D.bnd;
+    M.hold = D.bnd_hold;
     M.base = W->bnd_base;
     M.last = X->last;
     M.nb = D.n_bnd;

@@ -18,7 +18,7 @@ namespace dg {
 namespace {
 
 constexpr char kMagic[8] = {'D', 'G', 'L', 'A', 'Y', 'O', 'U', 'T'};
-constexpr uint32_t kVersion = 2;
+constexpr uint32_t kVersion = 3;
 
 struct Header {
     char magic[8];
@@ -67,7 +67,7 @@ int save_layout(const HostCSR& g, const HostLayout& L, const char* path, std::st
     bool ok = std::fwrite(&h, sizeof h, 1, F.f) == 1;
     ok = ok && put(F.f, L.path_off) && put(F.f, L.layer) && put(F.f, L.scc) && put(F.f, L.merged_index) &&
          put(F.f, L.hot) && put(F.f, L.e_idx) && put(F.f, L.e_w) && put(F.f, L.part_off) && put(F.f, L.new_id) &&
-         put(F.f, L.orig) && put(F.f, L.poutdeg) && put(F.f, L.boundary) && put(F.f, L.wsum);
+         put(F.f, L.orig) && put(F.f, L.poutdeg) && put(F.f, L.boundary) && put(F.f, L.wsum) && put(F.f, L.bnd_hold);
     if (!ok) { err = std::string("write failed: ") + path; return DG_EINVAL; }
     return DG_OK;
 }
@@ -93,9 +93,11 @@ int load_layout(HostCSR& g, HostLayout& L, const char* path, std::string& err) {
     bool ok = get(F.f, l.path_off, big) && get(F.f, l.layer, big) && get(F.f, l.scc, big) &&
               get(F.f, l.merged_index, big) && get(F.f, l.hot, big) && get(F.f, l.e_idx, big) &&
               get(F.f, l.e_w, big) && get(F.f, l.part_off, big) && get(F.f, l.new_id, nv) && get(F.f, l.orig, nv) &&
-              get(F.f, l.poutdeg, nv) && get(F.f, l.boundary, nv) && get(F.f, l.wsum, nv);
+              get(F.f, l.poutdeg, nv) && get(F.f, l.boundary, nv) && get(F.f, l.wsum, nv) &&
+              get(F.f, l.bnd_hold, nv);
     ok = ok && l.new_id.size() == nv && l.orig.size() == nv && l.poutdeg.size() == nv && l.wsum.size() == nv &&
-         !l.part_off.empty() && l.e_w.size() == l.e_idx.size() && (uint64_t)l.part_off.back() == l.e_idx.size();
+         !l.part_off.empty() && l.e_w.size() == l.e_idx.size() && (uint64_t)l.part_off.back() == l.e_idx.size() &&
+         l.bnd_hold.size() == l.boundary.size();
     if (!ok) { err = std::string(path) + ": truncated or inconsistent layout file"; return DG_EINVAL; }
     l.has_csr = false;
     l.built = true;

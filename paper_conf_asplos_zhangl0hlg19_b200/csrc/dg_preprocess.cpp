@@ -837,9 +837,15 @@ void build_layouts(const HostCSR& g, const dg_path_params& p, const std::vector<
                 for (int64_t k = moff[i]; k < moff[i + 1]; k++) present[mv[k]] |= bit;
             }
         }
+        // boundary vertices (internal ids, ascending) and their holder ranks
+        std::vector<std::pair<int32_t, uint64_t>> bh;
         for (int64_t v = 0; v < n; v++)
-            if (__builtin_popcountll(present[v]) > 1) L.boundary.push_back(L.new_id[v]);
-        std::sort(L.boundary.begin(), L.boundary.end());
+            if (__builtin_popcountll(present[v]) > 1) bh.emplace_back(L.new_id[v], present[v]);
+        std::sort(bh.begin(), bh.end());
+        for (const auto& x : bh) {
+            L.boundary.push_back(x.first);
+            L.bnd_hold.push_back(x.second);
+        }
     }
 
     // per-vertex sum of out-edge weights (Adsorption's W(u), reading R-ADS), so

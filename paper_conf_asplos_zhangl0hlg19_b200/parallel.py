@@ -145,8 +145,11 @@ def run_distributed(engine, algo, source=0, epsilon=1e-7, damping=0.85, local_ro
         syncs = _converge(engine, *args)
     stats = engine.run_end()
     bytes_per_sync = buf.numel() * buf.element_size()
-    if exchange in ("fused", "p2p"):  # every rank reads each peer's 8-byte slot per boundary vertex
-        bytes_per_sync = 8 * nb * (dist.get_world_size(group) - 1)
+    if exchange in ("fused", "p2p"):
+        # a rank reads, for each boundary vertex its paths hold, the 8-byte slot
+        # of every other rank holding it (dg_layout_info.boundary_reads)
+        reads = engine.layout_info().get("boundary_reads") if hasattr(engine, "layout_info") else None
+        bytes_per_sync = 8 * (reads if reads is not None else nb * (dist.get_world_size(group) - 1))
     info = {"syncs": syncs, "boundary": nb, "nvlink_bytes_per_sync": bytes_per_sync, "exchange": exchange}
     if algo == "scc":
         info["scc_iterations"] = iterations
