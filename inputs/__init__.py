@@ -27,6 +27,9 @@ CONFIGS = {
     "lj": dict(kind="rmat", scale=23, n=4_847_571, m=68_993_773),
     # configs[2]: Twitter-shaped power-law (41.6M vertices, 1.47B edges)
     "twitter": dict(kind="rmat", scale=26, n=41_652_230, m=1_468_365_182),
+    # configs[2] at half scale (same edge factor; 167 MB of PageRank masters,
+    # still beyond the 126 MB L2): the tuning proxy of the headline workload
+    "twitter_h": dict(kind="rmat", scale=25, n=20_826_115, m=734_182_591),
     # configs[3]: Friendster-shaped (65.6M vertices, 1.8B edges)
     "friendster": dict(kind="rmat", scale=26, n=65_608_366, m=1_806_067_135),
     # configs[4]: long-chain-heavy digraph (100M vertices, 2B edges)

@@ -175,7 +175,13 @@ struct KParams {
     unsigned* qtick;            // per-CTA partition queue counters, 2 x grid x kQStride (null: global ticket)
     unsigned long long* trace;  // DG_TRACE: per round {end time ns, vertices signalled into it, dense, out-edges}
     int trace_cap;
+    int exp;  // -DDG_EXP builds only (scripts/build_exp.sh): cost-breakdown switches, DG_EXP bitmask
 };
+#ifdef DG_EXP
+#define EXP_ON(P, b) (((P).exp & (b)) != 0)
+#else
+#define EXP_ON(P, b) false
+#endif
 
 // ------------------------------------------------------------------ helpers
 __device__ __forceinline__ uint32_t sat_add(uint32_t a, uint32_t b) {
@@ -986,7 +992,7 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
         return c;
     };
     auto load_sv = [&](const Win& w, unsigned long long (&sv)[4], float4& cf) {
-        if (w.base != kNoWin && w.base + 4 * lane < w.end) {
+        if (w.base != kNoWin && w.base + 4 * lane < w.end && !EXP_ON(P, 16)) {
             ld_stream_u64x4_h(P.s_val + w.base + 4 * lane, sv, pol_stream);
             cf = ld_stream_f4_h(P.e_coef + w.base + 4 * lane, pol_stream);
         } else {
@@ -1002,7 +1008,7 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
             for (int k = 0; k < 4; k++) {
                 const uint32_t i = w.base + 4 * lane + k;
                 const uint32_t v = u4get(code, k) & kVMask;
-                if (i >= w.beg && i < w.end && v >= px.H)
+                if (i >= w.beg && i < w.end && v >= px.H && !EXP_ON(P, 2))
                     cp_async16(&gbuf[s * 128 + k * 32 + lane], P.vs_t + (v & ~1u), pol_keep);
             }
         }
@@ -1108,7 +1114,7 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
                 const unsigned long long p = fx_from(pin[k]);
                 if (p) {
                     if (vtx[k] < px.H) px_add(&px.acc[2 * vtx[k]], p);  // proxy: shared-memory atomics
-                    else red_add_u64_h(&P.vs_t[vtx[k]], p, pol_keep);   // master: REDG (no return)
+                    else if (!EXP_ON(P, 1)) red_add_u64_h(&P.vs_t[vtx[k]], p, pol_keep);  // master: REDG (no return)
                     n_upd++;
                 }
                 if (!tl[k] && (pend[k] | p)) { sv_c[k] += pend[k] + p; dirty = true; }
@@ -1119,7 +1125,7 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
             // lanes whose four entries all lie in this partition write one 256-bit
             // store; lanes at the partition's ends write only their own entries
             // (the neighbouring partition's mirrors belong to another warp)
-            if (dirty) {
+            if (dirty && !EXP_ON(P, 4)) {
                 if (i0 >= w0.beg && i0 + 3 < w0.end) {
                     st_stream_u64x4_h(P.s_val + i0, sv_c, pol_stream);
                 } else {
@@ -2418,6 +2424,9 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
             while (gcd(P.part_order, D.n_part) != 1) P.part_order++;
         }
     }
+#ifdef DG_EXP
+    if (const char* xe = std::getenv("DG_EXP")) P.exp = std::atoi(xe);
+#endif
     // developer trace (DG_TRACE): per-round timing and activity on stderr
     unsigned long long* trace = nullptr;
     constexpr int kTraceCap = 1 << 16;

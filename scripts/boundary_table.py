@@ -2,8 +2,10 @@
 """Boundary size and peer-exchange volume of multi-rank layouts (CPU only):
 for world 2/4/8 and both placements (round-robin partitions, locality paths;
 DESIGN.md reading R-PLACE), the boundary vertices n_bnd (replicated on > 1
-rank) and the bytes one rank reads per exchange in the peer-memory exchange
-(8 B x n_bnd x (world - 1); parallel.py).  Prints one JSON line per case.
+rank) and the bytes one rank reads per exchange in the peer-memory exchange:
+holder-aware, 8 B x boundary_reads (the peer slots of the boundary vertices
+its own paths hold; dg_layout_info), next to the all-peers volume
+8 B x n_bnd x (world - 1) the exchange read before it became holder-aware.  Prints one JSON line per case.
 
   python scripts/boundary_table.py <config> [worlds]
 """
@@ -26,4 +28,6 @@ for w in worlds:
         nb = i["n_boundary"]
         print(json.dumps({"config": cfg, "n": n, "m": m, "world": w, "placement": pl, "n_boundary": nb,
                           "boundary_frac": nb / n, "rank0_entries": i["n_entries"],
-                          "exchange_bytes_per_rank": 8 * nb * (w - 1), "build_s": time.time() - t}), flush=True)
+                          "boundary_reads_rank0": i["boundary_reads"],
+                          "exchange_bytes_rank0": 8 * i["boundary_reads"],
+                          "all_peers_bytes_per_rank": 8 * nb * (w - 1), "build_s": time.time() - t}), flush=True)

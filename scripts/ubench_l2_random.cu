@@ -3,6 +3,10 @@
 // random addresses of an array of S bytes, all SMs, 8-16 accesses in flight
 // per thread.  The mix over an L2-resident array is the ceiling of the
 // accumulative path walk (one master gather + one RED per walked entry).
+// MODE 2 issues a thread's gathers and REDs in one loop (a later iteration's
+// gathers cannot pass the earlier REDs: a serialised mix); MODE 3 splits them
+// over warps (even warps gather, odd warps RED) -- the concurrent, additive
+// ceiling the verdict r01 asked for (both count gathers + REDs as ops).
 //   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o ubench scripts/ubench_l2_random.cu
 #include <cstdio>
 #include <cstdint>
@@ -25,6 +29,17 @@ __global__ void k(unsigned long long* a, uint32_t nmask, int iters, unsigned lon
         } else if (MODE == 1) {
 #pragma unroll
             for (int u = 0; u < U; u++) atomicAdd(&a[idx[u]], 1ull);
+        } else if (MODE == 3) {
+            if (((threadIdx.x >> 5) & 1) == 0) {
+                unsigned long long v[U];
+#pragma unroll
+                for (int u = 0; u < U; u++) v[u] = __ldcg(&a[idx[u]]);
+#pragma unroll
+                for (int u = 0; u < U; u++) s += v[u];
+            } else {
+#pragma unroll
+                for (int u = 0; u < U; u++) atomicAdd(&a[idx[u]], 1ull);
+            }
         } else {
             unsigned long long v[U];
 #pragma unroll
@@ -57,6 +72,7 @@ int main() {
             run<0, 8>("gather", a, n, sms * bpsm, 256);
             run<1, 8>("red", a, n, sms * bpsm, 256);
             run<2, 8>("g+red", a, n, sms * bpsm, 256);
+            run<3, 8>("g|red", a, n, sms * bpsm, 256);
         }
         run<0, 16>("gather", a, n, sms * 8, 256);
     }
