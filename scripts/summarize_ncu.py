@@ -17,6 +17,10 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "sm__throughput.avg.pct_of_peak_sustained_elapsed"]
 
 
+TIME_TO_MS = {"s": 1e3, "ms": 1.0, "us": 1e-3, "usecond": 1e-3, "msecond": 1.0, "second": 1e3, "ns": 1e-6,
+              "nsecond": 1e-6}
+
+
 def raw(rep):
     out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
@@ -65,7 +69,7 @@ def main():
     tj = os.path.join("profiles", "ncu_traffic.json")
     d = json.load(open(tj)) if os.path.exists(tj) else {}
     d[key] = {"dram_bytes_per_launch": dram, "report": os.path.basename(rep), "summary": name + ".md",
-              "kernel_ms": float(r["gpu__time_duration.sum"][0]) * (1 if r["gpu__time_duration.sum"][1] == "ms" else 1e-3)}
+              "kernel_ms": float(r["gpu__time_duration.sum"][0]) * TIME_TO_MS[r["gpu__time_duration.sum"][1]]}
     json.dump(d, open(tj, "w"), indent=1)
     print("\n".join(lines))
 
