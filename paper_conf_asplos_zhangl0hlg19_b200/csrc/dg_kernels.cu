@@ -30,7 +30,10 @@
 #include <cstdlib>
 #include <cstdio>
 #include <cstring>
+#include <map>
+#include <mutex>
 #include <string>
+#include <tuple>
 
 #include "dg_internal.h"
 
@@ -175,8 +178,10 @@ struct KParams {
     unsigned* qtick;            // per-CTA partition queue counters, 2 x grid x kQStride (null: global ticket)
     unsigned long long* trace;  // DG_TRACE: per round {end time ns, vertices signalled into it, dense, out-edges}
     int trace_cap;
+    unsigned long long* snap;  // DG_EXP 32/64: master snapshots gathered instead of the live masters (2 x n)
     int exp;  // -DDG_EXP builds only (scripts/build_exp.sh): cost-breakdown switches, DG_EXP bitmask
 };
+__device__ int g_exp_par;  // DG_EXP 32/64: the snapshot buffer gathered this round
 #ifdef DG_EXP
 #define EXP_ON(P, b) (((P).exp & (b)) != 0)
 #else
@@ -451,31 +456,14 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
     bool act_c[4], act_n[4];
     uint32_t a_c[4] = {INF, INF, INF, INF}, a_n[4] = {INF, INF, INF, INF};
     bool any_c = probe_finish(wc, code_c, words_c, act_c, a_c);
-    // SSSP: the path-edge weights of an active window are in flight one window ahead
-    auto load_w = [&](const Win& w, bool any) {
-        int4 wv = make_int4(0, 0, 0, 0);
-        if (MODE == 0 && any && w.base + 4 * lane < w.end) wv = ld_stream_i4(P.e_w + w.base + 4 * lane);
-        return wv;
-    };
-    int4 wv_c = load_w(wc, any_c);
     uint32_t carry = INF, carry_vtx = 0;
     bool carry_live = false;
-    // atomicMins in flight from the previous walked window (settled one window later)
-    uint32_t d_old[4] = {0u, 0u, 0u, 0u}, d_val[4] = {0u, 0u, 0u, 0u};
-    unsigned d_mask = 0;
-    auto settle = [&]() {
-#pragma unroll
-        for (int k = 0; k < 4; k++)
-            if (((d_mask >> k) & 1u) && d_val[k] < d_old[k]) acc.upd++;
-        d_mask = 0;
-    };
     while (wc.base != kNoWin) {
         const Win wn3 = win_next(P, wn2, ticket);
         const uint4 code_n3 = load_code(wn3);
         uint4 words_n2;
         probe_words(wn2, code_n2, words_n2);
         const bool any_n = probe_finish(wn, code_n, words_n, act_n, a_n);
-        const int4 wv_n = load_w(wn, any_n);
         if (wc.base == (wc.beg & ~3u)) { carry = INF; carry_live = false; }  // partition start
         const uint32_t i0 = wc.base + 4 * lane;
         // WCC looks one entry ahead: the path edge into the next window is walked backwards too
@@ -502,8 +490,8 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
                     a_c[k] = (i >= wc.beg && i < wc.end) ? P.vs_u[u4get(code_c, k) & kVMask] : INF;
                 }
             }
-            int4 wv = wv_c;
-            if (MODE == 0 && !any_c && i0 < wc.end) wv = ld_stream_i4(P.e_w + i0);  // walked for a carry only
+            int4 wv = make_int4(0, 0, 0, 0);
+            if (MODE == 0 && i0 < wc.end) wv = ld_stream_i4(P.e_w + i0);
             uint32_t vtx[4], a[4], wgt[4];
             bool hd[4], tl[4], live[4];
 #pragma unroll
@@ -569,39 +557,37 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
             // path predecessor of entry 0 (previous lane's last entry, or the carry's vertex)
             uint32_t pred0 = __shfl_up_sync(0xffffffffu, vtx[3], 1);
             if (lane == 0) pred0 = carry_vtx;
-            // the previous window's atomicMin results have had a whole window to
-            // arrive: count its successful updates now
-            settle();
-            // the lane's (up to four) atomicMins are issued back to back; their
-            // results are consumed one window later (settle), so no window waits
-            // for its atomics.  The signal of a lowered vertex is a fire-and-forget
-            // RED issued with the atomic: if another walk lowered the vertex
-            // further in the meantime, that walk signalled it too (a duplicate
-            // signal only re-walks the vertex), and the active counter is an
-            // upper bound, which is all its uses need (non-zero test, sparse
-            // threshold).  The bucket base (vmin) and the carry use the
-            // attempted value: the smallest attempt is the smallest commit.
+            // the lane's (up to four) atomicMins are issued back to back and
+            // are in flight together; their results are consumed afterwards
+            uint32_t old[4];
+#pragma unroll
+            for (int k = 0; k < 4; k++) {
+                old[k] = 0u;
+                if (live[k] && val[k] < a[k] && val[k] <= theta) old[k] = atomicMin(&P.vs_u[vtx[k]], val[k]);
+            }
 #pragma unroll
             for (int k = 0; k < 4; k++) {
                 if (!live[k]) continue;
                 acc.entries++;
                 if (!(u4get(code_c, k) & kHead)) acc.edges++;
-                if (!(val[k] < a[k])) continue;
-                if (val[k] > theta) {
-                    // beyond this round's bucket: not committed; the path
-                    // predecessor stays active so the edge is relaxed again
-                    const uint32_t pv = k ? vtx[k - 1] : pred0;
-                    atomicOr(&bnxt[pv >> 5], 1u << (pv & 31));
-                    acc.sig++;
-                    continue;
+                if (val[k] < a[k]) {
+                    if (val[k] > theta) {
+                        // beyond this round's bucket: not committed; the path
+                        // predecessor stays active so the edge is relaxed again
+                        acc.sig += signal_vertex(bnxt, k ? vtx[k - 1] : pred0);
+                        continue;
+                    }
+                    if (val[k] < old[k]) {
+                        acc.upd++;
+                        if (k == 3) changed3 = true;
+                        // fire-and-forget signal (RED): the active counter may count a
+                        // vertex lowered twice in one round twice -- an upper bound,
+                        // which is all its uses need (non-zero test, sparse threshold)
+                        atomicOr(&bnxt[vtx[k] >> 5], 1u << (vtx[k] & 31));
+                        acc.sig++;
+                        acc.vmin = min(acc.vmin, val[k]);
+                    }
                 }
-                d_old[k] = atomicMin(&P.vs_u[vtx[k]], val[k]);
-                d_val[k] = val[k];
-                d_mask |= 1u << k;
-                atomicOr(&bnxt[vtx[k] >> 5], 1u << (vtx[k] & 31));
-                acc.sig++;
-                acc.vmin = min(acc.vmin, val[k]);
-                if (k == 3) changed3 = true;
             }
             // the carry into the next window is live if the path continues and its
             // last vertex changed now or was signalled (its out-edge must be relaxed)
@@ -617,11 +603,9 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
         code_c = code_n; code_n = code_n2; code_n2 = code_n3;
         words_n = words_n2;
         any_c = any_n;
-        wv_c = wv_n;
 #pragma unroll
         for (int k = 0; k < 4; k++) { act_c[k] = act_n[k]; a_c[k] = a_n[k]; }
     }
-    settle();
 }
 
 // Sparse min-plus rounds (SSSP/BFS, the forward half of WCC, SCC's forward
@@ -1009,7 +993,9 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
                 const uint32_t i = w.base + 4 * lane + k;
                 const uint32_t v = u4get(code, k) & kVMask;
                 if (i >= w.beg && i < w.end && v >= px.H && !EXP_ON(P, 2))
-                    cp_async16(&gbuf[s * 128 + k * 32 + lane], P.vs_t + (v & ~1u), pol_keep);
+                    cp_async16(&gbuf[s * 128 + k * 32 + lane],
+                               (EXP_ON(P, 96) ? P.snap + (size_t)P.n * *(volatile int*)&g_exp_par : P.vs_t) + (v & ~1u),
+                               pol_keep);
             }
         }
         cp_async_commit();
@@ -1521,6 +1507,13 @@ __global__ void __launch_bounds__(NW * 32, MINB) path_kernel(KParams P) {
                 dense = false;
                 walk_sparse_acc<NW>(P, P.occ_items, *((volatile unsigned*)&P.ctr->qcur[cur]), &P.ctr->ticket[cur], bcur, acc);
             } else {
+            if (EXP_ON(P, 96)) {  // DG_EXP 32: gather this round's start snapshot; 64: the previous round's
+                unsigned long long* dst = P.snap + (size_t)P.n * (round & 1);
+                if (blockIdx.x == 0 && threadIdx.x == 0) g_exp_par = EXP_ON(P, 32) ? (round & 1) : ((round + 1) & 1);
+                for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.n + 2; i += (int64_t)gridDim.x * blockDim.x)
+                    dst[i] = __ldcg(&P.vs_t[i]);
+                grid.sync();
+            }
             if (px.H) {  // round-start snapshot of the proxied masters
                 for (int64_t i = threadIdx.x; i < px.H; i += blockDim.x) {
                     px.T[i] = __ldcg(&P.vs_t[i]);
@@ -2222,19 +2215,39 @@ int read_counters(DevWork* W, Counters& c, std::string& err) {
     CK(cudaMemcpy(&c, W->ctr, sizeof(Counters), cudaMemcpyDeviceToHost));
     return DG_OK;
 }
-int write_counters(DevWork* W, const Counters& c, std::string& err) {
-    CK(cudaMemcpy(W->ctr, &c, sizeof(Counters), cudaMemcpyHostToDevice));
+// the counters are set by a one-thread kernel in stream order (the struct
+// travels as a kernel argument): no host synchronisation before the launch
+__global__ void set_counters_kernel(Counters* ctr, Counters c) { *ctr = c; }
+int write_counters(DevWork* W, const Counters& c, std::string& err, RunState* S = nullptr) {
+    set_counters_kernel<<<1, 1>>>(W->ctr, c);
+    CK(cudaGetLastError());
+    if (S) S->stats.kernel_launches++;
     return DG_OK;
 }
 
 int coop_launch(DevWork* W, void* fn, KParams& P, RunState& S, std::string& err, size_t smem = 0,
                 int threads = kBlock) {
-    int dev = 0, sms = 0, per = 0;
+    // grid size per (device, kernel, block, shared memory), queried once:
+    // the occupancy query and the attribute call cost tens of microseconds,
+    // which small graphs (configs[0]: ~0.3 ms per run) would pay every run
+    static std::mutex mu;
+    static std::map<std::tuple<int, void*, int, size_t>, int> grids;
+    int dev = 0;
     CK(cudaGetDevice(&dev));
-    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-    if (smem) CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, threads, smem));
-    const int grid = std::min(sms * std::max(1, per), kMaxGrid);
+    int grid = 0;
+    {
+        std::lock_guard<std::mutex> lk(mu);
+        const auto key = std::make_tuple(dev, fn, threads, smem);
+        auto it = grids.find(key);
+        if (it == grids.end()) {
+            int sms = 0, per = 0;
+            CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+            if (smem) CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, threads, smem));
+            it = grids.emplace(key, std::min(sms * std::max(1, per), kMaxGrid)).first;
+        }
+        grid = it->second;
+    }
     if (P.qtick) CK(cudaMemsetAsync(P.qtick, 0, sizeof(unsigned) * 2 * kMaxGrid * kQStride));
     void* args[] = {&P};
     CK(cudaEventRecord(W->kev0));
@@ -2426,6 +2439,10 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
     }
 #ifdef DG_EXP
     if (const char* xe = std::getenv("DG_EXP")) P.exp = std::atoi(xe);
+    if (P.exp & 96) {
+        CK(cudaMalloc(&P.snap, sizeof(unsigned long long) * 2 * (D.n + 2)));
+        CK(cudaMemset(P.snap, 0, sizeof(unsigned long long) * 2 * (D.n + 2)));
+    }
 #endif
     // developer trace (DG_TRACE): per-round timing and activity on stderr
     unsigned long long* trace = nullptr;
@@ -2436,6 +2453,7 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
         P.trace_cap = kTraceCap;
     }
     int rc = coop_launch(W, fn, P, S, err, smem, accum ? kAccWarps * 32 : kBlock);
+    if (P.snap) cudaFree(P.snap);
     if (trace) {
         std::vector<unsigned long long> h(4 * (size_t)kTraceCap);
         cudaMemcpy(h.data(), trace, sizeof(unsigned long long) * h.size(), cudaMemcpyDeviceToHost);
@@ -2488,7 +2506,7 @@ int init_states(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
             S.stats.kernel_launches += 1;
         }
         CK(cudaGetLastError());
-        return write_counters(W, c, err);
+        return write_counters(W, c, err, &S);
     }
     CK(cudaMemsetAsync(W->bits, 0, sizeof(uint32_t) * 2 * W->nw));
     c.minval[0] = c.minval[1] = INF;
@@ -2520,13 +2538,14 @@ int init_states(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
         S.stats.kernel_launches += 2;
     }
     CK(cudaGetLastError());
-    return write_counters(W, c, err);
+    return write_counters(W, c, err, &S);
 }
 
-int collect_stats(DevWork* W, RunState& S, std::string& err) {
+int collect_stats(DevWork* W, RunState& S, std::string& err, Counters* out = nullptr) {
     Counters c;
     int rc;
     if ((rc = read_counters(W, c, err))) return rc;
+    if (out) *out = c;
     S.stats.rounds += c.round - (int)S.round;
     S.round = c.round;
     S.stats.vertex_updates = (int64_t)c.updates;
@@ -2564,7 +2583,7 @@ int run_scc(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, std
         scc_bits_kernel<<<grid_1d(W->nw), 256>>>(W->scc_label, D.n, W->bits, W->nw);
         Counters c0{};
         c0.active[0] = (unsigned)rem;
-        if ((rc = write_counters(W, c0, err))) return rc;
+        if ((rc = write_counters(W, c0, err, &S))) return rc;
         S.stats.kernel_launches += 2;
         if ((rc = launch_path(W, D, 100, rounds, S, err))) return rc;
         Counters c1;
@@ -2576,7 +2595,7 @@ int run_scc(DevWork* W, const DevLayout& D, RunState& S, int64_t max_rounds, std
         // backward reachability from the roots within their colours
         CK(cudaMemsetAsync(W->bits, 0, sizeof(uint32_t) * 2 * W->nw));
         Counters c2{};
-        if ((rc = write_counters(W, c2, err))) return rc;
+        if ((rc = write_counters(W, c2, err, &S))) return rc;
         scc_roots_kernel<<<g, 256>>>(W->vs_u, W->scc_label, D.orig, W->scc_mark, D.n, W->bits, W->ctr);
         S.stats.kernel_launches += 1;
         if ((rc = launch_path(W, D, 101, rounds, S, err))) return rc;
@@ -2807,9 +2826,8 @@ int dev_run(DevWork*& W, const DevLayout& D, RunState& S, int64_t max_rounds, st
     CK(cudaEventElapsedTime(&ms, W->ev0, W->ev1));
     S.stats.time_ms = ms;
     if (S.algo != DG_SCC) {
-        if ((rc = collect_stats(W, S, err))) return rc;
         Counters c;
-        if ((rc = read_counters(W, c, err))) return rc;
+        if ((rc = collect_stats(W, S, err, &c))) return rc;
         if (c.active[c.round & 1] != 0) {
             err = "max_rounds reached before convergence";
             return DG_ENOCONV;
