@@ -174,6 +174,10 @@ struct KParams {
     uint32_t sparse_max;      // rounds with at most this many signalled vertices are candidates (n/4)
     uint32_t sparse_occ;      // ... and are walked sparse if their out-edges are at most this many
     int sparse_walk;          // path edges a sparse walk follows at most
+    uint32_t probe_free_occ;  // min-plus dense rounds whose signalled vertices own at least this many
+                              // out-edges (or that signal more than sparse_max vertices) walk every
+                              // window without probing the bitmap (0: always probe)
+    uint32_t probe_free_act;  // ... or that signalled more than this many vertices (n/4)
     MultiRank mr;             // world > 1: fused multi-rank run
     unsigned* qtick;            // per-CTA partition queue counters, 2 x grid x kQStride (null: global ticket)
     unsigned long long* trace;  // DG_TRACE: per round {end time ns, vertices signalled into it, dense, out-edges}
@@ -395,6 +399,42 @@ __device__ __forceinline__ Win win_next(const KParams& P, const Win& w, const Qu
     return win_first_of(P, q);
 }
 
+// A warp's partition feed (both dense walks): with the global ticket
+// (default) the ticket of the partition after next and the bounds of the next
+// partition are fetched one partition early, so a partition switch waits for
+// no atomic or load.  With per-CTA queues (DG_DISPATCH=1) the switch takes
+// the next partition synchronously.
+struct Feed {
+    unsigned t_pend;     // lane 0: ticket taken for the partition after next
+    uint32_t nbeg, nend; // bounds of the next partition (nbeg == kNoWin: none)
+};
+__device__ __forceinline__ unsigned map_order(const KParams& P, unsigned t) {
+    if (P.part_order == 1) return (unsigned)P.n_part - 1 - t;  // developer knob: dispatch-order experiments
+    if (P.part_order > 1) return (unsigned)(((unsigned long long)t * P.part_order) % (unsigned long long)P.n_part);
+    return t;
+}
+__device__ __forceinline__ void feed_fetch(const KParams& P, const Queue& q, Feed& f) {
+    // the pending ticket becomes the next partition; a new ticket is taken
+    const unsigned t = __shfl_sync(0xffffffffu, f.t_pend, 0);
+    if (t < (unsigned)P.n_part) {
+        const unsigned u = map_order(P, t);
+        f.nbeg = (uint32_t)P.part_off[u];
+        f.nend = (uint32_t)P.part_off[u + 1];
+    } else {
+        f.nbeg = kNoWin;
+        f.nend = 0;
+    }
+    if ((threadIdx.x & 31) == 0) f.t_pend = atomicAdd(q.global, 1u);
+}
+__device__ __forceinline__ Win feed_next(const KParams& P, const Queue& q, const Win& w, Feed& f) {
+    if (w.base == kNoWin) return w;
+    if (w.base + 128 < w.end) return Win{w.base + 128, w.beg, w.end};
+    if (q.qt) return win_first_of(P, q);
+    const Win nw = f.nbeg == kNoWin ? Win{kNoWin, 0, 0} : Win{f.nbeg & ~3u, f.nbeg, f.nend};
+    if (nw.base != kNoWin) feed_fetch(P, q, f);
+    return nw;
+}
+
 // Min-plus walk.  MODE 0 SSSP (weights), 1 BFS (unit weights), 2 WCC (weight 0,
 // also backward along every path edge), 3 SCC forward colouring (weight 0,
 // assigned vertices -- scc_label >= 0 -- break their paths).
@@ -405,7 +445,7 @@ __device__ __forceinline__ Win win_next(const KParams& P, const Win& w, const Qu
 // authority), as are the indices of window w+2.
 template <int MODE>
 __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32_t* bcur, uint32_t* bnxt,
-                             uint32_t theta, Acc& acc) {
+                             uint32_t theta, Acc& acc, bool all) {
     const int lane = threadIdx.x & 31;
     const uint4 kFill = make_uint4(kHead | kTail, kHead | kTail, kHead | kTail, kHead | kTail);
     auto load_code = [&](const Win& w) {
@@ -414,9 +454,19 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
         return c;
     };
     // signal-bitmap words of a window's entries (issued two windows ahead)
+    // (a round that signalled most vertices -- `all` -- treats every entry as
+    // signalled: every window would be walked anyway, and the probes are one
+    // random L2 access per entry; walking an unsignalled vertex's edges only
+    // repeats relaxations that cannot improve)
     auto probe_words = [&](const Win& w, const uint4& code, uint4& words) {
         words = make_uint4(0u, 0u, 0u, 0u);
         if (w.base == kNoWin) return;
+        if (all) {
+            const uint32_t i = w.base + 4 * lane;
+            words = make_uint4(i >= w.beg && i < w.end ? ~0u : 0u, i + 1 >= w.beg && i + 1 < w.end ? ~0u : 0u,
+                               i + 2 >= w.beg && i + 2 < w.end ? ~0u : 0u, i + 3 >= w.beg && i + 3 < w.end ? ~0u : 0u);
+            return;
+        }
 #pragma unroll
         for (int k = 0; k < 4; k++) {
             const uint32_t i = w.base + 4 * lane + k;
@@ -445,10 +495,15 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
     };
 
     // pipeline: indices three windows ahead, bitmap words two ahead, masters one ahead
+    Feed f{0u, kNoWin, 0u};
     Win wc = win_first_of(P, ticket);
     if (wc.base == kNoWin) return;
-    Win wn = win_next(P, wc, ticket);
-    Win wn2 = win_next(P, wn, ticket);
+    if (!ticket.qt) {  // prime the feed: next partition's bounds and the ticket after it
+        if (lane == 0) f.t_pend = atomicAdd(ticket.global, 1u);
+        feed_fetch(P, ticket, f);
+    }
+    Win wn = feed_next(P, ticket, wc, f);
+    Win wn2 = feed_next(P, ticket, wn, f);
     uint4 code_c = load_code(wc), code_n = load_code(wn), code_n2 = load_code(wn2);
     uint4 words_c, words_n;
     probe_words(wc, code_c, words_c);
@@ -459,7 +514,7 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
     uint32_t carry = INF, carry_vtx = 0;
     bool carry_live = false;
     while (wc.base != kNoWin) {
-        const Win wn3 = win_next(P, wn2, ticket);
+        const Win wn3 = feed_next(P, ticket, wn2, f);
         const uint4 code_n3 = load_code(wn3);
         uint4 words_n2;
         probe_words(wn2, code_n2, words_n2);
@@ -918,42 +973,6 @@ __device__ __forceinline__ void px_refresh(const KParams& P, const Proxies& px) 
     }
 }
 
-// A warp's partition feed for the accumulative walk: with the global ticket
-// (default) the ticket of the partition after next and the bounds of the next
-// partition are fetched one partition early, so a partition switch waits for
-// no atomic or load.  With per-CTA queues (DG_DISPATCH=1) the switch takes
-// the next partition synchronously.
-struct Feed {
-    unsigned t_pend;     // lane 0: ticket taken for the partition after next
-    uint32_t nbeg, nend; // bounds of the next partition (nbeg == kNoWin: none)
-};
-__device__ __forceinline__ unsigned map_order(const KParams& P, unsigned t) {
-    if (P.part_order == 1) return (unsigned)P.n_part - 1 - t;  // developer knob: dispatch-order experiments
-    if (P.part_order > 1) return (unsigned)(((unsigned long long)t * P.part_order) % (unsigned long long)P.n_part);
-    return t;
-}
-__device__ __forceinline__ void feed_fetch(const KParams& P, const Queue& q, Feed& f) {
-    // the pending ticket becomes the next partition; a new ticket is taken
-    const unsigned t = __shfl_sync(0xffffffffu, f.t_pend, 0);
-    if (t < (unsigned)P.n_part) {
-        const unsigned u = map_order(P, t);
-        f.nbeg = (uint32_t)P.part_off[u];
-        f.nend = (uint32_t)P.part_off[u + 1];
-    } else {
-        f.nbeg = kNoWin;
-        f.nend = 0;
-    }
-    if ((threadIdx.x & 31) == 0) f.t_pend = atomicAdd(q.global, 1u);
-}
-__device__ __forceinline__ Win feed_next(const KParams& P, const Queue& q, const Win& w, Feed& f) {
-    if (w.base == kNoWin) return w;
-    if (w.base + 128 < w.end) return Win{w.base + 128, w.beg, w.end};
-    if (q.qt) return win_first_of(P, q);
-    const Win nw = f.nbeg == kNoWin ? Win{kNoWin, 0, 0} : Win{f.nbeg & ~3u, f.nbeg, f.nend};
-    if (nw.base != kNoWin) feed_fetch(P, q, f);
-    return nw;
-}
-
 // Walk all windows the warp obtains in this round.  Software pipeline over the
 // window stream (kRing-slot shared ring per warp): while window w is walked,
 // the master totals of windows w+1 and w+2 are in flight into shared memory
@@ -985,16 +1004,18 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
         }
     };
     // masters of a window into ring slot s: entry 4*lane+k -> gbuf[s*128 + k*32 + lane]
-    // (16-byte aligned pair {T[v & ~1], T[v | 1]}); proxies and invalid entries skip
+    // (16-byte aligned pair {T[v & ~1], T[v | 1]}); proxies, tails (no out-edge:
+    // nothing pending to forward) and invalid entries skip
     auto gather = [&](const Win& w, const uint4& code, int s) {
         if (w.base != kNoWin) {
 #pragma unroll
             for (int k = 0; k < 4; k++) {
                 const uint32_t i = w.base + 4 * lane + k;
-                const uint32_t v = u4get(code, k) & kVMask;
-                if (i >= w.beg && i < w.end && v >= px.H && !EXP_ON(P, 2))
+                const uint32_t c = u4get(code, k);
+                const uint32_t v = c & kVMask;
+                if (i >= w.beg && i < w.end && v >= px.H && !(c & kTail) && !EXP_ON(P, 2))
                     cp_async16(&gbuf[s * 128 + k * 32 + lane],
-                               (EXP_ON(P, 96) ? P.snap + (size_t)P.n * *(volatile int*)&g_exp_par : P.vs_t) + (v & ~1u),
+                               (EXP_ON(P, 96) ? P.snap + (size_t)((P.n + 3) & ~1ll) * *(volatile int*)&g_exp_par : P.vs_t) + (v & ~1u),
                                pol_keep);
             }
         }
@@ -1508,7 +1529,7 @@ __global__ void __launch_bounds__(NW * 32, MINB) path_kernel(KParams P) {
                 walk_sparse_acc<NW>(P, P.occ_items, *((volatile unsigned*)&P.ctr->qcur[cur]), &P.ctr->ticket[cur], bcur, acc);
             } else {
             if (EXP_ON(P, 96)) {  // DG_EXP 32: gather this round's start snapshot; 64: the previous round's
-                unsigned long long* dst = P.snap + (size_t)P.n * (round & 1);
+                unsigned long long* dst = P.snap + (size_t)((P.n + 3) & ~1ll) * (round & 1);
                 if (blockIdx.x == 0 && threadIdx.x == 0) g_exp_par = EXP_ON(P, 32) ? (round & 1) : ((round + 1) & 1);
                 for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.n + 2; i += (int64_t)gridDim.x * blockDim.x)
                     dst[i] = __ldcg(&P.vs_t[i]);
@@ -1540,14 +1561,21 @@ __global__ void __launch_bounds__(NW * 32, MINB) path_kernel(KParams P) {
             // signalled, compact them; walk from them if their out-edges are
             // at most 1/sparse_div of the path entries, else walk the windows
             const bool sparse = (ALGO == DG_SSSP || ALGO == DG_BFS || ALGO == 100) && sparse_round(P, grid, cur, bcur);
+            // probe-free dense round: most vertices signalled, or the signalled
+            // ones own most out-edges (counted by sparse_round)
+            const unsigned nact = *((volatile unsigned*)&P.ctr->active[cur]);
+            const bool all = P.probe_free_occ &&
+                             (nact > P.probe_free_act ||
+                              (P.occ_off && (ALGO == DG_SSSP || ALGO == DG_BFS || ALGO == 100) &&
+                               *((volatile unsigned*)&P.ctr->osum[cur]) >= P.probe_free_occ));
             if (sparse) {
                 dense = false;
                 const unsigned qn = *((volatile unsigned*)&P.ctr->qcur[cur]);
                 if (ALGO == DG_SSSP) walk_sparse<0>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
                 else if (ALGO == DG_BFS) walk_sparse<1>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
                 else walk_sparse<3>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
-            } else if (ALGO == DG_SSSP) walk_minplus<0>(P, dq, bcur, bnxt, theta, acc);
-            else if (ALGO == DG_BFS) walk_minplus<1>(P, dq, bcur, bnxt, theta, acc);
+            } else if (ALGO == DG_SSSP) walk_minplus<0>(P, dq, bcur, bnxt, theta, acc, all);
+            else if (ALGO == DG_BFS) walk_minplus<1>(P, dq, bcur, bnxt, theta, acc, all);
             else if (ALGO == DG_WCC) {
                 // sparse WCC round: labels go forward along the out-edges, then
                 // backward along the in-edges of the signalled vertices
@@ -1571,10 +1599,10 @@ __global__ void __launch_bounds__(NW * 32, MINB) path_kernel(KParams P) {
                     walk_sparse_bwd<true>(P, P.iocc_off, P.iocc, P.occ_items, *((volatile unsigned*)&P.ctr->qn_in[cur]),
                                           &P.ctr->ticket_in[cur], bnxt, acc);
                 } else {
-                    walk_minplus<2>(P, dq, bcur, bnxt, INF, acc);
+                    walk_minplus<2>(P, dq, bcur, bnxt, INF, acc, all);
                 }
             }
-            else if (ALGO == 100) walk_minplus<3>(P, dq, bcur, bnxt, INF, acc);
+            else if (ALGO == 100) walk_minplus<3>(P, dq, bcur, bnxt, INF, acc, all);
             else if (ALGO == 101 && sparse_round(P, grid, cur, bcur)) {
                 // sparse backward round (same decision as the forward rounds)
                 dense = false;
@@ -2230,19 +2258,28 @@ int coop_launch(DevWork* W, void* fn, KParams& P, RunState& S, std::string& err,
     // grid size per (device, kernel, block, shared memory), queried once:
     // the occupancy query and the attribute call cost tens of microseconds,
     // which small graphs (configs[0]: ~0.3 ms per run) would pay every run
+    // (the dynamic shared-memory attribute is per kernel: it is set again
+    // whenever a launch of that kernel asks for a different size)
     static std::mutex mu;
     static std::map<std::tuple<int, void*, int, size_t>, int> grids;
+    static std::map<std::pair<int, void*>, size_t> smem_attr;
     int dev = 0;
     CK(cudaGetDevice(&dev));
     int grid = 0;
     {
         std::lock_guard<std::mutex> lk(mu);
+        if (smem) {
+            auto a = smem_attr.find({dev, fn});
+            if (a == smem_attr.end() || a->second != smem) {
+                CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+                smem_attr[{dev, fn}] = smem;
+            }
+        }
         const auto key = std::make_tuple(dev, fn, threads, smem);
         auto it = grids.find(key);
         if (it == grids.end()) {
             int sms = 0, per = 0;
             CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
-            if (smem) CK(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
             CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, threads, smem));
             it = grids.emplace(key, std::min(sms * std::max(1, per), kMaxGrid)).first;
         }
@@ -2428,6 +2465,11 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
             const char* sw = std::getenv("DG_SPARSE_WALK");  // developer knob
             P.sparse_walk = sw ? std::max(1, std::atoi(sw)) : 4;
         }
+        {
+            const char* pf = std::getenv("DG_PROBE_FREE");  // developer knob: 0 = always probe
+            P.probe_free_occ = (pf && std::atoi(pf) == 0) ? 0u : (uint32_t)std::min<int64_t>(std::max<int64_t>(D.M / 4, 1), 0xFFFFFFFFll);
+            P.probe_free_act = (uint32_t)std::min<int64_t>(D.n / 4, 0xFFFFFFFFll);
+        }
         const char* hm = std::getenv("DG_HOT_MASTER_MB");  // developer knob (default 64 MB)
         P.hot_master_bytes = (uint64_t)(hm ? std::atof(hm) : 64.0) * (1ull << 20);
         const char* o = std::getenv("DG_PART_ORDER");
@@ -2440,8 +2482,8 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
 #ifdef DG_EXP
     if (const char* xe = std::getenv("DG_EXP")) P.exp = std::atoi(xe);
     if (P.exp & 96) {
-        CK(cudaMalloc(&P.snap, sizeof(unsigned long long) * 2 * (D.n + 2)));
-        CK(cudaMemset(P.snap, 0, sizeof(unsigned long long) * 2 * (D.n + 2)));
+        CK(cudaMalloc(&P.snap, sizeof(unsigned long long) * 2 * (D.n + 4)));
+        CK(cudaMemset(P.snap, 0, sizeof(unsigned long long) * 2 * (D.n + 4)));
     }
 #endif
     // developer trace (DG_TRACE): per-round timing and activity on stderr
