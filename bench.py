@@ -312,6 +312,9 @@ def main():
     ap.add_argument("--l2-flush-mb", type=int, default=512)
     ap.add_argument("--no-extras", action="store_true", help="skip ablation/e2e/cpu baseline/sssp (profiling runs)")
     ap.add_argument("--no-sssp", action="store_true", help="skip the SSSP record of the default PageRank line")
+    ap.add_argument("--layout-cache", default=None,
+                    help="N=1 profiling runs only: load the layout from this file if it exists, else build it and "
+                         "save it there (a loaded layout has no CSR, so use with --no-extras)")
     args = ap.parse_args()
     if args.config is None:
         args.config = DEFAULT_CONFIG[args.algo]
@@ -338,7 +341,12 @@ def main():
     dg = DiGraph(device=local)
     t_gen = t_load = t_pre = 0.0
     gname = f"{args.config}-seed{args.seed}"
-    if world == 1:
+    if world == 1 and args.layout_cache and os.path.exists(args.layout_cache):
+        t0 = time.time()
+        dg.load_layout(args.layout_cache)
+        t_load = time.time() - t0
+        gname = f"{args.config}-seed{args.seed} (layout file)"
+    elif world == 1:
         t0 = time.time()
         g = inputs.make(args.config, seed=args.seed)
         t_gen = time.time() - t0
@@ -350,6 +358,11 @@ def main():
         t0 = time.time()
         dg.build_paths(**bp)
         t_pre = time.time() - t0
+        if args.layout_cache:
+            try:
+                dg.save_layout(args.layout_cache)
+            except Exception as e:  # a profiling convenience only
+                log(f"[bench] layout cache not written: {e}")
     else:
         # preprocess ONCE (rank 0) and hand every rank its share through layout
         # files (dg_build_paths_shared / dg_load_layout):

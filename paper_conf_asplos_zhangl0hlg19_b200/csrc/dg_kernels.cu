@@ -95,6 +95,9 @@ struct DevWork {
     int64_t nw = 0;
     int32_t* vlist[2] = {nullptr, nullptr};  // ablation frontiers
     Counters* ctr = nullptr;
+    Counters* ctr_host = nullptr;          // mapped pinned mirror the path kernel writes at its end
+    Counters* ctr_host_dev = nullptr;      // ... its device address
+    bool ctr_mirror_fresh = false;         // the mirror holds the counters of the last path launch
     double* dsum = nullptr;
     int32_t* scc_label = nullptr;
     uint8_t* scc_mark = nullptr;
@@ -183,6 +186,7 @@ struct KParams {
     unsigned long long* trace;  // DG_TRACE: per round {end time ns, vertices signalled into it, dense, out-edges}
     int trace_cap;
     unsigned long long* snap;  // DG_EXP 32/64: master snapshots gathered instead of the live masters (2 x n)
+    Counters* ctr_out;  // mapped host mirror of *ctr written at the end of the launch (null: none)
     int exp;  // -DDG_EXP builds only (scripts/build_exp.sh): cost-breakdown switches, DG_EXP bitmask
 };
 __device__ int g_exp_par;  // DG_EXP 32/64: the snapshot buffer gathered this round
@@ -1684,6 +1688,12 @@ __global__ void __launch_bounds__(NW * 32, MINB) path_kernel(KParams P) {
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         P.ctr->round += r;
         P.ctr->mr_ex = ex;
+        if (P.ctr_out) {  // the host reads the counters without a copy call after the launch
+            const unsigned* src = reinterpret_cast<const unsigned*>(P.ctr);
+            volatile unsigned* dst = reinterpret_cast<volatile unsigned*>(P.ctr_out);
+            for (size_t k = 0; k < sizeof(Counters) / 4; k++) dst[k] = __ldcg(src + k);  // L2: other blocks' atomics
+            __threadfence_system();
+        }
     }
 }
 
@@ -2229,6 +2239,12 @@ int ensure_work(DevWork*& W, const DevLayout& D, std::string& err) {
     if ((rc = dalloc(&W->vlist[0], D.n + 1, bytes, err))) return rc;
     if ((rc = dalloc(&W->vlist[1], D.n + 1, bytes, err))) return rc;
     if ((rc = dalloc(&W->ctr, 1, bytes, err))) return rc;
+    if (cudaHostAlloc(&W->ctr_host, sizeof(Counters), cudaHostAllocMapped) != cudaSuccess ||
+        cudaHostGetDevicePointer(&W->ctr_host_dev, W->ctr_host, 0) != cudaSuccess) {
+        if (W->ctr_host) cudaFreeHost(W->ctr_host);
+        W->ctr_host = W->ctr_host_dev = nullptr;  // optional: counters are then copied back
+        cudaGetLastError();
+    }
     if ((rc = dalloc(&W->dsum, 1, bytes, err))) return rc;
     if ((rc = dalloc(&W->qtick, 2 * kMaxGrid * kQStride, bytes, err))) return rc;
     CK(cudaMemset(W->s_val, 0, sizeof(unsigned long long) * (D.M + kPad)));
@@ -2494,7 +2510,10 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
         P.trace = trace;
         P.trace_cap = kTraceCap;
     }
+    P.ctr_out = mr ? nullptr : W->ctr_host_dev;
+    W->ctr_mirror_fresh = false;
     int rc = coop_launch(W, fn, P, S, err, smem, accum ? kAccWarps * 32 : kBlock);
+    if (!rc && P.ctr_out) W->ctr_mirror_fresh = true;
     if (P.snap) cudaFree(P.snap);
     if (trace) {
         std::vector<unsigned long long> h(4 * (size_t)kTraceCap);
@@ -2583,10 +2602,15 @@ int init_states(DevWork* W, const DevLayout& D, RunState& S, std::string& err) {
     return write_counters(W, c, err, &S);
 }
 
-int collect_stats(DevWork* W, RunState& S, std::string& err, Counters* out = nullptr) {
+int collect_stats(DevWork* W, RunState& S, std::string& err, Counters* out = nullptr, bool mirror = false) {
     Counters c;
     int rc;
-    if ((rc = read_counters(W, c, err))) return rc;
+    if (mirror && W->ctr_mirror_fresh && W->ctr_host) {  // written by the path kernel that just completed
+        std::memcpy(&c, (const void*)W->ctr_host, sizeof(Counters));
+        W->ctr_mirror_fresh = false;
+    } else if ((rc = read_counters(W, c, err))) {
+        return rc;
+    }
     if (out) *out = c;
     S.stats.rounds += c.round - (int)S.round;
     S.round = c.round;
@@ -2798,6 +2822,8 @@ void dev_free_work(DevWork*& W) {
     if (!W) return;
     dfree(W->vs_u); dfree(W->vstamp); dfree(W->vs_f); dfree(W->vs_t); dfree(W->sigma); dfree(W->s_val); dfree(W->bnd_base);
     dfree(W->e_coef); dfree(W->pr_coef); dfree(W->ads_base); dfree(W->bits); dfree(W->vlist[0]); dfree(W->vlist[1]);
+    if (W->ctr_host) cudaFreeHost(W->ctr_host);
+    W->ctr_host = W->ctr_host_dev = nullptr;
     dfree(W->ctr); dfree(W->dsum); dfree(W->qtick); dfree(W->scc_label); dfree(W->scc_mark); dfree(W->remaining); dfree(W->out_stage);
     dfree(W->occ_off); dfree(W->occ); dfree(W->occ_items); dfree(W->iocc_off); dfree(W->iocc); dfree(W->occ_cur);
     if (W->cub_tmp) cudaFree(W->cub_tmp);
@@ -2869,7 +2895,8 @@ int dev_run(DevWork*& W, const DevLayout& D, RunState& S, int64_t max_rounds, st
     S.stats.time_ms = ms;
     if (S.algo != DG_SCC) {
         Counters c;
-        if ((rc = collect_stats(W, S, err, &c))) return rc;
+        // the mirror is valid only right after a single-rank path launch of this run
+        if ((rc = collect_stats(W, S, err, &c, S.mode != DG_MODE_VERTEX))) return rc;
         if (c.active[c.round & 1] != 0) {
             err = "max_rounds reached before convergence";
             return DG_ENOCONV;
