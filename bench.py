@@ -169,7 +169,7 @@ def load_ncu(algo, config):
         return None
 
 
-def roofline(algo, config, st, n, M, mode):
+def roofline(algo, config, st, n, M, mode, hub_frac=None):
     """`roofline` of the dominant kernel: compulsory bytes / CUDA-event time of
     this run's launch (`achieved`), against the measured HBM copy bandwidth;
     `traffic` and `hbm_measured` from the committed ncu capture (what the
@@ -188,10 +188,17 @@ def roofline(algo, config, st, n, M, mode):
         gbs = nc["dram_bytes_per_launch"] / (nc["kernel_ms"] / 1e3) / 1e9
         roof["hbm_measured"] = {"dram_bytes": nc["dram_bytes_per_launch"], "ncu_kernel_ms": nc["kernel_ms"],
                                 "gbs": gbs, "frac": gbs / peak, "report": nc.get("summary")}
-    # the L2 side: random master operations per second (one gather per
-    # walked non-proxy entry, one RED / atomicMin per update)
+    # the L2 side: random master operations per second -- one gather per
+    # walked entry, one RED / atomicMin per update; for PageRank/Adsorption
+    # the hub entries (shared-memory proxies) are not L2 operations: both
+    # counts are scaled by the non-hub share of the layout's entries
     ops = st["entries_processed"] + st["vertex_updates"]
+    if algo in ("pagerank", "adsorption") and hub_frac is not None:
+        ops *= 1.0 - hub_frac
+        roof["hub_entry_share"] = hub_frac
     roof["l2_random_ops_per_s"] = ops / (kms / 1e3) if kms > 0 else 0.0
+    roof["l2_mix_ceiling_ops_per_s"] = 145e9
+    roof["l2_mix_ceiling_source"] = "scripts/ubench_l2_random.cu, profiles/r02d_l2_random_ubench.txt (gather/RED mix)"
     return roof
 
 
@@ -415,7 +422,8 @@ def main():
     ms = float(ms_t.item())
     kernel_ms = sum(s["kernel_ms"] for s in stats) / len(stats)
     st0 = stats[-1]
-    roof = roofline(args.algo, args.config, st0, n, M, args.mode)
+    hub_frac = info["hub_entries"] / M if M else None
+    roof = roofline(args.algo, args.config, st0, n, M, args.mode, hub_frac)
     roof["kernel_share_of_step"] = kernel_ms / ms if ms else None
 
     extras = {}

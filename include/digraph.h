@@ -122,6 +122,8 @@ typedef struct {
     int64_t boundary_reads;       /* peer slots this rank reads per peer-memory exchange:
                                      sum over the boundary vertices its paths hold of
                                      (ranks holding the vertex - 1); x 8 B = NVLink bytes */
+    int64_t hub_entries;          /* path entries of the n_proxy highest-degree vertices
+                                     (the shared-memory proxies of PageRank/Adsorption) */
 } dg_layout_info;
 
 /* Create an empty graph bound to CUDA device `device` (cudaSetDevice is

@@ -55,7 +55,8 @@ class dg_layout_info(ctypes.Structure):
                 ("n_dep_sccs", ctypes.c_int64), ("giant_scc_paths", ctypes.c_int64),
                 ("n_boundary", ctypes.c_int64), ("paths_before_merge", ctypes.c_int64),
                 ("preprocess_ms", ctypes.c_double), ("device_bytes", ctypes.c_int64),
-                ("h2d_bytes", ctypes.c_int64), ("boundary_reads", ctypes.c_int64)]
+                ("h2d_bytes", ctypes.c_int64), ("boundary_reads", ctypes.c_int64),
+                ("hub_entries", ctypes.c_int64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -381,6 +381,15 @@ int dg_get_layout_info(const dg_graph* g, dg_layout_info* info) {
     const int rk = L.params.rank;
     for (const uint64_t h : L.bnd_hold)
         if ((h >> rk) & 1ull) info->boundary_reads += __builtin_popcountll(h) - 1;
+    if (L.hub_entries < 0) {
+        const uint32_t H = (uint32_t)std::max<int64_t>(0, L.n_proxy);
+        const int64_t M = (int64_t)L.e_idx.size();
+        int64_t c = 0;
+#pragma omp parallel for reduction(+ : c) schedule(static)
+        for (int64_t k = 0; k < M; k++) c += (L.e_idx[k] & dg::kVMask) < H;
+        L.hub_entries = c;
+    }
+    info->hub_entries = L.hub_entries;
     return DG_OK;
 }
 

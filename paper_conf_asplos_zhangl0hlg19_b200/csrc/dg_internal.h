@@ -31,6 +31,7 @@ struct HostCSR {
 // Host copy of the built layout (one rank's share).
 struct HostLayout {
     bool built = false;
+    mutable int64_t hub_entries = -1;   // entries of vertices [0, n_proxy), counted on first request
     dg_path_params params{};
     // paths of this rank in priority order
     std::vector<int64_t> path_off;      // n_paths+1, into entries
