@@ -23,7 +23,6 @@
 // the run ends when a round signals no vertex (device-side active counter,
 // north_star (4)).
 #include <cooperative_groups.h>
-#include <cooperative_groups/scan.h>
 #include <cub/device/device_scan.cuh>
 #include <cuda_runtime.h>
 
@@ -78,7 +77,6 @@ struct Counters {
     unsigned long long mr_ex;     // exchanges done by the last launch
     unsigned long long mr_err;    // a peer did not arrive (timeout)
     unsigned long long dense_rounds;  // rounds that streamed every window's path entries (not sparse)
-    unsigned long long fl_cnt[2];     // SSSP/BFS frontier list k: (out-edges << 32) | items appended
 };
 
 struct DevWork {
@@ -109,7 +107,6 @@ struct DevWork {
     uint32_t* occ_off = nullptr;           // vertex -> its non-tail path entries (sparse rounds), n+1
     uint32_t* occ = nullptr;               // entry indices grouped by vertex
     uint2* occ_items = nullptr;            // frontier items (v, chunk of <= kOccChunk occurrences)
-    uint2* flist[2] = {nullptr, nullptr};  // SSSP/BFS: next round's frontier items appended by sparse walks
     uint32_t* iocc_off = nullptr;          // vertex -> its non-head path entries (SCC backward), n+1
     uint32_t* iocc = nullptr;
     bool iocc_ok = false;
@@ -175,8 +172,6 @@ struct KParams {
     const uint32_t* occ_off;  // SSSP/BFS sparse rounds: occurrence index (null: dense rounds only)
     const uint32_t* occ;
     uint2* occ_items;         // the round's frontier items (v, chunk)
-    uint2* flist0;            // SSSP/BFS frontier lists (by bitmap parity; null: not used)
-    uint2* flist1;
     const uint32_t* iocc_off;  // WCC: the in-edge occurrence index as well
     const uint32_t* iocc;
     uint32_t sparse_max;      // rounds with at most this many signalled vertices are candidates (n/4)
@@ -761,34 +756,10 @@ __device__ bool sparse_round(const KParams& P, cg::grid_group& grid, int cur, co
     return true;
 }
 
-// A vertex signalled for the first time in this round (its bit set by this
-// call) is appended to the next round's frontier list as max(1, ceil(d/32))
-// items (d = its out-occurrences; a vertex without any still gets one empty
-// item, so the list names every set bit and the round that consumes it can
-// clear exactly those words).  Appends are aggregated over the lanes that
-// take them together: one 64-bit atomic adds (out-edges << 32) | items.
-__device__ __forceinline__ void flist_append(const KParams& P, uint2* fl, unsigned long long* fcnt, uint32_t u) {
-    const uint32_t d = P.occ_off[u + 1] - P.occ_off[u];
-    const uint32_t nch = d ? (d + kOccChunk - 1) / kOccChunk : 1u;
-    cg::coalesced_group g = cg::coalesced_threads();
-    const unsigned long long val = ((unsigned long long)d << 32) | nch;
-    const unsigned long long incl = cg::inclusive_scan(g, val);
-    unsigned long long base = 0;
-    if (g.thread_rank() == g.size() - 1) base = atomicAdd(fcnt, incl);
-    base = g.shfl(base, g.size() - 1);
-    const uint32_t at = (uint32_t)(base + incl - val);  // low half: items before this lane's
-    for (uint32_t k = 0; k < nch; k++) fl[at + k] = make_uint2(u, k);
-}
-__device__ __forceinline__ bool signal_append(const KParams& P, uint32_t* bnxt, uint2* fl, unsigned long long* fcnt,
-                                              uint32_t u) {
-    const bool first = signal_vertex(bnxt, u);
-    if (first && fl) flist_append(P, fl, fcnt, u);
-    return first;
-}
 template <int MODE>
 __device__ void walk_sparse(const KParams& P, const uint32_t* off, const uint32_t* occ, const uint2* list, unsigned qn,
                             unsigned* ticket, uint32_t* bnxt,
-                            uint32_t theta, Acc& acc, uint2* fl = nullptr, unsigned long long* fcnt = nullptr) {
+                            uint32_t theta, Acc& acc) {
     __shared__ uint32_t s_off[kWarps][33];
     __shared__ uint32_t s_beg[kWarps][32], s_x[kWarps][32], s_v[kWarps][32];
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
@@ -838,7 +809,7 @@ __device__ void walk_sparse(const KParams& P, const uint32_t* off, const uint32_
                 acc.entries++;
                 acc.edges++;
                 if (cand > theta) {  // beyond the bucket: not committed, the predecessor stays signalled
-                    acc.sig += signal_append(P, bnxt, fl, fcnt, pred);
+                    acc.sig += signal_vertex(bnxt, pred);
                     break;
                 }
                 if (!last) {  // prefetch the path's next entry
@@ -851,7 +822,7 @@ __device__ void walk_sparse(const KParams& P, const uint32_t* off, const uint32_
                 const uint32_t old = atomicMin(&P.vs_u[u], cand);
                 if (cand >= old) break;
                 acc.upd++;
-                acc.sig += signal_append(P, bnxt, fl, fcnt, u);
+                acc.sig += signal_vertex(bnxt, u);
                 acc.vmin = min(acc.vmin, cand);
                 if (last) break;
                 cur = cand;
@@ -1536,15 +1507,7 @@ __global__ void __launch_bounds__(NW * 32, MINB) path_kernel(KParams P) {
     int r = 0, since = 0;
     unsigned long long ex = 0;
     __shared__ unsigned s_queue[2];
-    // SSSP/BFS frontier lists: a sparse round appends every vertex it signals
-    // first to the next round's list, so that round needs neither the count
-    // and compaction passes over the bitmap (nor their grid barriers) nor a
-    // full pass to retire its bitmap (DESIGN.md sec. 4 "Frontier lists")
-    constexpr bool kList = (ALGO == DG_SSSP || ALGO == DG_BFS) && !MR;
-    bool list_ready = false;  // the current bitmap's vertices are exactly the list's (uniform over threads)
     for (; r < P.max_rounds; r++) {
-        bool use_list = false;
-        unsigned lqn = 0;
         const int round = P.ctr->round + r;  // ctr->round only changes after the loop
         const int cur = round & 1, nxt = cur ^ 1;
         // this round's partition queues (per CTA, with stealing; or the global ticket)
@@ -1601,32 +1564,19 @@ __global__ void __launch_bounds__(NW * 32, MINB) path_kernel(KParams P) {
             // sparse round: when few vertices are
             // signalled, compact them; walk from them if their out-edges are
             // at most 1/sparse_div of the path entries, else walk the windows
-            const bool lists = kList && P.flist0 != nullptr;
-            uint2* lcur = lists ? (cur ? P.flist1 : P.flist0) : nullptr;
-            uint2* lnxt = lists ? (cur ? P.flist0 : P.flist1) : nullptr;
-            uint32_t losum = 0;
-            if (lists && list_ready) {  // the sparse test from the list's counts: no pass over the bitmap
-                const unsigned long long lc = *((volatile unsigned long long*)&P.ctr->fl_cnt[cur]);
-                lqn = (unsigned)lc;
-                losum = (uint32_t)(lc >> 32);
-                use_list = *((volatile unsigned*)&P.ctr->active[cur]) <= P.sparse_max && losum <= P.sparse_occ;
-            }
-            const bool sparse = use_list || ((ALGO == DG_SSSP || ALGO == DG_BFS || ALGO == 100) &&
-                                             !(lists && list_ready) && sparse_round(P, grid, cur, bcur));
+            const bool sparse = (ALGO == DG_SSSP || ALGO == DG_BFS || ALGO == 100) && sparse_round(P, grid, cur, bcur);
             // probe-free dense round: most vertices signalled, or the signalled
-            // ones own most out-edges (counted by sparse_round or the list)
+            // ones own most out-edges (counted by sparse_round)
             const unsigned nact = *((volatile unsigned*)&P.ctr->active[cur]);
-            const uint32_t osum_known = (lists && list_ready) ? losum : *((volatile unsigned*)&P.ctr->osum[cur]);
             const bool all = P.probe_free_occ &&
                              (nact > P.probe_free_act ||
                               (P.occ_off && (ALGO == DG_SSSP || ALGO == DG_BFS || ALGO == 100) &&
-                               osum_known >= P.probe_free_occ));
+                               *((volatile unsigned*)&P.ctr->osum[cur]) >= P.probe_free_occ));
             if (sparse) {
                 dense = false;
-                const unsigned qn = use_list ? lqn : *((volatile unsigned*)&P.ctr->qcur[cur]);
-                const uint2* items = use_list ? lcur : P.occ_items;
-                if (ALGO == DG_SSSP) walk_sparse<0>(P, P.occ_off, P.occ, items, qn, ticket, bnxt, theta, acc, lnxt, &P.ctr->fl_cnt[nxt]);
-                else if (ALGO == DG_BFS) walk_sparse<1>(P, P.occ_off, P.occ, items, qn, ticket, bnxt, theta, acc, lnxt, &P.ctr->fl_cnt[nxt]);
+                const unsigned qn = *((volatile unsigned*)&P.ctr->qcur[cur]);
+                if (ALGO == DG_SSSP) walk_sparse<0>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
+                else if (ALGO == DG_BFS) walk_sparse<1>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
                 else walk_sparse<3>(P, P.occ_off, P.occ, P.occ_items, qn, ticket, bnxt, theta, acc);
             } else if (ALGO == DG_SSSP) walk_minplus<0>(P, dq, bcur, bnxt, theta, acc, all);
             else if (ALGO == DG_BFS) walk_minplus<1>(P, dq, bcur, bnxt, theta, acc, all);
@@ -1687,21 +1637,10 @@ __global__ void __launch_bounds__(NW * 32, MINB) path_kernel(KParams P) {
         if (P.qtick && threadIdx.x == 0) P.qtick[((size_t)cur * gridDim.x + blockIdx.x) * kQStride] = 0u;
         if (!kAccum) {  // retire this round's bitmap for reuse two rounds later
             uint32_t* bc = P.bits + (int64_t)cur * P.nw;
-            if (kList && use_list) {  // its set bits are exactly the list's vertices
-                const uint2* lc = cur ? P.flist1 : P.flist0;
-                for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < lqn;
-                     i += (int64_t)gridDim.x * blockDim.x) {
-                    const uint2 it = lc[i];
-                    if (it.y == 0) bc[it.x >> 5] = 0u;
-                }
-            } else {
-                for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.nw;
-                     i += (int64_t)gridDim.x * blockDim.x)
-                    bc[i] = 0u;
-            }
+            for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < P.nw;
+                 i += (int64_t)gridDim.x * blockDim.x)
+                bc[i] = 0u;
         }
-        // the next round's bitmap was filled by a sparse SSSP/BFS walk only: its list is complete
-        list_ready = kList && P.flist0 != nullptr && !dense;
         if (blockIdx.x == 0 && threadIdx.x == 0) {
             if (P.trace && r < P.trace_cap) {  // developer trace (DG_TRACE)
                 unsigned long long t;
@@ -1723,7 +1662,6 @@ __global__ void __launch_bounds__(NW * 32, MINB) path_kernel(KParams P) {
             P.ctr->osum[cur] = 0;
             P.ctr->qcur[cur] = 0;
             P.ctr->qn_in[cur] = P.ctr->osum_in[cur] = P.ctr->qcur_in[cur] = P.ctr->ticket_in[cur] = 0;
-            P.ctr->fl_cnt[cur] = 0ull;  // this round consumed (or ignored) list cur
         }
         grid.sync();
         if (multi && (++since >= P.mr.every || *((volatile unsigned*)&P.ctr->active[nxt]) == 0)) {
@@ -2538,15 +2476,6 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
             P.occ_off = in ? W->iocc_off : W->occ_off;
             P.occ = in ? W->iocc : W->occ;
             P.occ_items = W->occ_items;
-            const char* fle = std::getenv("DG_FLIST");  // developer knob: 0 = no frontier lists
-            if ((algo_k == DG_SSSP || algo_k == DG_BFS) && !mr && !(fle && std::atoi(fle) == 0)) {
-                const size_t cap = (size_t)(D.n + D.m / kOccChunk + 1);  // >= sum over vertices of max(1, ceil(d/32))
-                int64_t bytes = 0;
-                for (int k = 0; k < 2; k++)
-                    if (!W->flist[k] && (rc = dalloc(&W->flist[k], cap, bytes, err))) return rc;
-                P.flist0 = W->flist[0];
-                P.flist1 = W->flist[1];
-            }
             P.sparse_max = (uint32_t)std::min<int64_t>(D.n / 4, 0xFFFFFFFFll);
             P.sparse_occ = (uint32_t)std::min<int64_t>(D.M / sd, 0xFFFFFFFFll);
             const char* sw = std::getenv("DG_SPARSE_WALK");  // developer knob
@@ -2896,7 +2825,7 @@ void dev_free_work(DevWork*& W) {
     if (W->ctr_host) cudaFreeHost(W->ctr_host);
     W->ctr_host = W->ctr_host_dev = nullptr;
     dfree(W->ctr); dfree(W->dsum); dfree(W->qtick); dfree(W->scc_label); dfree(W->scc_mark); dfree(W->remaining); dfree(W->out_stage);
-    dfree(W->occ_off); dfree(W->occ); dfree(W->occ_items); dfree(W->flist[0]); dfree(W->flist[1]); dfree(W->iocc_off); dfree(W->iocc); dfree(W->occ_cur);
+    dfree(W->occ_off); dfree(W->occ); dfree(W->occ_items); dfree(W->iocc_off); dfree(W->iocc); dfree(W->occ_cur);
     if (W->cub_tmp) cudaFree(W->cub_tmp);
     if (W->ev0) cudaEventDestroy(W->ev0);
     if (W->ev1) cudaEventDestroy(W->ev1);
