@@ -4,7 +4,7 @@ time each algorithm to convergence (3 timed runs after 2 warm-ups), and one
 vertex-centric ablation run for SSSP / BFS / PageRank / WCC (vertex updates next to
 the path kernel's).  Prints one JSON object.
 
-  python scripts/big_run.py <config> <algo,algo,...> [--no-ablation]
+  python scripts/big_run.py <config> <algo,algo,...> [--no-ablation | --ablation=algo,algo]
 """
 import json, os, resource, sys, time
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -15,6 +15,7 @@ from paper_conf_asplos_zhangl0hlg19_b200 import DiGraph
 cfg = sys.argv[1] if len(sys.argv) > 1 else "twitter"
 algos = sys.argv[2].split(",") if len(sys.argv) > 2 else ["pagerank", "sssp", "wcc"]
 ablation = "--no-ablation" not in sys.argv
+abl_only = next((a.split("=", 1)[1].split(",") for a in sys.argv if a.startswith("--ablation=")), None)
 res = {"config": cfg}
 t = time.time(); g = inputs.make(cfg); res["gen_s"] = time.time() - t; res["n"] = g.n; res["m"] = g.m
 print(f"[big] generated {g.name} in {res['gen_s']:.1f}s", file=sys.stderr, flush=True)
@@ -40,7 +41,7 @@ for algo in algos:
                  "vertex_updates": st["vertex_updates"], "entries_processed": st["entries_processed"],
                  "kernel_ms": st["kernel_ms"]}
     print(f"[big] {algo}: {res[algo]}", file=sys.stderr, flush=True)
-    if ablation and algo in ("pagerank", "sssp", "bfs", "wcc"):
+    if ablation and algo in ("pagerank", "sssp", "bfs", "wcc") and (abl_only is None or algo in abl_only):
         st = dg.run(algo, source=0, mode="vertex")
         res[algo]["ablation_vertex_centric"] = {"ms": st["time_ms"], "rounds": st["rounds"],
                                                 "vertex_updates": st["vertex_updates"],
