@@ -147,6 +147,9 @@ def algorithmic_bytes(algo, st, n, M):
     return 4 * M * Rd + per * E + 8 * U + n * R // 4
 
 
+L2_MIX_CEILING = 145e9  # random 8-byte gather/RED mix over an L2-resident array (r02d ubench: 142-149 G ops/s)
+
+
 def load_peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     try:
@@ -196,9 +199,14 @@ def roofline(algo, config, st, n, M, mode, hub_frac=None):
     if algo in ("pagerank", "adsorption") and hub_frac is not None:
         ops *= 1.0 - hub_frac
         roof["hub_entry_share"] = hub_frac
-    roof["l2_random_ops_per_s"] = ops / (kms / 1e3) if kms > 0 else 0.0
-    roof["l2_mix_ceiling_ops_per_s"] = 145e9
-    roof["l2_mix_ceiling_source"] = "scripts/ubench_l2_random.cu, profiles/r02d_l2_random_ubench.txt (gather/RED mix)"
+    rate = ops / (kms / 1e3) if kms > 0 else 0.0
+    roof["l2_random_ops_per_s"] = rate
+    # the resource that binds the walks (DESIGN.md sec. 4 "Bound"): random
+    # master operations against the measured L2 gather/RED-mix ceiling
+    roof["l2_random"] = {"achieved": rate, "peak": L2_MIX_CEILING, "unit": "ops/s", "frac": rate / L2_MIX_CEILING,
+                         "ops_per_launch": ops,
+                         "peak_source": "measured: scripts/ubench_l2_random.cu, profiles/r02d_l2_random_ubench.txt "
+                                        "(8-byte gathers and 64-bit REDs, even mix, L2-resident array)"}
     return roof
 
 

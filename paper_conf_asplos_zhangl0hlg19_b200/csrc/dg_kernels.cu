@@ -103,6 +103,8 @@ struct DevWork {
     uint8_t* scc_mark = nullptr;
     int32_t* remaining = nullptr;
     uint32_t* out_stage = nullptr;         // dg_get_states staging buffer (n words)
+    void* host_stage = nullptr;            // dg_get_states pinned host staging (n words)
+    int64_t host_stage_n = 0;
     unsigned* qtick = nullptr;             // per-CTA partition queue counters (2 x kMaxGrid x kQStride)
     uint32_t* occ_off = nullptr;           // vertex -> its non-tail path entries (sparse rounds), n+1
     uint32_t* occ = nullptr;               // entry indices grouped by vertex
@@ -408,10 +410,17 @@ __device__ __forceinline__ Win win_next(const KParams& P, const Win& w, const Qu
 // partition are fetched one partition early, so a partition switch waits for
 // no atomic or load.  With per-CTA queues (DG_DISPATCH=1) the switch takes
 // the next partition synchronously.
+// With the global ticket the first two partitions of every warp are static
+// (warp g of Gw takes ranks g and g + Gw) and the ticket hands out ranks from
+// 2 Gw on, so a round starts with two independent bound loads instead of two
+// dependent atomic + load round trips per warp (the stall at the start of
+// every round of a small graph, profiles/r02h_sssp_rmat16.md).
 struct Feed {
-    unsigned t_pend;     // lane 0: ticket taken for the partition after next
+    unsigned t_pend;     // lane 0: rank of the partition after next (a ticket + 2 Gw, or static)
     uint32_t nbeg, nend; // bounds of the next partition (nbeg == kNoWin: none)
 };
+__device__ __forceinline__ unsigned feed_warps() { return gridDim.x * (blockDim.x >> 5); }
+__device__ __forceinline__ unsigned feed_warp() { return blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); }
 __device__ __forceinline__ unsigned map_order(const KParams& P, unsigned t) {
     if (P.part_order == 1) return (unsigned)P.n_part - 1 - t;  // developer knob: dispatch-order experiments
     if (P.part_order > 1) return (unsigned)(((unsigned long long)t * P.part_order) % (unsigned long long)P.n_part);
@@ -428,7 +437,22 @@ __device__ __forceinline__ void feed_fetch(const KParams& P, const Queue& q, Fee
         f.nbeg = kNoWin;
         f.nend = 0;
     }
-    if ((threadIdx.x & 31) == 0) f.t_pend = atomicAdd(q.global, 1u);
+    if ((threadIdx.x & 31) == 0) f.t_pend = 2u * feed_warps() + atomicAdd(q.global, 1u);
+}
+// The warp's first window of a round and the primed feed (global ticket), or
+// the first window from its queue (per-CTA queues)
+__device__ __forceinline__ Win feed_start(const KParams& P, const Queue& q, Feed& f) {
+    if (q.qt) return win_first_of(P, q);
+    const unsigned g = feed_warp(), t0 = g;
+    Win w{kNoWin, 0, 0};
+    if (t0 < (unsigned)P.n_part) {
+        const unsigned u = map_order(P, t0);
+        const uint32_t beg = (uint32_t)P.part_off[u], end = (uint32_t)P.part_off[u + 1];
+        w = Win{beg & ~3u, beg, end};
+    }
+    f.t_pend = g + feed_warps();  // static second partition
+    feed_fetch(P, q, f);          // its bounds in flight; the first ticket taken
+    return w;
 }
 __device__ __forceinline__ Win feed_next(const KParams& P, const Queue& q, const Win& w, Feed& f) {
     if (w.base == kNoWin) return w;
@@ -500,12 +524,8 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
 
     // pipeline: indices three windows ahead, bitmap words two ahead, masters one ahead
     Feed f{0u, kNoWin, 0u};
-    Win wc = win_first_of(P, ticket);
+    Win wc = feed_start(P, ticket, f);
     if (wc.base == kNoWin) return;
-    if (!ticket.qt) {  // prime the feed: next partition's bounds and the ticket after it
-        if (lane == 0) f.t_pend = atomicAdd(ticket.global, 1u);
-        feed_fetch(P, ticket, f);
-    }
     Win wn = feed_next(P, ticket, wc, f);
     Win wn2 = feed_next(P, ticket, wn, f);
     uint4 code_c = load_code(wc), code_n = load_code(wn), code_n2 = load_code(wn2);
@@ -1027,12 +1047,8 @@ __device__ void walk_accum(const KParams& P, const Queue& q, Acc& acc, unsigned 
     };
 
     Feed f{0u, kNoWin, 0u};
-    Win w0 = win_first_of(P, q);
+    Win w0 = feed_start(P, q, f);
     if (w0.base == kNoWin) return;
-    if (!q.qt) {  // prime the feed: next partition's bounds and the ticket after it
-        if (lane == 0) f.t_pend = atomicAdd(q.global, 1u);
-        feed_fetch(P, q, f);
-    }
     Win w1 = feed_next(P, q, w0, f);
     Win w2 = feed_next(P, q, w1, f);
     uint4 c0 = load_code(w0), c1 = load_code(w1), c2 = load_code(w2);
@@ -2824,6 +2840,9 @@ void dev_free_work(DevWork*& W) {
     dfree(W->e_coef); dfree(W->pr_coef); dfree(W->ads_base); dfree(W->bits); dfree(W->vlist[0]); dfree(W->vlist[1]);
     if (W->ctr_host) cudaFreeHost(W->ctr_host);
     W->ctr_host = W->ctr_host_dev = nullptr;
+    if (W->host_stage) cudaFreeHost(W->host_stage);
+    W->host_stage = nullptr;
+    W->host_stage_n = 0;
     dfree(W->ctr); dfree(W->dsum); dfree(W->qtick); dfree(W->scc_label); dfree(W->scc_mark); dfree(W->remaining); dfree(W->out_stage);
     dfree(W->occ_off); dfree(W->occ); dfree(W->occ_items); dfree(W->iocc_off); dfree(W->iocc); dfree(W->occ_cur);
     if (W->cub_tmp) cudaFree(W->cub_tmp);
@@ -3261,8 +3280,32 @@ int dev_get_states(DevWork* W, const DevLayout& D, const RunState& S, void* out,
     }
     CK(cudaGetLastError());
     if (tmp) {
-        cudaError_t e = cudaMemcpy(out, tmp, 4 * (size_t)n, cudaMemcpyDeviceToHost);
-        if (e != cudaSuccess) { err = cudaGetErrorString(e); return DG_ENOCUDA; }
+        // D2H into a pinned staging buffer at full link speed, then a parallel
+        // host copy into the caller's (pageable) buffer: a copy straight into
+        // pageable memory runs at a fraction of the link (166 MB in 37 ms for
+        // the Twitter-shaped graph)
+        if (W->host_stage_n < n) {
+            if (W->host_stage) cudaFreeHost(W->host_stage);
+            W->host_stage = nullptr;
+            W->host_stage_n = 0;
+            if (cudaHostAlloc(&W->host_stage, 4 * (size_t)std::max<int64_t>(n, 1), cudaHostAllocDefault) == cudaSuccess)
+                W->host_stage_n = n;
+            else
+                cudaGetLastError();
+        }
+        if (W->host_stage) {
+            cudaError_t e = cudaMemcpy(W->host_stage, tmp, 4 * (size_t)n, cudaMemcpyDeviceToHost);
+            if (e != cudaSuccess) { err = cudaGetErrorString(e); return DG_ENOCUDA; }
+            const int64_t chunk = 1 << 20;
+#pragma omp parallel for schedule(static)
+            for (int64_t b = 0; b < (n + chunk - 1) / chunk; b++) {
+                const int64_t lo = b * chunk, hi = std::min<int64_t>(n, lo + chunk);
+                std::memcpy((uint32_t*)out + lo, (const uint32_t*)W->host_stage + lo, 4 * (size_t)(hi - lo));
+            }
+        } else {  // no pinned memory available: direct copy
+            cudaError_t e = cudaMemcpy(out, tmp, 4 * (size_t)n, cudaMemcpyDeviceToHost);
+            if (e != cudaSuccess) { err = cudaGetErrorString(e); return DG_ENOCUDA; }
+        }
     } else {
         CK(cudaDeviceSynchronize());
     }
