@@ -235,3 +235,34 @@ def test_edge_cases_in_sparse_rounds(sparse_div):
         assert np.array_equal(dg.get_states().astype(np.int64), OA.wcc_label_propagation(n, src, dst)[0])
         dg.run("pagerank")
         assert np.abs(dg.get_states() - OA.pagerank_power(n, src, dst)[0]).sum() <= 1e-4
+
+
+@pytest.fixture(params=["0", "1"])
+def probe_free(request):
+    """DG_PROBE_FREE=0 probes the signal bitmap in every dense min-plus round;
+    1 (the default) walks every window without probing when most vertices are
+    signalled (DESIGN.md sec. 4 "Probe-free dense min-plus rounds")."""
+    old = os.environ.get("DG_PROBE_FREE")
+    os.environ["DG_PROBE_FREE"] = request.param
+    yield request.param
+    if old is None:
+        os.environ.pop("DG_PROBE_FREE", None)
+    else:
+        os.environ["DG_PROBE_FREE"] = old
+
+
+def test_min_plus_exact_with_and_without_probing(probe_free):
+    # large enough (> 2^23 path entries) that sparse rounds, probing dense
+    # rounds and probe-free dense rounds all occur in one SSSP run
+    g = inputs.rmat(19, 1 << 19, 9_000_000, seed=5, oversample=1.15)
+    src, dst, w = g.edges()
+    dg = DiGraph()
+    dg.load_graph(g)
+    dg.build_paths()
+    st = dg.run("sssp", source=0)
+    assert st["dense_rounds"] >= 1 and st["rounds"] > st["dense_rounds"]
+    assert np.array_equal(dg.get_states().astype(np.int64), OA.sssp_bellman_ford(g.n, src, dst, w, 0)[0])
+    dg.run("bfs", source=0)
+    assert np.array_equal(dg.get_states().astype(np.int64), OA.bfs_levels(g.n, src, dst, 0))
+    dg.run("wcc")
+    assert np.array_equal(dg.get_states().astype(np.int64), OA.wcc_label_propagation(g.n, src, dst)[0])
