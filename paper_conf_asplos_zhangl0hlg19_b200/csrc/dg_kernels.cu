@@ -2286,7 +2286,7 @@ int write_counters(DevWork* W, const Counters& c, std::string& err, RunState* S 
 }
 
 int coop_launch(DevWork* W, void* fn, KParams& P, RunState& S, std::string& err, size_t smem = 0,
-                int threads = kBlock) {
+                int threads = kBlock, int max_per_sm = 0) {
     // grid size per (device, kernel, block, shared memory), queried once:
     // the occupancy query and the attribute call cost tens of microseconds,
     // which small graphs (configs[0]: ~0.3 ms per run) would pay every run
@@ -2316,6 +2316,11 @@ int coop_launch(DevWork* W, void* fn, KParams& P, RunState& S, std::string& err,
             it = grids.emplace(key, std::min(sms * std::max(1, per), kMaxGrid)).first;
         }
         grid = it->second;
+        if (max_per_sm > 0) {  // fewer resident CTAs than the occupancy allows (small graphs)
+            int sms = 0;
+            CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+            grid = std::min(grid, sms * max_per_sm);
+        }
     }
     if (P.qtick) CK(cudaMemsetAsync(P.qtick, 0, sizeof(unsigned) * 2 * kMaxGrid * kQStride));
     void* args[] = {&P};
@@ -2528,7 +2533,9 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
     }
     P.ctr_out = mr ? nullptr : W->ctr_host_dev;
     W->ctr_mirror_fresh = false;
-    int rc = coop_launch(W, fn, P, S, err, smem, accum ? kAccWarps * 32 : kBlock);
+    int per_sm = 0;
+    if (const char* ce = std::getenv("DG_MP_CTAS")) per_sm = std::atoi(ce);  // developer knob: min-plus CTAs per SM
+    int rc = coop_launch(W, fn, P, S, err, smem, accum ? kAccWarps * 32 : kBlock, accum ? 0 : per_sm);
     if (!rc && P.ctr_out) W->ctr_mirror_fresh = true;
     if (P.snap) cudaFree(P.snap);
     if (trace) {
