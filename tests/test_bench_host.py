@@ -47,6 +47,7 @@ def test_roofline_fields_and_hub_share(bench):
     # min-plus walks have no proxies: every gather/atomicMin counts
     r2 = bench.roofline("sssp", "nonexistent", st, 100, 1000, "path", hub_frac=0.25)
     assert r2["l2_random"]["ops_per_launch"] == 16_000
+    assert r2["l2_random"]["peak"] == bench.L2_GATHER_CEILING
 
 
 def test_hub_entries_counts_the_proxied_vertices():
