@@ -2533,7 +2533,10 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
     }
     P.ctr_out = mr ? nullptr : W->ctr_host_dev;
     W->ctr_mirror_fresh = false;
-    int per_sm = 0;
+    // min-plus walks of small graphs (< 2^21 path entries) run 2 CTAs per SM
+    // instead of 3: the per-round grid barriers and dispatch are cheaper and
+    // the fewer warps still cover the windows (R-MAT-16 SSSP)
+    int per_sm = D.M < ((int64_t)1 << 21) ? 2 : 0;
     if (const char* ce = std::getenv("DG_MP_CTAS")) per_sm = std::atoi(ce);  // developer knob: min-plus CTAs per SM
     int rc = coop_launch(W, fn, P, S, err, smem, accum ? kAccWarps * 32 : kBlock, accum ? 0 : per_sm);
     if (!rc && P.ctr_out) W->ctr_mirror_fresh = true;
