@@ -67,7 +67,7 @@ typedef struct {
     int32_t order;         /* successor/root order: 0 = degree desc (line 5), 1 = vertex id */
     float hot_factor;      /* hot path iff avg degree >= hot_factor * mean degree (R-HOT) */
     int32_t part_entries;  /* target path entries per partition (scheduling unit); 0 = auto
-                              (about 16K partitions, 128..2048 entries each) */
+                              (about 16K partitions, 512..2048 entries each) */
     int32_t rank;          /* this process's rank for multi-GPU path partitioning */
     int32_t world;         /* number of ranks (1 = single GPU) */
     int32_t merge_rule;    /* 0: paper-literal (no merge through a line-13 inner vertex of
