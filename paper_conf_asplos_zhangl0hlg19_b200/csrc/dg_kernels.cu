@@ -2503,8 +2503,10 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
             P.sparse_walk = sw ? std::max(1, std::atoi(sw)) : 4;
         }
         {
-            const char* pf = std::getenv("DG_PROBE_FREE");  // developer knob: 0 = always probe
-            P.probe_free_occ = (pf && std::atoi(pf) == 0) ? 0u : (uint32_t)std::min<int64_t>(std::max<int64_t>(D.M / 4, 1), 0xFFFFFFFFll);
+            const char* pf = std::getenv("DG_PROBE_FREE");  // developer knob: 0 = always probe, k > 1: out-edge share M/k
+            int64_t pdiv = pf ? std::atoll(pf) : 4;
+            if (pdiv == 1) pdiv = 4;  // 1: on, with the default share
+            P.probe_free_occ = pdiv == 0 ? 0u : (uint32_t)std::min<int64_t>(std::max<int64_t>(D.M / std::max<int64_t>(pdiv, 1), 1), 0xFFFFFFFFll);
             P.probe_free_act = (uint32_t)std::min<int64_t>(D.n / 4, 0xFFFFFFFFll);
         }
         const char* hm = std::getenv("DG_HOT_MASTER_MB");  // developer knob (default 64 MB)
