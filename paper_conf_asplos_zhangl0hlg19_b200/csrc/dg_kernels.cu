@@ -2140,7 +2140,7 @@ __global__ void p2p_signal_wait_kernel(PeerSlots flags, int world, int rank, uns
             if (v >= epoch) break;
             asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
             if (t - t0 > timeout_ns) {  // a peer never arrived: report instead of hanging the GPU
-                atomicExch(own_flags + kP2PMaxRanks, 1ull);
+                atomicExch(own_flags + kP2PErr, 1ull);
                 break;
             }
             __nanosleep(256);
@@ -3228,7 +3228,7 @@ int dev_boundary_exchange(DevWork* W, const DevLayout& D, RunState& S, P2P* X, i
     S.stats.kernel_launches += D.n_bnd ? 3 : 1;
     CK(cudaGetLastError());
     unsigned long long timed_out = 0;
-    CK(cudaMemcpy(&timed_out, own_flags + kP2PMaxRanks, sizeof(timed_out), cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(&timed_out, own_flags + kP2PErr, sizeof(timed_out), cudaMemcpyDeviceToHost));
     if (timed_out) { err = "dg_boundary_exchange: a peer did not arrive within 60 s"; return DG_ETIMEOUT; }
     if ((rc = read_counters(W, c, err))) return rc;
     *active = c.active[slot];
