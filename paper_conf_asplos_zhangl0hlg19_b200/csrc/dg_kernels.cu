@@ -111,6 +111,8 @@ struct DevWork {
     uint32_t* occ_off = nullptr;           // vertex -> its non-tail path entries (sparse rounds), n+1
     uint32_t* occ = nullptr;               // entry indices grouped by vertex
     uint2* occ_items = nullptr;            // frontier items (v, chunk of <= kOccChunk occurrences)
+    uint2* e_cw = nullptr;                 // SSSP sparse rounds: {e_idx, e_w} interleaved (one load per step)
+    bool cw_ok = false;
     uint32_t* iocc_off = nullptr;          // vertex -> its non-head path entries (SCC backward), n+1
     uint32_t* iocc = nullptr;
     bool iocc_ok = false;
@@ -176,6 +178,7 @@ struct KParams {
     const uint32_t* occ_off;  // SSSP/BFS sparse rounds: occurrence index (null: dense rounds only)
     const uint32_t* occ;
     uint2* occ_items;         // the round's frontier items (v, chunk)
+    const uint2* e_cw;        // SSSP sparse walk: path entry code and weight in one 8-byte word (null: separate)
     const uint32_t* iocc_off;  // WCC: the in-edge occurrence index as well
     const uint32_t* iocc;
     uint32_t sparse_max;      // rounds with at most this many signalled vertices are candidates (n/4)
@@ -821,8 +824,15 @@ __device__ void walk_sparse(const KParams& P, const uint32_t* off, const uint32_
             uint32_t cur = s_x[wid][lo], pred = s_v[wid][lo];
             uint32_t e = occ[s_beg[wid][lo] + (j - s_off[wid][lo])] + 1;  // the path edge out of the occurrence
             // the next entry of the path is loaded one step ahead
-            uint32_t code = __ldg(P.e_idx + e);
-            uint32_t w = MODE == 0 ? (uint32_t)__ldg(P.e_w + e) : (MODE == 1 ? 1u : 0u);
+            uint32_t code, w;
+            if (MODE == 0 && P.e_cw) {  // one random 8-byte load per step instead of two 4-byte ones
+                const uint2 cw = __ldg(P.e_cw + e);
+                code = cw.x;
+                w = cw.y;
+            } else {
+                code = __ldg(P.e_idx + e);
+                w = MODE == 0 ? (uint32_t)__ldg(P.e_w + e) : (MODE == 1 ? 1u : 0u);
+            }
             for (int step = 0; step < P.sparse_walk; step++) {
                 const uint32_t u = code & kVMask;
                 if (MODE == 3 && P.scc_label[u] >= 0) break;  // assigned vertices break their paths
@@ -835,8 +845,14 @@ __device__ void walk_sparse(const KParams& P, const uint32_t* off, const uint32_
                     break;
                 }
                 if (!last) {  // prefetch the path's next entry
-                    code = __ldg(P.e_idx + e + 1);
-                    if (MODE == 0) w = (uint32_t)__ldg(P.e_w + e + 1);
+                    if (MODE == 0 && P.e_cw) {
+                        const uint2 cw = __ldg(P.e_cw + e + 1);
+                        code = cw.x;
+                        w = cw.y;
+                    } else {
+                        code = __ldg(P.e_idx + e + 1);
+                        if (MODE == 0) w = (uint32_t)__ldg(P.e_w + e + 1);
+                    }
                 }
                 // read before the atomic: in-edges of hubs would otherwise
                 // serialise on one address
@@ -1835,6 +1851,11 @@ __global__ void init_u_kernel(uint32_t* vs, uint32_t* stamp, const int32_t* orig
         stamp[v] = 0u;
     }
 }
+// SSSP sparse walks: each path entry's code and the weight of the path edge
+// into it side by side, so a walk step is one random 8-byte load
+__global__ void cw_build_kernel(uint2* cw, const uint32_t* e_idx, const int32_t* e_w, int64_t n) {
+    GRID_STRIDE(i, n) cw[i] = make_uint2(e_idx[i], (uint32_t)e_w[i]);
+}
 // path-mode SSSP/BFS start state in one launch: distances (source 0),
 // bitmaps zeroed except the source's bit in bitmap 0, the run's counters
 __global__ void init_minplus_kernel(uint32_t* vs, uint32_t* stamp, int64_t n, int64_t source, uint32_t* bits,
@@ -2516,6 +2537,18 @@ int launch_path(DevWork* W, const DevLayout& D, int algo_k, int rounds, RunState
             P.occ_off = in ? W->iocc_off : W->occ_off;
             P.occ = in ? W->iocc : W->occ;
             P.occ_items = W->occ_items;
+            const char* cwe = std::getenv("DG_SPARSE_CW");  // developer knob: 0 = separate e_idx / e_w loads
+            if (algo_k == DG_SSSP && D.e_w && !(cwe && std::atoi(cwe) == 0)) {
+                if (!W->cw_ok) {
+                    int64_t bytes = 0;
+                    if (!W->e_cw && (rc = dalloc(&W->e_cw, (size_t)D.M + kPad, bytes, err))) return rc;
+                    cw_build_kernel<<<grid_1d(D.M + kPad), 256>>>(W->e_cw, D.e_idx, D.e_w, D.M + kPad);
+                    CK(cudaGetLastError());
+                    S.stats.kernel_launches++;
+                    W->cw_ok = true;
+                }
+                P.e_cw = W->e_cw;
+            }
             P.sparse_max = (uint32_t)std::min<int64_t>(D.n / 4, 0xFFFFFFFFll);
             P.sparse_occ = (uint32_t)std::min<int64_t>(D.M / sd, 0xFFFFFFFFll);
             const char* sw = std::getenv("DG_SPARSE_WALK");  // developer knob
@@ -2879,7 +2912,7 @@ void dev_free_work(DevWork*& W) {
     W->host_stage = nullptr;
     W->host_stage_n = 0;
     dfree(W->ctr); dfree(W->dsum); dfree(W->qtick); dfree(W->scc_label); dfree(W->scc_mark); dfree(W->remaining); dfree(W->out_stage);
-    dfree(W->occ_off); dfree(W->occ); dfree(W->occ_items); dfree(W->iocc_off); dfree(W->iocc); dfree(W->occ_cur);
+    dfree(W->occ_off); dfree(W->occ); dfree(W->occ_items); dfree(W->e_cw); dfree(W->iocc_off); dfree(W->iocc); dfree(W->occ_cur);
     if (W->cub_tmp) cudaFree(W->cub_tmp);
     if (W->ev0) cudaEventDestroy(W->ev0);
     if (W->ev1) cudaEventDestroy(W->ev1);
@@ -2893,6 +2926,7 @@ void dev_layout_changed(DevWork* W) {
     if (!W) return;
     W->pr_coef_d = -1.0;
     W->occ_ok = W->iocc_ok = false;  // rebuilt on next use (allocations kept: same n, M)
+    W->cw_ok = false;
 }
 
 int dev_set_vertex_params(DevWork*& W, const DevLayout& D, const double* p_inj, const double* p_cont,
