@@ -844,7 +844,13 @@ __device__ void walk_sparse(const KParams& P, const uint32_t* off, const uint32_
                     acc.sig += signal_vertex(bnxt, pred);
                     break;
                 }
-                if (!last) {  // prefetch the path's next entry
+                // when even a weight-1 relaxation after this entry would lie
+                // beyond the bucket, the walk ends here -- the vertex it lowers
+                // is signalled and relaxes its edges in a later round (no wasted
+                // load of the next entry, no redundant re-signal; a 0-weight
+                // continuation is merely deferred, which label correction allows)
+                const bool stop_next = (MODE == 0 || MODE == 1) && sat_add(cand, 1u) > theta;
+                if (!last && !stop_next) {  // prefetch the path's next entry
                     if (MODE == 0 && P.e_cw) {
                         const uint2 cw = __ldg(P.e_cw + e + 1);
                         code = cw.x;
@@ -862,7 +868,7 @@ __device__ void walk_sparse(const KParams& P, const uint32_t* off, const uint32_
                 acc.upd++;
                 acc.sig += signal_vertex(bnxt, u);
                 acc.vmin = min(acc.vmin, cand);
-                if (last) break;
+                if (last || stop_next) break;
                 cur = cand;
                 pred = u;
                 e++;
