@@ -18,7 +18,9 @@ cfg, algos, name, vals = sys.argv[1], sys.argv[2].split(","), sys.argv[3], sys.a
 g = inputs.make(cfg)
 dg = DiGraph().load_graph(g)
 del g
-dg.build_paths()
+# DG_BUILD_NPROXY: the layout's proxy count (default: the library's 8192)
+npx = os.environ.get("DG_BUILD_NPROXY")
+dg.build_paths(**({"n_proxy": int(npx)} if npx else {}))
 dg.upload()
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 first = {}
