@@ -271,3 +271,19 @@ def test_bad_layout_file_keeps_the_handle(tmp_path):
     with pytest.raises(DGError, match="DG_EINVAL"):
         dg.load_layout(str(p))
     assert dg.layout_info() == before
+
+
+def test_auto_partitions_hold_at_least_512_entries():
+    # part_entries = 0 (auto): about 16 K partitions of 512..2048 whole-path
+    # entries (DESIGN.md sec. 4 "Small graphs"); a partition may exceed the
+    # target only by the path that crosses it
+    for scale, m in ((12, 40_000), (16, 1 << 20)):
+        g = inputs.rmat(scale, 1 << scale, m, seed=4)
+        dg = DiGraph().load_graph(g).build_paths()
+        info = dg.layout_info()
+        part_off = dg.export_paths()["part_off"]
+        sizes = np.diff(part_off)
+        assert info["n_partitions"] == len(sizes)
+        # every partition but the last reaches the 512-entry target
+        assert sizes[:-1].min() >= 512
+        assert info["n_partitions"] <= info["n_entries"] // 512 + 1
