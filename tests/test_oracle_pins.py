@@ -383,6 +383,26 @@ def test_dependency_layers_are_longest_path_layers(seed):
         assert np.all(layer[scc == c] == lc)
         if lc > 0:
             assert any(scc[j] == c and scc[i] != c and layer[i] == lc - 1 for i, j in dep)
+    # independently: peel the condensation (built from the brute-force
+    # reachability) source layer by source layer (Kahn by rounds) -- round t
+    # removes exactly the SCCs whose longest chain of predecessors has t SCCs
+    comp = {}
+    for i in range(k):
+        comp.setdefault(frozenset(j for j in range(k) if R[i, j] and R[j, i]) | {i}, []).append(i)
+    cid = {i: c for c, members in enumerate(comp.values()) for i in members}
+    preds = {c: set() for c in range(len(comp))}
+    for i, j in brute:
+        if cid[i] != cid[j]:
+            preds[cid[j]].add(cid[i])
+    peel, left, t = {}, set(preds), 0
+    while left:
+        src_now = {c for c in left if not (preds[c] & left)}
+        assert src_now  # a DAG always has a source
+        for c in src_now:
+            peel[c] = t
+        left -= src_now
+        t += 1
+    assert all(layer[i] == peel[cid[i]] for i in range(k))
 
 
 def test_priority_orders_layers_first():
