@@ -421,3 +421,29 @@ def test_path_stats_on_figure4():
     assert np.allclose(dbar, [11 / 6, 13 / 5, 2.0, 2.5])
     assert nv.tolist() == [6, 5, 4, 4]
     assert hot.tolist() == [False, True, False, True]   # threshold 2.5
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_relaxed_merge_is_maximal(seed):
+    """Reading R-MERGE, relaxed rule, no length cap: the merge links pieces
+    at every vertex until one side runs out, so afterwards no vertex has
+    both a merged path that only ends there and one that only starts there;
+    paths that start and end at the same vertex (a closed piece, or a cycle
+    of links cut there -- the cut frees an end and a start of the same path)
+    are exempt.  A merge that skipped a possible link, or linked pieces that
+    do not meet, fails this or the cover check."""
+    n = 80
+    src, dst, _ = rand_graph(n, 400, 900 + seed, self_loops=False)
+    row_ptr, col, _, _ = to_csr(n, src, dst)
+    paths, inner = P.graphp_decompose(n, row_ptr, col, d_max=4)
+    merged = P.merge_short_paths(n, src, dst, paths, set(), l_max=1 << 30)
+    assert check_cover(n, src, dst, merged)
+    ends, starts = {}, {}
+    for i, p in enumerate(merged):
+        ends.setdefault(p[-1], set()).add(i)
+        starts.setdefault(p[0], set()).add(i)
+    for x in set(ends) & set(starts):
+        only_end, only_start = ends[x] - starts[x], starts[x] - ends[x]
+        assert not (only_end and only_start), (x, ends[x], starts[x])
+    # and the merge really merged: every piece boundary inside a merged path joins at one vertex
+    assert len(merged) < len(paths)
