@@ -583,7 +583,10 @@ __device__ void walk_minplus(const KParams& P, const Queue& ticket, const uint32
                 const uint32_t i = i0 + k;
                 const uint32_t c = u4get(code_c, k);
                 vtx[k] = c & kVMask;
-                live[k] = i >= wc.beg && i < wc.end && (MODE != 3 || P.scc_label[vtx[k]] < 0);
+                // SCC colouring: an assigned vertex holds INF (scc_init_kernel) and
+                // breaks its paths -- the gathered master says so without a
+                // second random load of its label
+                live[k] = i >= wc.beg && i < wc.end && (MODE != 3 || a_c[k] != INF);
                 hd[k] = !live[k] || (c & kHead);
                 tl[k] = !live[k] || (c & kTail);
                 wgt[k] = MODE == 0 ? (uint32_t)i4get(wv, k) : (MODE == 1 ? 1u : 0u);
@@ -835,7 +838,11 @@ __device__ void walk_sparse(const KParams& P, const uint32_t* off, const uint32_
             }
             for (int step = 0; step < P.sparse_walk; step++) {
                 const uint32_t u = code & kVMask;
-                if (MODE == 3 && P.scc_label[u] >= 0) break;  // assigned vertices break their paths
+                // the head's state, read once (before the atomic: in-edges of hubs
+                // would otherwise serialise on one address); SCC colouring: an
+                // assigned vertex holds INF and breaks its paths
+                const uint32_t cu = __ldcg(&P.vs_u[u]);
+                if (MODE == 3 && cu == INF) break;
                 const uint32_t cand = MODE == 3 ? cur : sat_add(cur, w);
                 const bool last = code & kTail;
                 acc.entries++;
@@ -860,9 +867,7 @@ __device__ void walk_sparse(const KParams& P, const uint32_t* off, const uint32_
                         if (MODE == 0) w = (uint32_t)__ldg(P.e_w + e + 1);
                     }
                 }
-                // read before the atomic: in-edges of hubs would otherwise
-                // serialise on one address
-                if (cand >= __ldcg(&P.vs_u[u])) break;
+                if (cand >= cu) break;
                 const uint32_t old = atomicMin(&P.vs_u[u], cand);
                 if (cand >= old) break;
                 acc.upd++;
