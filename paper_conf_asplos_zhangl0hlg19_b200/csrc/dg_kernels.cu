@@ -937,7 +937,7 @@ __device__ void walk_sparse_bwd(const KParams& P, const uint32_t* off, const uin
                     acc.upd++;
                     acc.sig += signal_vertex(bnxt, u);
                 } else {
-                    if (P.scc_label[u] >= 0 || P.vs_u[u] != c || P.mark[u]) break;
+                    if (P.vs_u[u] != c || P.mark[u]) break;  // assigned vertices hold INF != c
                     P.mark[u] = 1;  // idempotent byte store; the signal bit counts it once
                     if (signal_vertex(bnxt, u)) {
                         acc.upd++;
@@ -1343,9 +1343,12 @@ __device__ void walk_scc_bwd(const KParams& P, int64_t beg, int64_t end, const u
 #pragma unroll
         for (int k = 0; k < 4; k++) {
             const uint32_t c = u4get(code, k);
-            live[k] = valid[k] && P.scc_label[vtx[k]] < 0;
+            // an assigned vertex holds INF (scc_init_kernel): its colour says
+            // it breaks the path, without a load of its label
+            const uint32_t cv = valid[k] ? P.vs_u[vtx[k]] : INF;
+            live[k] = cv != INF;
             tl[k] = !live[k] || (c & kTail);
-            col[k] = live[k] ? P.vs_u[vtx[k]] : INF;
+            col[k] = cv;
             mk[k] = live[k] && P.mark[vtx[k]];
         }
         // element k on the successor's mark x:  m_k = mk_k | (x & eq_k),
